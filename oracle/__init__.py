@@ -1,0 +1,169 @@
+"""oracle -- TEST INFRASTRUCTURE ONLY.
+
+Plain, slow, obviously-correct CPU implementation of CUDAlign 2.0 Stage 1
+(Sandes & de Melo, IPDPS 2011; ``/root/reference/PAPER.md`` = ``P:<line>``):
+Smith-Waterman with Gotoh affine gaps (Eq. 1-3), best score and its
+end cell, special rows of H and F, and the anchored
+global reverse pass used to find the start cell.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
+``--impl reference`` legs may import this package.  It shares no code with
+the CUDA path (``paper_conf_ipps_sandesm11_b200``) and imports nothing from
+it; the only module both sides use is ``synth`` (seeded inputs, none of the
+method's arithmetic).
+
+Functions (all scores in the API convention: ``match``/``mismatch`` are added,
+``gap_open``/``gap_ext`` are non-negative penalties that are subtracted,
+G_first = gap_open + gap_ext, reading S2 in DESIGN.md):
+
+- ``stage1(A, B, ma, mi, go, ge, k=0)`` -> ``(score, i, j), rows``
+- ``full_matrix(A, B, ...)`` -> ``H, E, F`` (numpy int64, (m+1) x (n+1))
+- ``band(A, B, ..., r0, r1, Htop, Ftop)`` -> ``Hbot, Fbot, (score, i, j)``
+- ``global_score(A, B, ...)`` -> NW/Gotoh global score
+- ``reverse_goal(A, i_end, B, j_end, ..., goal)`` -> ``(goal, i_s, j_s)`` or None
+- ``flush_rows(m, n, alphaT, sra_bytes)`` -> special-row spacing
+
+Parity pins live in ``tests/test_oracle_pins.py``; every function above is
+pinned (none is "parity unpinned").
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "sw_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lock = threading.Lock()
+_lib = None
+
+NEG = -(1 << 40)  # the oracle's "minus infinity" (sw_oracle.c)
+
+
+class _Res(ctypes.Structure):
+    _fields_ = [("score", ctypes.c_int64), ("i", ctypes.c_int64), ("j", ctypes.c_int64)]
+
+
+_SINK = ctypes.CFUNCTYPE(
+    ctypes.c_int,
+    ctypes.c_void_p,
+    ctypes.c_int64,
+    ctypes.POINTER(ctypes.c_int64),
+    ctypes.POINTER(ctypes.c_int64),
+    ctypes.c_int64,
+)
+
+
+def build(force: bool = False) -> str:
+    """Compile sw_oracle.c with gcc (plain -O2, no vectorisation pragmas)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", tmp, _SRC])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    with _lock:
+        if _lib is None:
+            lib = ctypes.CDLL(build())
+            i64, cp, vp = ctypes.c_int64, ctypes.c_char_p, ctypes.c_void_p
+            p64 = ctypes.POINTER(ctypes.c_int64)
+            lib.or_stage1.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, _SINK, vp, ctypes.POINTER(_Res)]
+            lib.or_full_matrix.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, p64, p64, p64]
+            lib.or_band.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, i64, p64, p64, p64, p64, ctypes.POINTER(_Res)]
+            lib.or_global.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64]
+            lib.or_global.restype = i64
+            lib.or_reverse_goal.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, ctypes.POINTER(_Res)]
+            lib.or_flush_rows.argtypes = [i64, i64, i64, i64]
+            lib.or_flush_rows.restype = i64
+            _lib = lib
+    return _lib
+
+
+def _b(s) -> bytes:
+    if isinstance(s, np.ndarray):
+        return s.tobytes()
+    if isinstance(s, str):
+        return s.encode("ascii")
+    return bytes(s)
+
+
+def _p64(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+
+
+def stage1(A, B, ma, mi, go, ge, k=0, sink=None, keep_rows=True):
+    """Stage 1.  Returns ((score, i, j), rows) where rows is a list
+    of (i, H[1..n], F[1..n]) for every special row (if keep_rows), and calls
+    ``sink(i, H, F)`` (numpy int64 copies) for each if given."""
+    lib = _load()
+    a, b = _b(A), _b(B)
+    rows = []
+
+    def _cb(_user, row, H, F, n):
+        h = np.ctypeslib.as_array(H, shape=(n,)).copy()
+        f = np.ctypeslib.as_array(F, shape=(n,)).copy()
+        if keep_rows:
+            rows.append((int(row), h, f))
+        if sink is not None:
+            return int(bool(sink(int(row), h, f)))
+        return 0
+
+    cb = _SINK(_cb)
+    res = _Res()
+    rc = lib.or_stage1(a, len(a), b, len(b), ma, mi, go, ge, k, cb, None, ctypes.byref(res))
+    if rc != 0:
+        raise RuntimeError(f"or_stage1 failed rc={rc}")
+    return (res.score, res.i, res.j), rows
+
+
+def full_matrix(A, B, ma, mi, go, ge):
+    lib = _load()
+    a, b = _b(A), _b(B)
+    m, n = len(a), len(b)
+    H = np.zeros((m + 1, n + 1), np.int64)
+    E = np.zeros_like(H)
+    F = np.zeros_like(H)
+    lib.or_full_matrix(a, m, b, n, ma, mi, go, ge, _p64(H), _p64(E), _p64(F))
+    return H, E, F
+
+
+def band(A, B, ma, mi, go, ge, r0, r1, Htop, Ftop):
+    """Rows r0+1..r1 from row r0 (each length n+1, column 0 included)."""
+    lib = _load()
+    a, b = _b(A), _b(B)
+    n = len(b)
+    Ht = np.ascontiguousarray(Htop, dtype=np.int64)
+    Ft = np.ascontiguousarray(Ftop, dtype=np.int64)
+    assert Ht.shape == (n + 1,) and Ft.shape == (n + 1,)
+    Hb = np.zeros(n + 1, np.int64)
+    Fb = np.zeros(n + 1, np.int64)
+    res = _Res()
+    rc = lib.or_band(a, len(a), b, n, ma, mi, go, ge, r0, r1, _p64(Ht), _p64(Ft), _p64(Hb), _p64(Fb), ctypes.byref(res))
+    if rc != 0:
+        raise RuntimeError(f"or_band failed rc={rc}")
+    return Hb, Fb, (res.score, res.i, res.j)
+
+
+def global_score(A, B, ma, mi, go, ge) -> int:
+    lib = _load()
+    a, b = _b(A), _b(B)
+    return int(lib.or_global(a, len(a), b, len(b), ma, mi, go, ge))
+
+
+def reverse_goal(A, i_end, B, j_end, ma, mi, go, ge, goal):
+    lib = _load()
+    a, b = _b(A), _b(B)
+    res = _Res()
+    found = lib.or_reverse_goal(a, i_end, b, j_end, ma, mi, go, ge, goal, ctypes.byref(res))
+    return (res.score, res.i, res.j) if found else None
+
+
+def flush_rows(m, n, alphaT, sra_bytes) -> int:
+    return int(_load().or_flush_rows(m, n, alphaT, sra_bytes))

@@ -1,0 +1,289 @@
+/*
+ * oracle/sw_oracle.c -- TEST INFRASTRUCTURE ONLY.
+ *
+ * A plain, slow, obviously-correct, single-threaded CPU implementation of
+ * the computation CUDAlign 2.0's Stage 1 performs (Sandes & de Melo,
+ * IPDPS 2011; /root/reference/PAPER.md, cited below as P:<line>).
+ *
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+ * --impl reference legs may load this library.  The product path
+ * (paper_conf_ipps_sandesm11_b200/) never includes, links or calls it, and
+ * this file includes nothing from the product path.
+ *
+ * Notation follows the paper: S0 (length m, rows i) and S1 (length n,
+ * columns j); matrices H, E, F (Eq. 1-3); ma, mi
+ * the match / mismatch scores; G_first the first-gap penalty,
+ * G_ext the extension penalty, G_open = G_first - G_ext.
+ *
+ * Readings of the paper that this file takes:
+ *   S1  Eq. 1 is read as H_{i-1,j-1} + p(i,j) with a signed p (P:62-64,
+ *       P:315, Table X).
+ *   S2  the API's gap_open is G_open, so G_first = gap_open + gap_ext.
+ *   S3  E(i,0) = F(0,j) = -infinity (NEG below); H(i,0) = H(0,j) = 0.
+ *   S4  argmax tie-break: highest score, then smallest i, then smallest j;
+ *       score 0 reports (0,0).  Implemented as a row-major scan with '>'.
+ *   S5/S6 special rows hold columns 1..n of H and F for every i = k,2k,..<=m.
+ *   S7  characters are compared case-insensitively (codes A,C,G,T).
+ *   S9/S10 reverse pass: anchored global recurrence on the reversed
+ *       prefixes; first hit in row-major order of the reverse matrix.
+ *
+ * Arithmetic: int64 everywhere (wider than any kernel; the paper uses
+ * 4-byte cells, and all values here stay far inside int32).
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define NEG (-(int64_t)1 << 40) /* "minus infinity": never produced by a real cell */
+
+typedef struct {
+    int64_t score;
+    int64_t i;
+    int64_t j;
+} or_result;
+
+typedef int (*or_row_sink)(void *user, int64_t row, const int64_t *H, const int64_t *F, int64_t n);
+
+static int up(char c) { return (c >= 'a' && c <= 'z') ? c - 32 : c; }
+
+/* p(i,j) = ma if S0[i] = S1[j] (match) and mi otherwise. */
+static int64_t p_score(char a, char b, int64_t ma, int64_t mi) { return up(a) == up(b) ? ma : mi; }
+
+static int64_t max2(int64_t a, int64_t b) { return a > b ? a : b; }
+
+/*
+ * Stage 1, linear space: row-by-row fill of Eq. 1-3 keeping
+ * one previous row of H and F; E is carried along the row.  Returns the
+ * best score and the first (row-major) cell holding it.
+ * Every k-th row (k > 0) is handed to `sink` as H[1..n], F[1..n].
+ */
+int or_stage1(const char *S0, int64_t m, const char *S1, int64_t n, int64_t ma, int64_t mi,
+              int64_t G_open, int64_t G_ext, int64_t k, or_row_sink sink, void *user,
+              or_result *best)
+{
+    const int64_t G_first = G_open + G_ext;
+    int64_t *Hprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Hcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    if (!Hprev || !Fprev || !Hcur || !Fcur) {
+        free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+        return -1;
+    }
+    /* "the first row and column are filled with zeroes" */
+    for (int64_t j = 0; j <= n; j++) { Hprev[j] = 0; Fprev[j] = NEG; }
+    best->score = 0; best->i = 0; best->j = 0;
+    for (int64_t i = 1; i <= m; i++) {
+        int64_t E = NEG; /* E(i,0) */
+        Hcur[0] = 0;
+        Fcur[0] = NEG;
+        for (int64_t j = 1; j <= n; j++) {
+            /* Eq. 2: E_{i,j} = max(E_{i,j-1} - G_ext, H_{i,j-1} - G_first) */
+            E = max2(E - G_ext, Hcur[j - 1] - G_first);
+            /* Eq. 3: F_{i,j} = max(F_{i-1,j} - G_ext, H_{i-1,j} - G_first) */
+            Fcur[j] = max2(Fprev[j] - G_ext, Hprev[j] - G_first);
+            /* Eq. 1: H_{i,j} = max(0, E_{i,j}, F_{i,j}, H_{i-1,j-1} + p(i,j)) */
+            int64_t h = 0;
+            h = max2(h, E);
+            h = max2(h, Fcur[j]);
+            h = max2(h, Hprev[j - 1] + p_score(S0[i - 1], S1[j - 1], ma, mi));
+            Hcur[j] = h;
+            if (h > best->score) { best->score = h; best->i = i; best->j = j; }
+        }
+        if (k > 0 && i % k == 0 && sink) {
+            if (sink(user, i, Hcur + 1, Fcur + 1, n)) {
+                free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+                return -2;
+            }
+        }
+        int64_t *t;
+        t = Hprev; Hprev = Hcur; Hcur = t;
+        t = Fprev; Fprev = Fcur; Fcur = t;
+    }
+    free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+    return 0;
+}
+
+/*
+ * The same definition with the whole (m+1) x (n+1) matrices kept, for
+ * tiny inputs: H, E, F are row-major with row stride n+1.  Boundary cells
+ * hold H = 0, E = F = NEG (reading S3).
+ */
+int or_full_matrix(const char *S0, int64_t m, const char *S1, int64_t n, int64_t ma, int64_t mi,
+                   int64_t G_open, int64_t G_ext, int64_t *H, int64_t *E, int64_t *F)
+{
+    const int64_t G_first = G_open + G_ext;
+    const int64_t w = n + 1;
+    for (int64_t i = 0; i <= m; i++)
+        for (int64_t j = 0; j <= n; j++) {
+            if (i == 0 || j == 0) {
+                H[i * w + j] = 0;
+                E[i * w + j] = NEG;
+                F[i * w + j] = NEG;
+                continue;
+            }
+            E[i * w + j] = max2(E[i * w + j - 1] - G_ext, H[i * w + j - 1] - G_first);     /* Eq. 2 */
+            F[i * w + j] = max2(F[(i - 1) * w + j] - G_ext, H[(i - 1) * w + j] - G_first); /* Eq. 3 */
+            int64_t h = 0;                                                                   /* Eq. 1 */
+            h = max2(h, E[i * w + j]);
+            h = max2(h, F[i * w + j]);
+            h = max2(h, H[(i - 1) * w + j - 1] + p_score(S0[i - 1], S1[j - 1], ma, mi));
+            H[i * w + j] = h;
+        }
+    return 0;
+}
+
+/*
+ * One band of Stage 1: given row r0's H[0..n], F[0..n] (column 0 included:
+ * H = 0, F = NEG), compute rows r0+1..r1 and return row r1 in Hbot/Fbot
+ * (length n+1) plus the band's best (score, i, j) under the same order.
+ * Used to check special rows produced at scale by induction: row r0 + k
+ * must equal band(row r0).
+ */
+int or_band(const char *S0, int64_t m, const char *S1, int64_t n, int64_t ma, int64_t mi,
+            int64_t G_open, int64_t G_ext, int64_t r0, int64_t r1, const int64_t *Htop,
+            const int64_t *Ftop, int64_t *Hbot, int64_t *Fbot, or_result *best)
+{
+    const int64_t G_first = G_open + G_ext;
+    if (r0 < 0 || r1 < r0 || r1 > m) return -1;
+    int64_t *Hprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Hcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    if (!Hprev || !Fprev || !Hcur || !Fcur) {
+        free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+        return -1;
+    }
+    memcpy(Hprev, Htop, (size_t)(n + 1) * sizeof(int64_t));
+    memcpy(Fprev, Ftop, (size_t)(n + 1) * sizeof(int64_t));
+    best->score = 0; best->i = 0; best->j = 0;
+    for (int64_t i = r0 + 1; i <= r1; i++) {
+        int64_t E = NEG;
+        Hcur[0] = 0;
+        Fcur[0] = NEG;
+        for (int64_t j = 1; j <= n; j++) {
+            E = max2(E - G_ext, Hcur[j - 1] - G_first);
+            Fcur[j] = max2(Fprev[j] - G_ext, Hprev[j] - G_first);
+            int64_t h = 0;
+            h = max2(h, E);
+            h = max2(h, Fcur[j]);
+            h = max2(h, Hprev[j - 1] + p_score(S0[i - 1], S1[j - 1], ma, mi));
+            Hcur[j] = h;
+            if (h > best->score) { best->score = h; best->i = i; best->j = j; }
+        }
+        int64_t *t;
+        t = Hprev; Hprev = Hcur; Hcur = t;
+        t = Fprev; Fprev = Fcur; Fcur = t;
+    }
+    memcpy(Hbot, Hprev, (size_t)(n + 1) * sizeof(int64_t));
+    memcpy(Fbot, Fprev, (size_t)(n + 1) * sizeof(int64_t));
+    free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+    return 0;
+}
+
+/*
+ * Global (Needleman-Wunsch style) Gotoh score of S0[1..m] vs S1[1..n]:
+ * the recurrence of Eq. 1-3 without the 0 term, with the textbook global
+ * initialisation H(0,0) = 0, H(0,j) = E(0,j) = -(G_open + j G_ext),
+ * H(i,0) = F(i,0) = -(G_open + i G_ext), E(i,0) = F(0,j) = -infinity.
+ * This is the "global recurrence" Stage 2 runs (reading S9).
+ */
+int64_t or_global(const char *S0, int64_t m, const char *S1, int64_t n, int64_t ma, int64_t mi,
+                  int64_t G_open, int64_t G_ext)
+{
+    const int64_t G_first = G_open + G_ext;
+    int64_t *Hprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Hcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    Hprev[0] = 0;
+    Fprev[0] = NEG;
+    for (int64_t j = 1; j <= n; j++) { Hprev[j] = -(G_open + j * G_ext); Fprev[j] = NEG; }
+    for (int64_t i = 1; i <= m; i++) {
+        Hcur[0] = -(G_open + i * G_ext);
+        Fcur[0] = Hcur[0];
+        int64_t E = NEG;
+        for (int64_t j = 1; j <= n; j++) {
+            E = max2(E - G_ext, Hcur[j - 1] - G_first);
+            Fcur[j] = max2(Fprev[j] - G_ext, Hprev[j] - G_first);
+            int64_t h = max2(E, Fcur[j]);
+            h = max2(h, Hprev[j - 1] + p_score(S0[i - 1], S1[j - 1], ma, mi));
+            Hcur[j] = h;
+        }
+        int64_t *t;
+        t = Hprev; Hprev = Hcur; Hcur = t;
+        t = Fprev; Fprev = Fcur; Fcur = t;
+    }
+    int64_t r = (m == 0 && n == 0) ? 0 : Hprev[n];
+    if (m == 0 && n > 0) r = -(G_open + n * G_ext);
+    free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+    return r;
+}
+
+/*
+ * Reverse pass (Stage 2 reuse of the Stage-1 engine):
+ * reverse the prefixes S0[1..i_end] and S1[1..j_end], run the global
+ * recurrence (or_global's initialisation, no 0 term) and return the first
+ * cell (i', j'), i', j' >= 1, in row-major order of the reverse matrix with
+ * H = goal.  The forward start is (i_end - i', j_end - j'): the DP cell
+ * *before* the first aligned pair (reading S8, Table III).
+ * goal == 0 returns the end itself.  Returns 1 if found, 0 if not.
+ */
+int or_reverse_goal(const char *S0, int64_t i_end, const char *S1, int64_t j_end, int64_t ma,
+                    int64_t mi, int64_t G_open, int64_t G_ext, int64_t goal, or_result *start)
+{
+    const int64_t G_first = G_open + G_ext;
+    if (goal == 0) { start->score = 0; start->i = i_end; start->j = j_end; return 1; }
+    const int64_t m = i_end, n = j_end;
+    char *R0 = malloc((size_t)m + 1), *R1 = malloc((size_t)n + 1);
+    for (int64_t i = 0; i < m; i++) R0[i] = S0[i_end - 1 - i];
+    for (int64_t j = 0; j < n; j++) R1[j] = S1[j_end - 1 - j];
+    int64_t *Hprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fprev = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Hcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    int64_t *Fcur = malloc((size_t)(n + 1) * sizeof(int64_t));
+    Hprev[0] = 0;
+    Fprev[0] = NEG;
+    for (int64_t j = 1; j <= n; j++) { Hprev[j] = -(G_open + j * G_ext); Fprev[j] = NEG; }
+    int found = 0;
+    for (int64_t i = 1; i <= m && !found; i++) {
+        Hcur[0] = -(G_open + i * G_ext);
+        Fcur[0] = Hcur[0];
+        int64_t E = NEG;
+        for (int64_t j = 1; j <= n; j++) {
+            E = max2(E - G_ext, Hcur[j - 1] - G_first);
+            Fcur[j] = max2(Fprev[j] - G_ext, Hprev[j] - G_first);
+            int64_t h = max2(E, Fcur[j]);
+            h = max2(h, Hprev[j - 1] + p_score(R0[i - 1], R1[j - 1], ma, mi));
+            Hcur[j] = h;
+            if (!found && h == goal) {
+                found = 1;
+                start->score = goal;
+                start->i = i_end - i;
+                start->j = j_end - j;
+            }
+        }
+        int64_t *t;
+        t = Hprev; Hprev = Hcur; Hcur = t;
+        t = Fprev; Fprev = Fcur; Fcur = t;
+    }
+    free(R0); free(R1); free(Hprev); free(Fprev); free(Hcur); free(Fcur);
+    return found;
+}
+
+/*
+ * Flush-interval rule: the flush interval, in blocks of alpha*T
+ * rows, must be at least ceil(8 m n / (alpha T |SRA|)).  Returns the
+ * special-row spacing R = alpha*T * ceil(8 m n / (alpha T |SRA|)) in rows.
+ */
+int64_t or_flush_rows(int64_t m, int64_t n, int64_t alphaT, int64_t sra_bytes)
+{
+    /* 8 m n can exceed 2^63 for huge inputs: compute with long double and fix up. */
+    long double num = 8.0L * (long double)m * (long double)n;
+    long double den = (long double)alphaT * (long double)sra_bytes;
+    int64_t q = (int64_t)(num / den);
+    while ((long double)q * den < num) q++;
+    while (q > 0 && (long double)(q - 1) * den >= num) q--;
+    if (q < 1) q = 1;
+    return alphaT * q;
+}
