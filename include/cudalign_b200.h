@@ -1,0 +1,147 @@
+/*
+ * cudalign_b200.h -- C ABI of the B200-native Stage-1 Smith-Waterman/Gotoh
+ * engine (CUDAlign 2.0, Sandes & de Melo, IPDPS 2011; citations P:<line> are
+ * lines of /root/reference/PAPER.md).
+ *
+ * What it computes:
+ *   Stage 1: the Smith-Waterman matrix H with Gotoh affine gaps
+ *   (Eq. 1-3) over S0 (m rows, i) and S1 (n columns, j) in linear
+ *   space; the best score and its end cell; every k-th
+ *   "special row" of H and F handed to the host.
+ *   Reverse pass: the same engine on the reversed
+ *   prefixes with the global recurrence, returning the start cell.
+ *
+ * Scoring convention (readings S1, S2 of DESIGN.md):
+ *   match, mismatch : signed scores ADDED to H_{i-1,j-1} (Eq. 1 read as "+p").
+ *   gap_open, gap_ext : non-negative penalties SUBTRACTED; a gap of length L
+ *   costs gap_open + L*gap_ext, i.e. G_first = gap_open + gap_ext and
+ *   G_ext = gap_ext.  The paper's experiments are (+1, -3, 3, 2)
+ *   ("first gap -5, extension -2").
+ *   Supported range (the kernel packs the substitution profile into int8):
+ *   |match + gap_open + gap_ext| <= 127 and |mismatch + gap_open + gap_ext| <= 127.
+ *
+ * Coordinates (reading S8): 1-based DP cells.  The end cell is the last
+ * aligned pair; the start cell is the cell *before* the first aligned pair
+ * (so end - start = length for a gapless alignment, Table III).
+ *
+ * Errors: every int-returning call returns SW_OK (0) or a negative code;
+ * on error the output structs are left untouched.  There is no CPU fallback:
+ * without a usable CUDA device sw_init fails with SW_ECUDA.
+ *
+ * Threading: one call at a time per context.  Special-row sinks are called
+ * on the calling thread, in strictly ascending row order.
+ */
+#ifndef CUDALIGN_B200_H
+#define CUDALIGN_B200_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SW_OK 0
+#define SW_EINVAL (-1)     /* null pointer, negative size, bad scoring, bad device list */
+#define SW_EALPHABET (-2)  /* a byte outside ACGTacgt (reading S7) */
+#define SW_ERANGE (-3)     /* scores could leave the int32-safe range (+-2^30) */
+#define SW_ENOMEM (-4)     /* device or pinned host allocation failed */
+#define SW_ECUDA (-5)      /* CUDA runtime error (message via sw_last_error) */
+#define SW_EABORTED (-6)   /* the special-row sink returned non-zero */
+#define SW_ENOTFOUND (-7)  /* sw_reverse_goal: no cell equals goal (goal > H(i_end, j_end)) */
+
+typedef struct sw_ctx sw_ctx;
+
+/* Best (score, i, j).  Stage 1: highest score, then smallest i, then smallest
+ * j (reading S4); (0, 0, 0) iff the best score is 0. */
+typedef struct {
+    int32_t score;
+    int64_t i;
+    int64_t j;
+} sw_result;
+
+/* Special-row sink: H and F are columns 1..n of DP row `row`, int32,
+ * in library-owned pinned host memory valid only during the call.  Called
+ * from the thread that called sw_align_stage1, rows strictly ascending.
+ * A non-zero return aborts the alignment with SW_EABORTED. */
+typedef int (*sw_row_sink)(void *user, int64_t row, const int32_t *H, const int32_t *F, int64_t n);
+
+/* Timing breakdown of the last call (milliseconds, CUDA events on the
+ * library's stream). */
+typedef struct {
+    double total_ms;   /* whole call (host API, includes copies) */
+    double upload_ms;  /* host -> device copy of the sequences (0 for *_dev calls) */
+    double encode_ms;  /* encode/pack kernel */
+    double fill_ms;    /* the Stage-1 / reverse matrix-fill kernel */
+    double reduce_ms;  /* best-cell reduction kernel + result copy */
+    int64_t kernel_launches; /* kernels launched by the call */
+    int64_t replays;   /* tiles replayed for exact argmax tracking */
+    int64_t special_rows;
+    int64_t special_bytes_d2h;
+    int32_t alpha, warps, width, grid; /* launch configuration */
+} sw_stats;
+
+/* Create a context on the given CUDA devices.  Round 1 supports exactly one
+ * device per context (one process per GPU); device_ids[0] is used.
+ * Allocates the library's streams.  Returns SW_EINVAL / SW_ECUDA. */
+int sw_init(const int *device_ids, int n_devices, sw_ctx **out);
+
+/* Stage 1 on host sequences.
+ *   seqA : S0, m bytes of ACGTacgt (not NUL-terminated, borrowed for the call)
+ *   seqB : S1, n bytes
+ *   special_row_interval k >= 0: rows k, 2k, ... <= m go to `sink` (0 = none;
+ *   any k >= 1 is correct, multiples of sw_row_granularity() are fastest).
+ *   sink may be NULL when k == 0.
+ *   out  : best score and end cell.
+ * m or n == 0 returns {0,0,0} and no rows.  m, n < 2^31. */
+int sw_align_stage1(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, int64_t n,
+                    int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                    int64_t special_row_interval, sw_row_sink sink, void *user, sw_result *out);
+
+/* Same as sw_align_stage1 but the sequences are DEVICE pointers (bytes of
+ * ACGTacgt already resident in HBM on the context's device) and the work is
+ * ordered after `stream` (a cudaStream_t, or NULL for the library stream).
+ * Returns when the result is on the host. */
+int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                        int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                        int64_t special_row_interval, sw_row_sink sink, void *user, void *stream,
+                        sw_result *out);
+
+/* Reverse pass (readings S9, S10): run the global
+ * recurrence over S0[1..i_end]^R x S1[1..j_end]^R from H(0,0) = 0 and return
+ * the first cell (i', j') (row-major, i', j' >= 1) whose H equals `goal`,
+ * mapped to the forward start cell (i_end - i', j_end - j').  goal == 0
+ * returns (0, i_end, j_end).  start_out = {goal, i_s, j_s}.
+ * SW_ENOTFOUND when no cell equals goal. */
+int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, const char *seqB, int64_t j_end,
+                    int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                    int32_t goal, sw_result *start_out);
+
+/* sw_reverse_goal on DEVICE pointers (bytes of ACGTacgt resident in HBM). */
+int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end, const char *dseqB, int64_t j_end,
+                        int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                        int32_t goal, sw_result *start_out);
+
+/* Rows per thread strip (alpha): special_row_interval multiples of this take
+ * the fast special-row path. */
+int64_t sw_row_granularity(const sw_ctx *ctx);
+
+/* Flush-interval rule of P:178 as a helper: the special-row spacing in rows,
+ * R = bh * ceil(8 m n / (bh * sra_bytes)), for a byte budget sra_bytes. */
+int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int64_t bh, int64_t sra_bytes);
+
+/* Stats of the last successful call on this context. */
+int sw_get_stats(const sw_ctx *ctx, sw_stats *out);
+
+/* Release everything.  NULL is a no-op. */
+void sw_shutdown(sw_ctx *ctx);
+
+/* Static description of an error code. */
+const char *sw_strerror(int code);
+
+/* Text of the last CUDA error seen on this context (empty if none). */
+const char *sw_last_error(const sw_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUDALIGN_B200_H */

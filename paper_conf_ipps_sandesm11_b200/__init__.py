@@ -1,0 +1,253 @@
+"""paper_conf_ipps_sandesm11_b200 -- B200-native CUDAlign 2.0 Stage 1.
+
+Thin ctypes binding (argument marshalling only) over the C ABI declared in
+``include/cudalign_b200.h`` and implemented by ``libcudalign_b200.so``
+(csrc/sw_api.cu, csrc/sw_fill.cuh).  Every step of the path runs in the
+library's sm_100a kernels; there is no CPU fallback -- if the shared library
+is missing or no CUDA device is usable, the calls raise.
+
+Paper: Sandes & de Melo, "Smith-Waterman Alignment of Huge Sequences with GPU
+in Linear Space", IPDPS 2011 (``P:<line>`` = /root/reference/PAPER.md).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import build as _build
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libcudalign_b200.so")
+
+SW_OK = 0
+SW_EINVAL = -1
+SW_EALPHABET = -2
+SW_ERANGE = -3
+SW_ENOMEM = -4
+SW_ECUDA = -5
+SW_EABORTED = -6
+SW_ENOTFOUND = -7
+
+EXPORTED = [
+    "sw_init",
+    "sw_align_stage1",
+    "sw_align_stage1_dev",
+    "sw_reverse_goal",
+    "sw_reverse_goal_dev",
+    "sw_row_granularity",
+    "sw_special_row_interval_for_budget",
+    "sw_get_stats",
+    "sw_shutdown",
+    "sw_strerror",
+    "sw_last_error",
+]
+
+
+class SwError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{msg} (code {code})")
+        self.code = code
+
+
+class _Result(ctypes.Structure):
+    _fields_ = [("score", ctypes.c_int32), ("i", ctypes.c_int64), ("j", ctypes.c_int64)]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [
+        ("total_ms", ctypes.c_double),
+        ("upload_ms", ctypes.c_double),
+        ("encode_ms", ctypes.c_double),
+        ("fill_ms", ctypes.c_double),
+        ("reduce_ms", ctypes.c_double),
+        ("kernel_launches", ctypes.c_int64),
+        ("replays", ctypes.c_int64),
+        ("special_rows", ctypes.c_int64),
+        ("special_bytes_d2h", ctypes.c_int64),
+        ("alpha", ctypes.c_int32),
+        ("warps", ctypes.c_int32),
+        ("width", ctypes.c_int32),
+        ("grid", ctypes.c_int32),
+    ]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+SINK = ctypes.CFUNCTYPE(
+    ctypes.c_int,
+    ctypes.c_void_p,
+    ctypes.c_int64,
+    ctypes.POINTER(ctypes.c_int32),
+    ctypes.POINTER(ctypes.c_int32),
+    ctypes.c_int64,
+)
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Load libcudalign_b200.so (raises if it is missing: no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built; run __graft_entry__.build() or python -m paper_conf_ipps_sandesm11_b200.build")
+    lib = ctypes.CDLL(path)
+    i32, i64, vp, cp = ctypes.c_int32, ctypes.c_int64, ctypes.c_void_p, ctypes.c_char_p
+    R = ctypes.POINTER(_Result)
+    lib.sw_init.argtypes = [ctypes.POINTER(ctypes.c_int), ctypes.c_int, ctypes.POINTER(vp)]
+    lib.sw_init.restype = ctypes.c_int
+    lib.sw_align_stage1.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i64, SINK, vp, R]
+    lib.sw_align_stage1.restype = ctypes.c_int
+    lib.sw_align_stage1_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i64, SINK, vp, vp, R]
+    lib.sw_align_stage1_dev.restype = ctypes.c_int
+    lib.sw_reverse_goal.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, R]
+    lib.sw_reverse_goal.restype = ctypes.c_int
+    lib.sw_reverse_goal_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, R]
+    lib.sw_reverse_goal_dev.restype = ctypes.c_int
+    lib.sw_row_granularity.argtypes = [vp]
+    lib.sw_row_granularity.restype = i64
+    lib.sw_special_row_interval_for_budget.argtypes = [i64, i64, i64, i64]
+    lib.sw_special_row_interval_for_budget.restype = i64
+    lib.sw_get_stats.argtypes = [vp, ctypes.POINTER(Stats)]
+    lib.sw_get_stats.restype = ctypes.c_int
+    lib.sw_shutdown.argtypes = [vp]
+    lib.sw_shutdown.restype = None
+    lib.sw_strerror.argtypes = [ctypes.c_int]
+    lib.sw_strerror.restype = cp
+    lib.sw_last_error.argtypes = [vp]
+    lib.sw_last_error.restype = cp
+    _lib = lib
+    return lib
+
+
+def special_row_interval_for_budget(m: int, n: int, bh: int, sra_bytes: int) -> int:
+    """Flush-interval rule of P:178 (computed in the library)."""
+    return int(load_library().sw_special_row_interval_for_budget(m, n, bh, sra_bytes))
+
+
+def _as_bytes_ptr(x):
+    """(pointer, length, keepalive) for bytes / str / numpy uint8 host sequences."""
+    if isinstance(x, str):
+        x = x.encode("ascii")
+    if isinstance(x, (bytes, bytearray)):
+        arr = np.frombuffer(bytes(x), dtype=np.uint8)
+    else:
+        arr = np.ascontiguousarray(x, dtype=np.uint8)
+    return arr.ctypes.data, arr.size, arr
+
+
+@dataclass
+class Result:
+    score: int
+    i: int
+    j: int
+
+    def astuple(self):
+        return (self.score, self.i, self.j)
+
+
+class Context:
+    """One engine context on one CUDA device (one process per GPU)."""
+
+    def __init__(self, device: int = 0):
+        self._lib = load_library()
+        self._h = ctypes.c_void_p()
+        ids = (ctypes.c_int * 1)(device)
+        rc = self._lib.sw_init(ids, 1, ctypes.byref(self._h))
+        if rc != SW_OK:
+            raise SwError(rc, f"sw_init(device={device}) failed: {self._lib.sw_strerror(rc).decode()}")
+        self.device = device
+
+    # ------------------------------------------------------------------ helpers
+    def _check(self, rc, what):
+        if rc != SW_OK:
+            detail = self._lib.sw_last_error(self._h).decode()
+            raise SwError(rc, f"{what}: {self._lib.sw_strerror(rc).decode()}" + (f" [{detail}]" if detail else ""))
+
+    @staticmethod
+    def _make_sink(sink, keep_rows, rows):
+        def _cb(_user, row, H, F, n):
+            try:
+                h = np.ctypeslib.as_array(H, shape=(n,))
+                f = np.ctypeslib.as_array(F, shape=(n,))
+                if keep_rows:
+                    rows.append((int(row), h.copy(), f.copy()))
+                if sink is not None:
+                    return 1 if sink(int(row), h, f) else 0
+                return 0
+            except Exception:  # never let an exception cross the C boundary
+                return 1
+
+        return SINK(_cb)
+
+    # ------------------------------------------------------------------ API
+    def align_stage1(self, A, B, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0, sink=None, keep_rows=False):
+        """Stage 1 on host sequences.  Returns (Result, rows) where rows is the
+        list of (row, H, F) if keep_rows.  ``sink(row, H, F)`` (views valid only
+        during the call) may return True to abort."""
+        pa, m, ka = _as_bytes_ptr(A)
+        pb, n, kb = _as_bytes_ptr(B)
+        rows = []
+        cb = self._make_sink(sink, keep_rows, rows) if k > 0 else SINK()
+        out = _Result()
+        rc = self._lib.sw_align_stage1(self._h, pa, m, pb, n, match, mismatch, gap_open, gap_ext, k, cb, None, ctypes.byref(out))
+        self._check(rc, "sw_align_stage1")
+        return Result(out.score, out.i, out.j), rows
+
+    def align_stage1_dev(self, dA_ptr: int, m: int, dB_ptr: int, n: int, match=1, mismatch=-3, gap_open=3, gap_ext=2,
+                         k=0, sink=None, keep_rows=False, stream: int = 0):
+        """Stage 1 on DEVICE byte buffers (e.g. torch uint8 cuda tensors' data_ptr())."""
+        rows = []
+        cb = self._make_sink(sink, keep_rows, rows) if k > 0 else SINK()
+        out = _Result()
+        rc = self._lib.sw_align_stage1_dev(self._h, dA_ptr, m, dB_ptr, n, match, mismatch, gap_open, gap_ext, k, cb,
+                                           None, stream or None, ctypes.byref(out))
+        self._check(rc, "sw_align_stage1_dev")
+        return Result(out.score, out.i, out.j), rows
+
+    def reverse_goal(self, A, i_end, B, j_end, goal, match=1, mismatch=-3, gap_open=3, gap_ext=2):
+        """Start cell of the alignment ending at (i_end, j_end) with score goal."""
+        pa, m, ka = _as_bytes_ptr(A)
+        pb, n, kb = _as_bytes_ptr(B)
+        if i_end > m or j_end > n:
+            raise ValueError("end cell outside the sequences")
+        out = _Result()
+        rc = self._lib.sw_reverse_goal(self._h, pa, i_end, pb, j_end, match, mismatch, gap_open, gap_ext, goal, ctypes.byref(out))
+        self._check(rc, "sw_reverse_goal")
+        return Result(out.score, out.i, out.j)
+
+    def reverse_goal_dev(self, dA_ptr, i_end, dB_ptr, j_end, goal, match=1, mismatch=-3, gap_open=3, gap_ext=2):
+        out = _Result()
+        rc = self._lib.sw_reverse_goal_dev(self._h, dA_ptr, i_end, dB_ptr, j_end, match, mismatch, gap_open, gap_ext, goal, ctypes.byref(out))
+        self._check(rc, "sw_reverse_goal_dev")
+        return Result(out.score, out.i, out.j)
+
+    def row_granularity(self) -> int:
+        return int(self._lib.sw_row_granularity(self._h))
+
+    def stats(self) -> dict:
+        s = Stats()
+        self._check(self._lib.sw_get_stats(self._h, ctypes.byref(s)), "sw_get_stats")
+        return s.as_dict()
+
+    def close(self):
+        if self._h:
+            self._lib.sw_shutdown(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

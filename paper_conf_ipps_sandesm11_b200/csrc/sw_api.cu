@@ -1,0 +1,677 @@
+// sw_api.cu -- C ABI (include/cudalign_b200.h) and host runtime of the
+// B200-native Stage-1 engine: parameter validation, sequence encode/pack,
+// persistent fill launch, special-row streaming to the host sink through
+// pinned memory on a side stream, best-cell reduction, and the
+// reverse goal pass.  No CPU fallback: every step runs in the
+// kernels below or in sw_fill.cuh.
+#include <algorithm>
+#include <chrono>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <thread>
+
+#include "../../include/cudalign_b200.h"
+#include "sw_fill.cuh"
+
+using namespace swb;
+
+// ---------------------------------------------------------------- small device kernels
+
+// a1: ASCII -> 2-bit codes (A=0, C=1, G=2, T=3, case-insensitive, reading S7),
+// 16 codes per 32-bit word; optional reversal (reverse pass).  Any other byte
+// sets *err.
+__global__ void sw_encode_kernel(const unsigned char *sa, long long la, int reva, uint32_t *da, long long wa,
+                                 const unsigned char *sb, long long lb, int revb, uint32_t *db, long long wb,
+                                 int *err)
+{
+    long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const unsigned char *src;
+    long long len;
+    int rev;
+    uint32_t *dst;
+    if (w < wa) {
+        src = sa; len = la; rev = reva; dst = da;
+    } else {
+        w -= wa;
+        if (w >= wb) return;
+        src = sb; len = lb; rev = revb; dst = db;
+    }
+    uint32_t word = 0;
+    int bad = 0;
+#pragma unroll
+    for (int x = 0; x < 16; x++) {
+        const long long i = w * 16 + x;
+        if (i < len) {
+            const unsigned char ch = src[rev ? len - 1 - i : i] | 0x20;
+            uint32_t code = 0;
+            if (ch == 'a') code = 0;
+            else if (ch == 'c') code = 1;
+            else if (ch == 'g') code = 2;
+            else if (ch == 't') code = 3;
+            else bad = 1;
+            word |= code << (2 * x);
+        }
+    }
+    dst[w] = word;
+    if (bad) atomicOr(err, 1);
+}
+
+// a5: final (score, i, j) over the per-CTA slots (LOCAL), or decode the first
+// hit (GLOBAL).  out = {score, i, j, status}.
+__global__ void sw_reduce_kernel(const int4 *slots, int nslots, int local, const unsigned long long *hit_key,
+                                 int goal, int4 *out)
+{
+    __shared__ int4 red[32];
+    const int tid = threadIdx.x;
+    if (!local) {
+        if (tid == 0) {
+            const unsigned long long k = *hit_key;
+            if (k == ~0ull) *out = make_int4(goal, 0, 0, 0);
+            else *out = make_int4(goal, (int)(k >> 32), (int)(k & 0xffffffffu), 1);
+        }
+        return;
+    }
+    int bs = 0, bi = 0, bj = 0;
+    for (int x = tid; x < nslots; x += blockDim.x) {
+        const int4 v = slots[x];
+        if (v.x > 0 && better(v.x, v.y, v.z, bs, bi, bj)) { bs = v.x; bi = v.y; bj = v.z; }
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+        const int s2 = __shfl_down_sync(0xffffffffu, bs, o);
+        const int i2 = __shfl_down_sync(0xffffffffu, bi, o);
+        const int j2 = __shfl_down_sync(0xffffffffu, bj, o);
+        if (s2 > 0 && better(s2, i2, j2, bs, bi, bj)) { bs = s2; bi = i2; bj = j2; }
+    }
+    if ((tid & 31) == 0) red[tid >> 5] = make_int4(bs, bi, bj, 0);
+    __syncthreads();
+    if (tid == 0) {
+        int4 r = make_int4(0, 0, 0, 1);
+        for (int w = 0; w < (int)(blockDim.x + 31) / 32; w++)
+            if (red[w].x > 0 && better(red[w].x, red[w].y, red[w].z, r.x, r.y, r.z)) r = make_int4(red[w].x, red[w].y, red[w].z, 1);
+        *out = r;
+    }
+}
+
+// ---------------------------------------------------------------- kernel variants
+
+struct Variant {
+    int alpha, nw, w;
+    const void *local_fn, *global_fn;
+    size_t smem;
+};
+
+template <int ALPHA, int NW, int W>
+static Variant make_variant()
+{
+    Variant v;
+    v.alpha = ALPHA;
+    v.nw = NW;
+    v.w = W;
+    v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
+    v.global_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, false>;
+    v.smem = Fill<ALPHA, NW, W, true>::smem_bytes();
+    return v;
+}
+
+static const Variant &variant_for(int idx)
+{
+    static const Variant vs[] = {
+        make_variant<16, 4, 32>(),
+        make_variant<16, 8, 32>(),
+        make_variant<8, 4, 32>(),
+    };
+    const int n = sizeof(vs) / sizeof(vs[0]);
+    return vs[idx < 0 ? 0 : idx >= n ? n - 1 : idx];
+}
+
+// ---------------------------------------------------------------- context
+
+struct DevBuf {
+    void *p = nullptr;
+    size_t cap = 0;
+};
+
+struct sw_ctx {
+    int device = 0;
+    int num_sms = 0;
+    cudaStream_t stream = nullptr, side = nullptr;
+    cudaEvent_t ev[6] = {};
+    DevBuf seq, a2, b2, rowb, progress, misc, slots, sp;
+    unsigned int *flags_h = nullptr, *flags_d = nullptr;
+    size_t flags_cap = 0;
+    int32_t *stage_h = nullptr;
+    size_t stage_cap = 0;
+    int4 *res_h = nullptr;  // pinned: result + err
+    sw_stats stats{};
+    char errbuf[512] = {0};
+    int variant_override = -1;
+};
+
+static int cuda_fail(sw_ctx *c, cudaError_t e, const char *what)
+{
+    if (c) snprintf(c->errbuf, sizeof(c->errbuf), "%s: %s", what, cudaGetErrorString(e));
+    return SW_ECUDA;
+}
+
+#define CK(call)                                                          \
+    do {                                                                  \
+        cudaError_t e_ = (call);                                          \
+        if (e_ != cudaSuccess) return cuda_fail(ctx, e_, #call);          \
+    } while (0)
+
+static int grow(sw_ctx *ctx, DevBuf &b, size_t bytes)
+{
+    if (b.cap >= bytes && b.p) return SW_OK;
+    if (b.p) cudaFree(b.p);
+    b.p = nullptr;
+    b.cap = 0;
+    size_t want = std::max<size_t>(bytes, 256);
+    cudaError_t e = cudaMalloc(&b.p, want);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "cudaMalloc(%zu): %s", want, cudaGetErrorString(e));
+        return SW_ENOMEM;
+    }
+    b.cap = want;
+    return SW_OK;
+}
+
+extern "C" const char *sw_strerror(int code)
+{
+    switch (code) {
+    case SW_OK: return "ok";
+    case SW_EINVAL: return "invalid argument";
+    case SW_EALPHABET: return "sequence byte outside ACGTacgt";
+    case SW_ERANGE: return "scores could exceed the int32-safe range";
+    case SW_ENOMEM: return "out of memory";
+    case SW_ECUDA: return "CUDA error";
+    case SW_EABORTED: return "aborted by the special-row sink";
+    case SW_ENOTFOUND: return "no cell equals the goal score";
+    default: return "unknown error";
+    }
+}
+
+extern "C" const char *sw_last_error(const sw_ctx *ctx) { return ctx ? ctx->errbuf : ""; }
+
+extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
+{
+    if (!out || n_devices != 1 || !device_ids) return SW_EINVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0) { cudaGetLastError(); return SW_ECUDA; }
+    if (device_ids[0] < 0 || device_ids[0] >= ndev) return SW_EINVAL;
+    sw_ctx *ctx = new sw_ctx();
+    ctx->device = device_ids[0];
+    int rc = SW_OK;
+    do {
+        cudaError_t e;
+        if ((e = cudaSetDevice(ctx->device)) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaSetDevice"); break; }
+        cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, ctx->device);
+        if ((e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
+        if ((e = cudaStreamCreateWithFlags(&ctx->side, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
+        for (auto &ev : ctx->ev)
+            if ((e = cudaEventCreate(&ev)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
+        if (rc) break;
+        if ((e = cudaHostAlloc(&ctx->res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
+        for (int i = 0; i < 3; i++) {
+            const Variant &v = variant_for(i);
+            cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+            cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+        }
+        if ((e = cudaGetLastError()) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaFuncSetAttribute"); break; }
+        const char *ov = getenv("SWB_VARIANT");
+        if (ov) ctx->variant_override = atoi(ov);
+    } while (0);
+    if (rc) { sw_shutdown(ctx); return rc; }
+    *out = ctx;
+    return SW_OK;
+}
+
+extern "C" void sw_shutdown(sw_ctx *ctx)
+{
+    if (!ctx) return;
+    cudaSetDevice(ctx->device);
+    if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    if (ctx->side) cudaStreamSynchronize(ctx->side);
+    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->rowb, &ctx->progress, &ctx->misc, &ctx->slots, &ctx->sp})
+        if (b->p) cudaFree(b->p);
+    if (ctx->flags_h) cudaFreeHost(ctx->flags_h);
+    if (ctx->stage_h) cudaFreeHost(ctx->stage_h);
+    if (ctx->res_h) cudaFreeHost(ctx->res_h);
+    for (auto &ev : ctx->ev)
+        if (ev) cudaEventDestroy(ev);
+    if (ctx->stream) cudaStreamDestroy(ctx->stream);
+    if (ctx->side) cudaStreamDestroy(ctx->side);
+    delete ctx;
+}
+
+extern "C" int64_t sw_row_granularity(const sw_ctx *ctx)
+{
+    if (!ctx) return 0;
+    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0).alpha;
+}
+
+extern "C" int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int64_t bh, int64_t sra_bytes)
+{
+    // Flush interval (blocks of bh rows) >= ceil(8 m n / (bh |SRA|)).
+    if (m <= 0 || n <= 0 || bh <= 0 || sra_bytes <= 0) return 0;
+    const unsigned __int128 num = (unsigned __int128)8 * (unsigned __int128)m * (unsigned __int128)n;
+    const unsigned __int128 den = (unsigned __int128)bh * (unsigned __int128)sra_bytes;
+    unsigned __int128 q = (num + den - 1) / den;
+    if (q < 1) q = 1;
+    return (int64_t)(bh * (int64_t)q);
+}
+
+extern "C" int sw_get_stats(const sw_ctx *ctx, sw_stats *out)
+{
+    if (!ctx || !out) return SW_EINVAL;
+    *out = ctx->stats;
+    return SW_OK;
+}
+
+// ---------------------------------------------------------------- validation
+
+static int check_scoring(int32_t ma, int32_t mi, int32_t go, int32_t ge, int64_t m, int64_t n)
+{
+    if (go < 0 || ge < 0) return SW_EINVAL;
+    const long long gf = (long long)go + ge;
+    if (llabs(ma + gf) > 127 || llabs(mi + gf) > 127) return SW_EINVAL;  // int8 profile
+    const long long lim = 1ll << 30;
+    const long long mn = std::min(m, n);
+    if (mn * (long long)std::max(std::abs(ma), std::abs(mi)) >= lim) return SW_ERANGE;
+    if ((m + n + 2) * (gf + 1) + mn * (long long)std::abs(mi) >= lim) return SW_ERANGE;
+    return SW_OK;
+}
+
+// ---------------------------------------------------------------- the core call
+
+namespace {
+struct Job {
+    const unsigned char *dA;
+    int64_t m;
+    const unsigned char *dB;
+    int64_t n;
+    bool revA, revB;
+    int32_t ma, mi, go, ge;
+    int64_t k;
+    sw_row_sink sink;
+    void *user;
+    bool local;
+    int32_t goal;
+};
+}  // namespace
+
+static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
+{
+    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0);
+    const int W = V.w;
+    const int BH = V.alpha * 32 * V.nw;
+    const int m = (int)J.m, n = (int)J.n;
+    const int ncols_pad = ((n + W - 1) / W) * W;
+    const int NT = ncols_pad / W + 1;
+    const int nb = (m + BH - 1) / BH;
+    const long long wa = (J.m + 15) / 16 + 2, wb = (J.n + 15) / 16 + 2;
+    int rc;
+    if ((rc = grow(ctx, ctx->a2, wa * 4))) return rc;
+    if ((rc = grow(ctx, ctx->b2, wb * 4))) return rc;
+    if ((rc = grow(ctx, ctx->rowb, (size_t)(NT * W + 2 * W) * sizeof(int2)))) return rc;
+    if ((rc = grow(ctx, ctx->progress, (size_t)(nb + 1) * sizeof(int)))) return rc;
+    // misc: err, ticket, gbest, hit_band, (pad), hit_key(8B), replays(8B)
+    if ((rc = grow(ctx, ctx->misc, 64))) return rc;
+    int blocks_per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, J.local ? V.local_fn : V.global_fn, V.nw * 32 + 32, V.smem);
+    if (blocks_per_sm < 1) blocks_per_sm = 1;
+    int grid = std::min(nb, blocks_per_sm * ctx->num_sms);
+    if (const char *g = getenv("SWB_GRID")) grid = std::max(1, std::min(nb, atoi(g)));
+    if ((rc = grow(ctx, ctx->slots, (size_t)grid * sizeof(int4)))) return rc;
+
+    // special rows: all of them stay resident on the device (180 GB HBM) and
+    // are streamed to the host as bands complete.
+    const long long nsp = (J.local && J.k > 0) ? J.m / J.k : 0;
+    const int ld = ((n + 31) / 32) * 32;
+    const long long stride = 2ll * ld;
+    if (nsp > 0) {
+        size_t freeb = 0, totb = 0;
+        cudaMemGetInfo(&freeb, &totb);
+        const size_t need = (size_t)nsp * stride * sizeof(int);
+        if (need > ctx->sp.cap && need > (size_t)(0.8 * (double)(freeb + ctx->sp.cap))) {
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special rows need %zu bytes on the device", need);
+            return SW_ENOMEM;
+        }
+        if ((rc = grow(ctx, ctx->sp, need))) return rc;
+        if ((size_t)nsp > ctx->flags_cap) {
+            if (ctx->flags_h) cudaFreeHost(ctx->flags_h);
+            ctx->flags_h = nullptr;
+            ctx->flags_cap = 0;
+            if (cudaHostAlloc(&ctx->flags_h, nsp * sizeof(unsigned int), cudaHostAllocMapped) != cudaSuccess) {
+                cudaGetLastError();
+                return SW_ENOMEM;
+            }
+            ctx->flags_cap = nsp;
+            CK(cudaHostGetDevicePointer((void **)&ctx->flags_d, ctx->flags_h, 0));
+        }
+        memset(ctx->flags_h, 0, nsp * sizeof(unsigned int));
+        if ((size_t)stride > ctx->stage_cap) {
+            if (ctx->stage_h) cudaFreeHost(ctx->stage_h);
+            ctx->stage_h = nullptr;
+            ctx->stage_cap = 0;
+            if (cudaHostAlloc(&ctx->stage_h, stride * sizeof(int32_t), cudaHostAllocDefault) != cudaSuccess) {
+                cudaGetLastError();
+                return SW_ENOMEM;
+            }
+            ctx->stage_cap = stride;
+        }
+    }
+
+    cudaStream_t st = ctx->stream;
+    if (user_stream) {
+        // order our work after the caller's stream
+        CK(cudaEventRecord(ctx->ev[5], user_stream));
+        CK(cudaStreamWaitEvent(st, ctx->ev[5], 0));
+    }
+    char *misc = (char *)ctx->misc.p;
+    int *d_err = (int *)(misc + 0);
+    int *d_ticket = (int *)(misc + 4);
+    int *d_gbest = (int *)(misc + 8);
+    int *d_hit_band = (int *)(misc + 12);
+    unsigned long long *d_hit_key = (unsigned long long *)(misc + 16);
+    unsigned long long *d_replays = (unsigned long long *)(misc + 24);
+    int4 *d_res = (int4 *)(misc + 32);
+
+    CK(cudaEventRecord(ctx->ev[0], st));
+    CK(cudaMemsetAsync(misc, 0, 16, st));
+    CK(cudaMemsetAsync(d_hit_band, 0x7f, 4, st));
+    CK(cudaMemsetAsync(d_hit_key, 0xff, 8, st));
+    CK(cudaMemsetAsync(d_replays, 0, 8, st));
+    CK(cudaMemsetAsync(ctx->progress.p, 0, (size_t)(nb + 1) * sizeof(int), st));
+    {
+        const long long words = wa + wb;
+        const int tpb = 256;
+        sw_encode_kernel<<<(unsigned)((words + tpb - 1) / tpb), tpb, 0, st>>>(
+            J.dA, J.m, J.revA, (uint32_t *)ctx->a2.p, wa, J.dB, J.n, J.revB, (uint32_t *)ctx->b2.p, wb, d_err);
+        CK(cudaGetLastError());
+    }
+    CK(cudaEventRecord(ctx->ev[1], st));
+
+    FillArgs a{};
+    a.m = m;
+    a.n = n;
+    a.ncols_pad = ncols_pad;
+    a.NT = NT;
+    a.nb = nb;
+    a.go = J.go;
+    a.ge = J.ge;
+    a.gf = J.go + J.ge;
+    for (int x = 0; x < 4; x++) {
+        uint32_t w = 0;
+        for (int y = 0; y < 4; y++) {
+            const int v = (x == y ? J.ma : J.mi) + a.gf;
+            w |= (uint32_t)(uint8_t)(int8_t)v << (8 * y);
+        }
+        a.prof[x] = w;
+    }
+    a.A2 = (const uint32_t *)ctx->a2.p;
+    a.B2 = (const uint32_t *)ctx->b2.p;
+    a.err = d_err;
+    a.rowb = (int2 *)ctx->rowb.p;
+    a.progress = (int *)ctx->progress.p;
+    a.ticket = d_ticket;
+    a.k = (int)(nsp > 0 ? J.k : 0);
+    a.sp = (int *)ctx->sp.p;
+    a.sp_stride = stride;
+    a.sp_ld = ld;
+    a.row_done = ctx->flags_d;
+    a.gbest = d_gbest;
+    a.slots = (int4 *)ctx->slots.p;
+    a.goal = J.goal;
+    a.hit_key = d_hit_key;
+    a.hit_band = d_hit_band;
+    a.replays = d_replays;
+    {
+        void *args[] = {&a};
+        CK(cudaLaunchKernel(J.local ? V.local_fn : V.global_fn, dim3(grid), dim3(V.nw * 32 + 32), args, V.smem, st));
+    }
+    CK(cudaEventRecord(ctx->ev[2], st));
+    sw_reduce_kernel<<<1, 256, 0, st>>>((const int4 *)ctx->slots.p, grid, J.local ? 1 : 0, d_hit_key, J.goal, d_res);
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(ctx->res_h, d_res, sizeof(int4), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(ctx->res_h + 1, d_err, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(ctx->res_h + 2, d_replays, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    CK(cudaEventRecord(ctx->ev[3], st));
+
+    // stream special rows to the sink in ascending order while the fill runs
+    int sink_rc = 0;
+    long long bytes = 0;
+    for (long long q = 0; q < nsp; q++) {
+        volatile unsigned int *f = ctx->flags_h + q;
+        while (*f == 0) {
+            const cudaError_t qe = cudaEventQuery(ctx->ev[2]);
+            if (qe == cudaSuccess) {
+                if (*f == 0) {
+                    // fill finished without publishing: only legitimate on an alphabet error
+                    CK(cudaStreamSynchronize(st));
+                    if (ctx->res_h[1].x) return SW_EALPHABET;
+                    snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published", q);
+                    return SW_ECUDA;
+                }
+                break;
+            } else if (qe != cudaErrorNotReady) {
+                return cuda_fail(ctx, qe, "fill kernel");
+            }
+            std::this_thread::yield();
+        }
+        if (sink_rc) continue;  // aborted: drain flags, skip copies
+        const int32_t *src = (const int32_t *)ctx->sp.p + q * stride;
+        CK(cudaMemcpyAsync(ctx->stage_h, src, (size_t)n * 4, cudaMemcpyDeviceToHost, ctx->side));
+        CK(cudaMemcpyAsync(ctx->stage_h + ld, src + ld, (size_t)n * 4, cudaMemcpyDeviceToHost, ctx->side));
+        CK(cudaStreamSynchronize(ctx->side));
+        bytes += 8ll * n;
+        if (J.sink && J.sink(J.user, (q + 1) * J.k, ctx->stage_h, ctx->stage_h + ld, J.n)) sink_rc = SW_EABORTED;
+    }
+    CK(cudaStreamSynchronize(st));
+    if (ctx->res_h[1].x) return SW_EALPHABET;
+    if (sink_rc) return sink_rc;
+    *res = ctx->res_h[0];
+
+    float t01 = 0, t12 = 0, t23 = 0;
+    cudaEventElapsedTime(&t01, ctx->ev[0], ctx->ev[1]);
+    cudaEventElapsedTime(&t12, ctx->ev[1], ctx->ev[2]);
+    cudaEventElapsedTime(&t23, ctx->ev[2], ctx->ev[3]);
+    ctx->stats.encode_ms += t01;
+    ctx->stats.fill_ms += t12;
+    ctx->stats.reduce_ms += t23;
+    ctx->stats.kernel_launches += 3;
+    ctx->stats.replays += (long long)*(unsigned long long *)(ctx->res_h + 2);
+    ctx->stats.special_rows += nsp;
+    ctx->stats.special_bytes_d2h += bytes;
+    ctx->stats.alpha = V.alpha;
+    ctx->stats.warps = V.nw;
+    ctx->stats.width = W;
+    ctx->stats.grid = grid;
+    return SW_OK;
+}
+
+static int stage1_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const unsigned char *dB, int64_t n,
+                         int32_t ma, int32_t mi, int32_t go, int32_t ge, int64_t k, sw_row_sink sink, void *user,
+                         cudaStream_t us, sw_result *out)
+{
+    Job J{};
+    J.dA = dA; J.m = m; J.dB = dB; J.n = n;
+    J.revA = J.revB = false;
+    J.ma = ma; J.mi = mi; J.go = go; J.ge = ge;
+    J.k = k; J.sink = sink; J.user = user;
+    J.local = true;
+    J.goal = 0;
+    int4 r;
+    const int rc = run_job(ctx, J, us, &r);
+    if (rc) return rc;
+    out->score = r.x;
+    out->i = r.y;
+    out->j = r.z;
+    return SW_OK;
+}
+
+static bool valid_common(sw_ctx *ctx, int64_t m, int64_t n, int64_t k, sw_row_sink sink, sw_result *out)
+{
+    if (!ctx || !out || m < 0 || n < 0 || k < 0) return false;
+    if (m >= (1ll << 31) - 1024 || n >= (1ll << 31) - 1024) return false;
+    if (k > 0 && !sink) return false;
+    return true;
+}
+
+static int upload(sw_ctx *ctx, const char *A, int64_t m, const char *B, int64_t n)
+{
+    int rc = grow(ctx, ctx->seq, (size_t)(m + n + 16));
+    if (rc) return rc;
+    if (m) CK(cudaMemcpyAsync(ctx->seq.p, A, (size_t)m, cudaMemcpyHostToDevice, ctx->stream));
+    if (n) CK(cudaMemcpyAsync((char *)ctx->seq.p + m, B, (size_t)n, cudaMemcpyHostToDevice, ctx->stream));
+    return SW_OK;
+}
+
+static void begin_stats(sw_ctx *ctx) { ctx->stats = sw_stats{}; }
+
+extern "C" int sw_align_stage1(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, int64_t n, int32_t match,
+                               int32_t mismatch, int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
+                               sw_row_sink sink, void *user, sw_result *out)
+{
+    if (!valid_common(ctx, m, n, special_row_interval, sink, out)) return SW_EINVAL;
+    if ((m && !seqA) || (n && !seqB)) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    if (m == 0 || n == 0) {
+        out->score = 0; out->i = 0; out->j = 0;
+        return SW_OK;
+    }
+    CK(cudaEventRecord(ctx->ev[4], ctx->stream));
+    if ((rc = upload(ctx, seqA, m, seqB, n))) return rc;
+    rc = stage1_common(ctx, (const unsigned char *)ctx->seq.p, m, (const unsigned char *)ctx->seq.p + m, n, match,
+                       mismatch, gap_open, gap_ext, special_row_interval, sink, user, nullptr, out);
+    if (rc) return rc;
+    float up = 0;
+    cudaEventElapsedTime(&up, ctx->ev[4], ctx->ev[0]);
+    ctx->stats.upload_ms = up;
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return SW_OK;
+}
+
+extern "C" int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                                   int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                                   int64_t special_row_interval, sw_row_sink sink, void *user, void *stream,
+                                   sw_result *out)
+{
+    if (!valid_common(ctx, m, n, special_row_interval, sink, out)) return SW_EINVAL;
+    if ((m && !dseqA) || (n && !dseqB)) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    if (m == 0 || n == 0) {
+        out->score = 0; out->i = 0; out->j = 0;
+        return SW_OK;
+    }
+    rc = stage1_common(ctx, (const unsigned char *)dseqA, m, (const unsigned char *)dseqB, n, match, mismatch,
+                       gap_open, gap_ext, special_row_interval, sink, user, (cudaStream_t)stream, out);
+    if (rc) return rc;
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return SW_OK;
+}
+
+// Reverse pass.  Exact pruning: a cell (i', j')
+// of the reverse matrix scores at most pmax*min(i',j') - [i' != j'](G_open +
+// |i'-j'| G_ext), so a hit in rows <= L lies in columns <= J(L) = L +
+// (pmax*L - G_open - goal)/G_ext.  The rectangle [1..L] x [1..J(L)] is closed
+// under the recurrence's dependencies, so filling it exactly finds the first
+// hit among rows <= L; L grows geometrically until a hit appears or L = i_end.
+static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, const unsigned char *dB,
+                          int64_t j_end, int32_t ma, int32_t mi, int32_t go, int32_t ge, int32_t goal,
+                          sw_result *out)
+{
+    const long long pmax = std::max(ma, mi);
+    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0);
+    const long long BH = (long long)V.alpha * 32 * V.nw;
+    long long L = std::max<long long>(BH, pmax > 0 ? (goal + pmax - 1) / pmax : i_end);
+    for (;;) {
+        L = std::min<long long>(L, i_end);
+        long long Jc = j_end;
+        if (ge > 0 && pmax > 0) {
+            const long long slack = pmax * L - go - goal;
+            const long long jl = slack < 0 ? L : L + slack / ge;
+            Jc = std::min<long long>(j_end, std::max<long long>(jl, L));
+        }
+        Jc = std::min<long long>(Jc, j_end);
+        Job J{};
+        // reversed prefixes: row i' <-> S0[i_end - i'], column j' <-> S1[j_end - j'];
+        // restricting to the first L rows / Jc columns of the reversed strings means
+        // taking the LAST L (Jc) characters of the prefixes.
+        J.dA = dA + (i_end - L);
+        J.m = L;
+        J.dB = dB + (j_end - Jc);
+        J.n = Jc;
+        J.revA = J.revB = true;
+        J.ma = ma; J.mi = mi; J.go = go; J.ge = ge;
+        J.k = 0; J.sink = nullptr; J.user = nullptr;
+        J.local = false;
+        J.goal = goal;
+        int4 r;
+        const int rc = run_job(ctx, J, nullptr, &r);
+        if (rc) return rc;
+        if (r.w) {
+            out->score = goal;
+            out->i = i_end - r.y;
+            out->j = j_end - r.z;
+            return SW_OK;
+        }
+        if (L >= i_end) return SW_ENOTFOUND;  // the rectangle held every possible hit
+        L = std::min<long long>(i_end, L * 4);
+    }
+}
+
+extern "C" int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, const char *seqB, int64_t j_end,
+                               int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext, int32_t goal,
+                               sw_result *start_out)
+{
+    if (!ctx || !start_out || i_end < 0 || j_end < 0 || goal < 0) return SW_EINVAL;
+    if ((i_end && !seqA) || (j_end && !seqB)) return SW_EINVAL;
+    if (i_end >= (1ll << 31) - 1024 || j_end >= (1ll << 31) - 1024) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, i_end, j_end);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    if (goal == 0) {
+        start_out->score = 0; start_out->i = i_end; start_out->j = j_end;
+        return SW_OK;
+    }
+    if (i_end == 0 || j_end == 0) return SW_ENOTFOUND;
+    CK(cudaEventRecord(ctx->ev[4], ctx->stream));
+    if ((rc = upload(ctx, seqA, i_end, seqB, j_end))) return rc;
+    rc = reverse_common(ctx, (const unsigned char *)ctx->seq.p, i_end, (const unsigned char *)ctx->seq.p + i_end,
+                        j_end, match, mismatch, gap_open, gap_ext, goal, start_out);
+    if (rc) return rc;
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return SW_OK;
+}
+
+extern "C" int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end, const char *dseqB, int64_t j_end,
+                                   int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext, int32_t goal,
+                                   sw_result *start_out)
+{
+    if (!ctx || !start_out || i_end < 0 || j_end < 0 || goal < 0) return SW_EINVAL;
+    if ((i_end && !dseqA) || (j_end && !dseqB)) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, i_end, j_end);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    begin_stats(ctx);
+    if (goal == 0) {
+        start_out->score = 0; start_out->i = i_end; start_out->j = j_end;
+        return SW_OK;
+    }
+    if (i_end == 0 || j_end == 0) return SW_ENOTFOUND;
+    return reverse_common(ctx, (const unsigned char *)dseqA, i_end, (const unsigned char *)dseqB, j_end, match,
+                          mismatch, gap_open, gap_ext, goal, start_out);
+}

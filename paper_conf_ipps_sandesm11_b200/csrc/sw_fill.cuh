@@ -1,0 +1,477 @@
+// sw_fill.cuh -- sm_100a Stage-1 / reverse-pass matrix fill (CUDAlign 2.0,
+// Sandes & de Melo IPDPS 2011; P:<line> = /root/reference/PAPER.md line).
+//
+// What one launch computes: the Smith-Waterman/Gotoh recurrences Eq. 1-3
+// over all m x n cells in linear space, the best score with its
+// exact (min i, min j) end cell, and every k-th special row of
+// (H, F); or, in GLOBAL mode, the anchored global recurrence of
+// the reverse pass and its first cell equal to `goal`.
+//
+// B200 design (the paper's GT200 external-diagonal
+// launches, short/long phases and shifted bus are replaced):
+//  * Band = BH = ALPHA*32*NW consecutive rows.  One persistent CTA takes a band
+//    from an atomic ticket and sweeps ALL columns of it left to right; bands
+//    are taken in order, so a CTA only ever waits on a band owned by a running
+//    CTA (deadlock-free with any grid size).
+//  * Lane = ALPHA consecutive rows whose (E, t = H - G_first) live in
+//    registers; the substitution score p(i,j)+G_first for the lane's rows is a
+//    per-row int8x4 "profile" word selected with one PRMT per cell by the
+//    column's 2-bit code.  Lanes of a warp form a wavefront skewed by one column;
+//    (t, F) of a lane's bottom row passes to the next lane by SHFL, to the next
+//    warp through a shared-memory ring, to the next band through the row border
+//    in global memory (in place, n x 8 B), gated by a per-band progress counter
+//    (release/acquire at gpu scope).
+//  * Warps of a CTA are skewed by 2 tiles of W columns and advance in lockstep
+//    intervals separated by __syncthreads.  A dedicated I/O warp loads the top
+//    border and column codes one tile ahead and drains the bottom row one tile
+//    behind, publishing progress.
+//  * Best cell: a per-tile maximum (cheap); a warp replays a tile with exact
+//    (score, i, j) tracking only when some lane's tile maximum reaches the
+//    running threshold max(own best, global best hint, 1).  Any cell equal to
+//    the final best is therefore replayed, so the reported cell is exact.
+#pragma once
+#include <cstdint>
+#include <climits>
+#include <cuda_runtime.h>
+
+namespace swb {
+
+constexpr int NEG = -(1 << 30);            // E(i,0), F(0,j) = "-infinity" (reading S3)
+constexpr uint32_t PADPROF = 0x80808080u;  // profile of padding rows / padding column: -128
+
+struct FillArgs {
+    int m, n;            // real sizes (rows of S0, columns of S1)
+    int ncols_pad;       // n rounded up to a multiple of W
+    int NT;              // tiles each warp runs per band = ncols_pad / W + 1
+    int nb;              // number of bands
+    int go, ge, gf;      // G_open, G_ext, G_first = go + ge
+    uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
+    const uint32_t *A2;  // S0 codes, 2 bits each, 16 per word
+    const uint32_t *B2;  // S1 codes
+    const int *err;      // non-zero: encode found a bad byte -> do nothing
+    int2 *rowb;          // row border: (t, F) per column, >= NT*W + W entries
+    int *progress;       // per band: number of leading columns of its bottom row published
+    int *ticket;         // band ticket
+    // special rows (LOCAL only)
+    int k;               // interval (0 = none)
+    int *sp;             // device rows: slot q at sp + q*sp_stride: H[0..n), then F at + sp_ld
+    long long sp_stride;
+    int sp_ld;
+    unsigned int *row_done;  // mapped host flags, one per special row
+    // best (LOCAL) / goal (GLOBAL)
+    int *gbest;          // running best-score hint
+    int4 *slots;         // per-CTA (score, i, j, 0)
+    int goal;
+    unsigned long long *hit_key;  // min over hits of (i' << 32 | j')
+    int *hit_band;       // min band containing a hit
+    unsigned long long *replays;
+};
+
+__device__ __forceinline__ uint32_t col_sel(uint32_t code)  // code 0..3, 4 = pad
+{
+    const uint32_t s = code | 8u;  // PRMT: bit 3 of a selector nibble replicates the sign
+    return code | (s << 4) | (s << 8) | (s << 12);
+}
+
+__device__ __forceinline__ int prmt(uint32_t a, uint32_t b, uint32_t sel)
+{
+    int r;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+    return r;
+}
+
+__device__ __forceinline__ int ld_acquire(const int *p)
+{
+    int v;
+    asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ int ld_relaxed(const int *p)
+{
+    int v;
+    asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(int *p, int v)
+{
+    asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_sys(unsigned int *p, unsigned int v)
+{
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// (score, i, j) total order: higher score, then smaller i, then smaller j (reading S4)
+__device__ __forceinline__ bool better(int s, int i, int j, int bs, int bi, int bj)
+{
+    return s > bs || (s == bs && (i < bi || (i == bi && j < bj)));
+}
+
+template <int W, int NW>
+struct Smem {
+    static constexpr int RING = 4 * W;
+    static constexpr int SRING_MIN = 2 * NW * W + 32;
+    static constexpr int SRING = SRING_MIN <= 256 ? 256 : SRING_MIN <= 512 ? 512 : SRING_MIN <= 1024 ? 1024 : 2048;
+};
+
+template <int ALPHA, int NW, int W, bool LOCAL>
+struct Fill {
+    static constexpr int BH = ALPHA * 32 * NW;
+    static constexpr int RING = Smem<W, NW>::RING;
+    static constexpr int SRING = Smem<W, NW>::SRING;
+    static constexpr int NSAVE = 2 * ALPHA + 3;
+    static_assert(W % 32 == 0 && W >= 32, "W multiple of 32");
+    static_assert(ALPHA % 2 == 0 && ALPHA <= 16, "ALPHA even, <= 16");
+
+    static size_t smem_bytes()
+    {
+        return sizeof(int2) * RING * (NW + 1) + sizeof(uint32_t) * SRING + sizeof(int) * NSAVE * 32 * NW;
+    }
+
+    // ---------------------------------------------------------------- per-lane state
+    struct Lane {
+        uint32_t P[ALPHA];
+        int e[ALPHA];
+        int t[ALPHA];
+        int tprev;         // t of the row above this strip at the previous column (diagonal input)
+        int out_t, out_f;  // (t, F) of this strip's bottom row at the last column done
+        __device__ __forceinline__ void P_copy_from(const Lane &o)
+        {
+#pragma unroll
+            for (int r = 0; r < ALPHA; r++) P[r] = o.P[r];
+        }
+    };
+
+    // One column step of one lane (warp-synchronous).  k = warp step; the lane
+    // handles 0-based column j = k - lane.  TRACK: exact best/hit tracking.
+    // SPM: 0 = no special rows, 1 = special row is the strip's bottom row,
+    // 2 = special rows anywhere in the strip (bitmask).
+    template <bool GUARD, bool TRACK, int SPM>
+    static __device__ __forceinline__ int step(const FillArgs &a, Lane &L, int k, int lane, const int2 *ring_in,
+                                               int2 *ring_out, const uint32_t *selr, int tmax, int row1,
+                                               int &bs, int &bi, int &bj, int *sp_ptr, uint32_t smask)
+    {
+        int in_t = __shfl_up_sync(0xffffffffu, L.out_t, 1);
+        int in_f = __shfl_up_sync(0xffffffffu, L.out_f, 1);
+        const int j = k - lane;
+        if (lane == 0) {
+            const int2 v = ring_in[j & (RING - 1)];
+            in_t = v.x;
+            in_f = v.y;
+        }
+        if (GUARD && j < 0) return tmax;
+        const uint32_t sel = selr[j & (SRING - 1)];
+        int td = L.tprev;
+        L.tprev = in_t;
+        int tu = in_t, fu = in_f;
+        const int nge = -a.ge;
+        const int gf = a.gf;
+        int *spp = sp_ptr;
+#pragma unroll
+        for (int r = 0; r < ALPHA; r += 2) {
+            // row r: Eq. 2, Eq. 3, Eq. 1 (with p' = p + G_first applied to t = H - G_first)
+            L.e[r] = __viaddmax_s32(L.e[r], nge, L.t[r]);
+            fu = max(fu - a.ge, tu);
+            int p = prmt(L.P[r], PADPROF, sel);
+            int mx = max(L.e[r], fu);
+            int h0 = LOCAL ? __viaddmax_s32_relu(td, p, mx) : __viaddmax_s32(td, p, mx);
+            td = L.t[r];
+            L.t[r] = h0 - gf;
+            tu = L.t[r];
+            if (SPM == 2) {
+                if (smask & (1u << r)) {
+                    if (j < a.n) { spp[j] = h0; spp[a.sp_ld + j] = fu; }
+                    spp += a.sp_stride;
+                }
+            }
+            if (TRACK) {
+                const int row = row1 + r, col = j + 1;
+                if (row <= a.m && col <= a.n) {
+                    if (LOCAL) {
+                        if (better(h0, row, col, bs, bi, bj)) { bs = h0; bi = row; bj = col; }
+                    } else if (h0 == a.goal && (row < bi || (row == bi && col < bj))) {
+                        bi = row; bj = col;
+                    }
+                }
+            }
+            // row r + 1
+            L.e[r + 1] = __viaddmax_s32(L.e[r + 1], nge, L.t[r + 1]);
+            fu = max(fu - a.ge, tu);
+            p = prmt(L.P[r + 1], PADPROF, sel);
+            mx = max(L.e[r + 1], fu);
+            int h1 = LOCAL ? __viaddmax_s32_relu(td, p, mx) : __viaddmax_s32(td, p, mx);
+            td = L.t[r + 1];
+            L.t[r + 1] = h1 - gf;
+            tu = L.t[r + 1];
+            if (SPM == 2) {
+                if (smask & (2u << r)) {
+                    if (j < a.n) { spp[j] = h1; spp[a.sp_ld + j] = fu; }
+                    spp += a.sp_stride;
+                }
+            }
+            if (TRACK) {
+                const int row = row1 + r + 1, col = j + 1;
+                if (row <= a.m && col <= a.n) {
+                    if (LOCAL) {
+                        if (better(h1, row, col, bs, bi, bj)) { bs = h1; bi = row; bj = col; }
+                    } else if (h1 == a.goal && (row < bi || (row == bi && col < bj))) {
+                        bi = row; bj = col;
+                    }
+                }
+            }
+            tmax = __vimax3_s32(tmax, h0, h1);
+        }
+        L.out_t = tu;
+        L.out_f = fu;
+        if (SPM == 1 && sp_ptr != nullptr && j < a.n) {
+            sp_ptr[j] = tu + gf;  // H = t + G_first
+            sp_ptr[a.sp_ld + j] = fu;
+        }
+        if (!TRACK && lane == 31) ring_out[j & (RING - 1)] = make_int2(tu, fu);
+        return tmax;
+    }
+
+    template <bool GUARD, bool TRACK, int SPM>
+    static __device__ __noinline__ int tile(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
+                                            int2 *ring_out, const uint32_t *selr, int row1, int &bs, int &bi,
+                                            int &bj, int *sp_ptr, uint32_t smask)
+    {
+        int tmax = INT_MIN;
+        const int k0 = c * W;
+#pragma unroll 2
+        for (int kk = 0; kk < W; kk++)
+            tmax = step<GUARD, TRACK, SPM>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1, bs, bi, bj,
+                                           sp_ptr, smask);
+        return tmax;
+    }
+
+    // The hot path: no guard, no tracking, no special rows; inlined.
+    static __device__ __forceinline__ int tile_fast(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
+                                                    int2 *ring_out, const uint32_t *selr)
+    {
+        int tmax = INT_MIN;
+        int d0 = 0, d1 = 0, d2 = 0;
+        const int k0 = c * W;
+#pragma unroll 4
+        for (int kk = 0; kk < W; kk++)
+            tmax = step<false, false, 0>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, 0, d0, d1, d2, nullptr,
+                                         0u);
+        return tmax;
+    }
+
+    static __device__ __forceinline__ void save(const Lane &L, int *sv, int lane)
+    {
+#pragma unroll
+        for (int r = 0; r < ALPHA; r++) {
+            sv[r * 32 + lane] = L.e[r];
+            sv[(ALPHA + r) * 32 + lane] = L.t[r];
+        }
+        sv[(2 * ALPHA) * 32 + lane] = L.tprev;
+        sv[(2 * ALPHA + 1) * 32 + lane] = L.out_t;
+        sv[(2 * ALPHA + 2) * 32 + lane] = L.out_f;
+    }
+    static __device__ __forceinline__ void restore(Lane &L, const int *sv, int lane)
+    {
+#pragma unroll
+        for (int r = 0; r < ALPHA; r++) {
+            L.e[r] = sv[r * 32 + lane];
+            L.t[r] = sv[(ALPHA + r) * 32 + lane];
+        }
+        L.tprev = sv[(2 * ALPHA) * 32 + lane];
+        L.out_t = sv[(2 * ALPHA + 1) * 32 + lane];
+        L.out_f = sv[(2 * ALPHA + 2) * 32 + lane];
+    }
+};
+
+// Boundary values of row 0 / column 0 as t = H - G_first (reading S3, and the
+// global initialisation of reading S9): column index j is 0-based (DP j+1).
+template <bool LOCAL>
+__device__ __forceinline__ int2 top_boundary(const FillArgs &a, int j)
+{
+    if (LOCAL) return make_int2(-a.gf, NEG);
+    return make_int2(-(a.go + (j + 1) * a.ge) - a.gf, NEG);  // H(0, j+1) = -(G_open + (j+1) G_ext)
+}
+
+template <int ALPHA, int NW, int W, bool LOCAL>
+__global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a)
+{
+    using F = Fill<ALPHA, NW, W, LOCAL>;
+    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    int2 *rings = reinterpret_cast<int2 *>(smem_raw);                    // (NW+1) x RING
+    uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * RING);  // SRING
+    int *saves = reinterpret_cast<int *>(selr + SRING);                 // NW x NSAVE x 32
+    __shared__ int s_band, s_abort;
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    int bs = LOCAL ? 0 : 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
+    long long nrep = 0;
+    if (*a.err) return;
+
+    for (;;) {
+        if (threadIdx.x == 0) {
+            int b = atomicAdd(a.ticket, 1);
+            if (!LOCAL && b > ld_relaxed(a.hit_band)) b = a.nb;
+            s_band = b;
+            s_abort = 0;
+        }
+        __syncthreads();
+        const int b = s_band;
+        if (b >= a.nb) break;
+
+        typename F::Lane L;
+        const int row0 = b * BH + (warp * 32 + lane) * ALPHA;  // 0-based first row of the strip
+        int *sp_ptr = nullptr;
+        uint32_t smask = 0;
+        bool warp_sp = false;
+        if (warp < NW) {
+            const uint32_t w = row0 < a.m ? a.A2[row0 >> 4] : 0u;
+            const int sh = (row0 & 15) * 2;
+#pragma unroll
+            for (int r = 0; r < ALPHA; r++) {
+                const uint32_t code = (w >> (sh + 2 * r)) & 3u;
+                L.P[r] = (row0 + r < a.m) ? a.prof[code] : PADPROF;
+                L.e[r] = NEG;
+                L.t[r] = LOCAL ? -a.gf : -(a.go + (row0 + r + 1) * a.ge) - a.gf;  // H(i,0) - G_first
+            }
+            L.tprev = LOCAL ? -a.gf : (row0 == 0 ? -a.gf : -(a.go + row0 * a.ge) - a.gf);
+            L.out_t = 0;
+            L.out_f = 0;
+            if (LOCAL && a.k > 0) {
+                // special rows among DP rows row0+1 .. row0+ALPHA (<= m)
+                for (int r = 0; r < ALPHA; r++) {
+                    const int row = row0 + r + 1;
+                    if (row <= a.m && row % a.k == 0) smask |= 1u << r;
+                }
+                if (smask) {
+                    const int first = __ffs(smask) - 1;
+                    sp_ptr = a.sp + (long long)((row0 + first + 1) / a.k - 1) * a.sp_stride;
+                }
+            }
+            warp_sp = __any_sync(0xffffffffu, smask != 0);
+        }
+        const int spm = (a.k > 0 && a.k % ALPHA == 0) ? 1 : 2;
+
+        // prologue: I/O warp loads tile 0
+        auto io_load = [&](int c) {
+            const int need = min((c + 1) * W, a.NT * W - 31);
+            if (b > 0) {
+                if (lane == 0) {
+                    while (ld_acquire(a.progress + b - 1) < need) {
+                        if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
+                        __nanosleep(64);
+                    }
+                }
+                __syncwarp();
+            }
+            int2 *ring0 = rings;
+#pragma unroll
+            for (int x = lane; x < W; x += 32) {
+                const int col = c * W + x;
+                int2 v = (b == 0) ? top_boundary<LOCAL>(a, col) : __ldcg(a.rowb + col);
+                ring0[col & (RING - 1)] = v;
+                uint32_t code = 4u;
+                if (col < a.n) code = (__ldg(a.B2 + (col >> 4)) >> ((col & 15) * 2)) & 3u;
+                selr[col & (SRING - 1)] = col_sel(code);
+            }
+        };
+        auto io_drain = [&](int cd) {
+            const int2 *ringN = rings + NW * RING;
+#pragma unroll
+            for (int x = lane; x < W; x += 32) {
+                const int col = cd * W - 31 + x;
+                if (col >= 0) __stcg(a.rowb + col, ringN[col & (RING - 1)]);
+            }
+            __threadfence();
+            __syncwarp();
+            if (lane == 0) st_release(a.progress + b, cd * W + W - 31);
+        };
+
+        if (warp == NW) io_load(0);
+        __syncthreads();
+        const int S_END = a.NT + 2 * (NW - 1);
+        int *sv = saves + warp * F::NSAVE * 32;
+        for (int s = 0; s <= S_END; ++s) {
+            if (warp < NW) {
+                const int c = s - 2 * warp;
+                if (c >= 0 && c < a.NT) {
+                    const int2 *rin = rings + warp * RING;
+                    int2 *rout = rings + (warp + 1) * RING;
+                    int thr;
+                    if (LOCAL) thr = max(max(bs, ld_relaxed(a.gbest)), 1);
+                    else thr = a.goal;
+                    F::save(L, sv, lane);
+                    int tmax;
+                    if (c == 0 || warp_sp) {
+                        // slow tiles work on a copy so that L itself never has its address taken
+                        typename F::Lane T = L;
+                        if (!warp_sp) tmax = F::template tile<true, false, 0>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, nullptr, 0u);
+                        else if (spm == 1) tmax = F::template tile<true, false, 1>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, sp_ptr, smask);
+                        else tmax = F::template tile<true, false, 2>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, sp_ptr, smask);
+                        L = T;
+                    } else {
+                        tmax = F::tile_fast(a, L, c, lane, rin, rout, selr);
+                    }
+                    if (__any_sync(0xffffffffu, tmax >= thr)) {
+                        // exact replay of this tile from the saved state (rare)
+                        typename F::Lane T;
+                        F::restore(T, sv, lane);
+                        T.P_copy_from(L);
+                        const int obs = bs, obi = bi, obj = bj;
+                        F::template tile<true, true, 0>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, nullptr, 0u);
+                        if (lane == 0) nrep++;
+                        if (LOCAL) {
+                            if (bs > obs) atomicMax(a.gbest, bs);
+                        } else if (bi != obi || bj != obj) {
+                            atomicMin(a.hit_key, ((unsigned long long)(unsigned)bi << 32) | (unsigned)bj);
+                            atomicMin(a.hit_band, b);
+                        }
+                    }
+                }
+            } else {
+                if (s + 1 < a.NT) io_load(s + 1);
+                const int cd = s - 1 - 2 * (NW - 1);
+                if (cd >= 0) io_drain(cd);
+                if (!LOCAL && lane == 0 && ld_relaxed(a.hit_band) < b) s_abort = 1;
+            }
+            __syncthreads();
+            if (!LOCAL && s_abort) break;
+        }
+        if (warp == NW && lane == 0) st_release(a.progress + b, INT_MAX);
+        if (LOCAL && a.k > 0) {
+            // publish this band's special rows to the host
+            __threadfence();
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                const long long lo = (long long)b * BH + 1, hi = min((long long)(b + 1) * BH, (long long)a.m);
+                long long q = (lo + a.k - 1) / a.k;
+                if (q * a.k <= hi) {
+                    __threadfence_system();
+                    for (; q * a.k <= hi; q++) st_release_sys(a.row_done + (q - 1), 1u);
+                }
+            }
+        }
+    }
+
+    // ---------------------------------------------------------------- final per-CTA reduction
+    if (lane == 0 && nrep) atomicAdd(a.replays, (unsigned long long)nrep);
+    if (LOCAL) {
+        __shared__ int4 red[NW + 1];
+        for (int o = 16; o > 0; o >>= 1) {
+            const int s2 = __shfl_down_sync(0xffffffffu, bs, o);
+            const int i2 = __shfl_down_sync(0xffffffffu, bi, o);
+            const int j2 = __shfl_down_sync(0xffffffffu, bj, o);
+            if (better(s2, i2, j2, bs, bi, bj)) { bs = s2; bi = i2; bj = j2; }
+        }
+        if (lane == 0) red[warp] = make_int4(bs, bi, bj, 0);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int4 r = make_int4(0, 0, 0, 0);
+            for (int w = 0; w < NW; w++)
+                if (red[w].x > 0 && better(red[w].x, red[w].y, red[w].z, r.x, r.y, r.z)) r = red[w];
+            a.slots[blockIdx.x] = r;
+        }
+    }
+}
+
+}  // namespace swb

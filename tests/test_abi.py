@@ -1,0 +1,89 @@
+"""C-ABI checks that need no GPU: the shared library builds, loads, exports every
+symbol include/cudalign_b200.h declares, and its host-only helpers behave."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "cudalign_b200.h")
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_ipps_sandesm11_b200 import build, load_library
+
+    build.build()
+    return load_library()
+
+
+def declared_functions():
+    text = open(HEADER).read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    names = re.findall(r"^\s*(?:const\s+)?[A-Za-z_][A-Za-z0-9_]*\s*\*?\s*(sw_[a-z0-9_]+)\s*\(", text, flags=re.M)
+    return sorted(set(names))
+
+
+def test_header_declares_the_boundary():
+    names = declared_functions()
+    for want in ("sw_init", "sw_align_stage1", "sw_reverse_goal", "sw_row_granularity", "sw_shutdown", "sw_strerror"):
+        assert want in names
+
+
+def test_library_exports_every_declared_symbol(lib):
+    from paper_conf_ipps_sandesm11_b200 import EXPORTED
+
+    for name in declared_functions():
+        assert hasattr(lib, name), name
+        assert name in EXPORTED
+    # the .so is sm_100a code: the fatbin carries SASS for sm_100a
+    import subprocess
+
+    out = subprocess.run(["cuobjdump", "--list-elf", os.path.join(ROOT, "paper_conf_ipps_sandesm11_b200", "libcudalign_b200.so")],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_strerror(lib):
+    assert lib.sw_strerror(0) == b"ok"
+    assert b"ACGT" in lib.sw_strerror(-2)
+    assert lib.sw_strerror(-99) == b"unknown error"
+
+
+def test_null_and_bad_args(lib):
+    from paper_conf_ipps_sandesm11_b200 import SW_EINVAL
+
+    h = ctypes.c_void_p()
+    assert lib.sw_init(None, 1, ctypes.byref(h)) == SW_EINVAL
+    ids = (ctypes.c_int * 2)(0, 1)
+    assert lib.sw_init(ids, 2, ctypes.byref(h)) == SW_EINVAL  # round 1: one device per context
+    lib.sw_shutdown(None)  # no-op
+
+
+def test_init_without_gpu_fails_loudly(lib):
+    import torch
+
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    from paper_conf_ipps_sandesm11_b200 import Context, SwError
+
+    with pytest.raises(SwError):
+        Context(0)
+
+
+def test_flush_interval_helper_matches_table_viii(lib):
+    """sw_special_row_interval_for_budget implements the P:178 rule: Table VIII's
+    |L_2| is reproduced (exactly at 10/30/50 GiB) and it agrees with the oracle's
+    independent implementation."""
+    m, n, end_row = 32_799_110, 46_944_323, 32_718_231
+    printed = {10: 30, 20: 58, 30: 87, 40: 115, 50: 144}
+    for gib, l2 in printed.items():
+        R = lib.sw_special_row_interval_for_budget(m, n, 256, gib << 30)
+        assert R == oracle.flush_rows(m, n, 256, gib << 30)
+        pred = end_row // R + 2
+        assert pred == l2 if gib in (10, 30, 50) else abs(pred - l2) <= 1
+    assert lib.sw_special_row_interval_for_budget(0, 5, 256, 1) == 0
+    assert lib.sw_special_row_interval_for_budget(10, 10, 256, 1 << 40) == 256  # at least one block
