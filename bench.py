@@ -1,0 +1,353 @@
+#!/usr/bin/env python3
+"""bench.py -- CUDAlign 2.0 Stage-1 hot path on B200 (BASELINE.json metric).
+
+One step = the whole hot path of SURVEY.md 8(a) over one synthetic pair:
+encode/pack (a1) -> Stage-1 matrix fill with the exact best cell (a2-a5) ->
+every k-th special row (H, F) streamed to a host sink (a6) -> reverse goal
+pass to the start cell (a8).  GCUPS = m n / (t 10^9).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl ours|reference]
+
+N > 1 (torchrun, one process per GPU): round 1 runs one independent replica
+of the workload per GPU (weak scaling, no data-path collective); the
+column-stripe exchange of 8(e) is not built yet.
+
+--impl reference: the CPU oracle (oracle/, single-threaded plain C) timed on a
+bounded row-band sample of the same workload on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GCUPS at 1/2/4/8 B200 (33×47 MBP synthetic) + % of INT-pipe roofline"
+SCORING = (1, -3, 3, 2)  # match +1, mismatch -3, first gap -5 (G_open 3), extension -2
+# Paper Table IV 543K x 536K Stage 1 with flush (SRA 50M): 21,419 MCUPS on a GTX 285.
+PAPER_GCUPS = {"C2": 21.419}
+# Roofline: best instruction mix for one int32 cell update:
+# 3.5 half-rate (64 lanes/clk/SM) + 4 full-rate ops -> 17.07 cells/clk/SM.
+ROOF_CELLS_PER_CLK_SM = 17.07
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--workload", default=os.environ.get("SWB_WORKLOAD", "C2"))
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--k", type=int, default=None, help="special_row_interval override")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    return p.parse_args()
+
+
+# ---------------------------------------------------------------- clocks sampler
+
+class ClockSampler:
+    FIELDS = "clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown," \
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- oracle (CPU) timing
+
+def oracle_sample(A, B, k, target_s=12.0):
+    """Time the oracle's band recompute (the same loop as its Stage 1) on a
+    bounded sample of rows of the workload: single-threaded, as it stands."""
+    import numpy as np
+
+    import oracle
+
+    n = len(B)
+    # calibrate on a small band, then size the sample for ~target_s seconds
+    ma, mi, go, ge = SCORING
+    Htop = np.zeros(n + 1, np.int64)
+    Ftop = np.full(n + 1, oracle.NEG, np.int64)
+    r = max(1, int(2e8 // max(n, 1)))
+    t0 = time.perf_counter()
+    oracle.band(A, B, ma, mi, go, ge, 0, min(r, len(A)), Htop, Ftop)
+    dt = time.perf_counter() - t0
+    rate = (min(r, len(A)) * n) / max(dt, 1e-9)
+    rows = int(min(len(A), max(1, target_s * rate / n)))
+    t0 = time.perf_counter()
+    oracle.band(A, B, ma, mi, go, ge, 0, rows, Htop, Ftop)
+    dt = time.perf_counter() - t0
+    cells = rows * n
+    return cells / dt / 1e9, f"oracle.band rows 1..{rows} x all {n} columns of the workload ({cells:.3g} cells, {dt:.1f} s, 1 thread)", dt
+
+
+# ---------------------------------------------------------------- main
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    import numpy as np
+
+    import synth
+
+    cfg = synth.CONFIGS[args.workload]
+    k = cfg.k if args.k is None else args.k
+
+    if args.impl == "reference":
+        if rank != 0:
+            return 0  # rank 0 alone runs the CPU oracle
+        A, B = synth.make_pair(cfg)
+        import oracle
+
+        oracle.build()
+        vals, samples = [], ""
+        for _ in range(args.warmup):
+            oracle_sample(A, B, k, target_s=2.0)
+        times = []
+        for _ in range(args.steps):
+            v, samples, dt = oracle_sample(A, B, k, target_s=10.0)
+            vals.append(v)
+            times.append(dt)
+        value = statistics.median(vals)
+        line = {
+            "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GCUPS",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": {"workload": cfg.name, "m": cfg.m, "n": cfg.n, "k": k, "scoring": list(SCORING)},
+            "cpu_baseline": {"value": round(value, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": samples},
+            "e2e": {"value": round(value, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        }
+        print(json.dumps(line), flush=True)
+        return 0
+
+    import torch
+
+    if world > 1:
+        import torch.distributed as dist
+
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    else:
+        torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+
+    from paper_conf_ipps_sandesm11_b200 import Context, build
+
+    build.build()
+    A, B = synth.make_pair(cfg)
+    m, n = len(A), len(B)
+    dA = torch.from_numpy(A).to(dev)
+    dB = torch.from_numpy(B).to(dev)
+    stream = torch.cuda.current_stream(dev)
+    sptr = stream.cuda_stream
+    ctx = Context(local_rank)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    sink_rows = [0]
+
+    def sink(row, H, F):
+        sink_rows[0] += 1
+        return False
+
+    def step():
+        r, _ = ctx.align_stage1_dev(dA.data_ptr(), m, dB.data_ptr(), n, *SCORING, k=k, sink=sink, stream=sptr)
+        s1 = ctx.stats()
+        st = ctx.reverse_goal_dev(dA.data_ptr(), r.i, dB.data_ptr(), r.j, r.score, *SCORING, stream=sptr)
+        s2 = ctx.stats()
+        return r, st, s1, s2
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    fill_ms, launches, replays, sp_bytes = [], 0, 0, 0
+    results = set()
+    sink_rows[0] = 0
+    with ClockSampler(local_rank) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+        t_wall0 = time.perf_counter()
+        for s in range(args.steps):
+            flush.fill_(s & 0xFF)  # evict L2 between timed steps (outside the events)
+            ev[s][0].record(stream)
+            r, st, s1, s2 = step()
+            ev[s][1].record(stream)
+            fill_ms.append(s1["fill_ms"])
+            launches += s1["kernel_launches"] + s2["kernel_launches"]
+            replays += s1["replays"]
+            sp_bytes += s1["special_bytes_d2h"]
+            results.add((r.astuple(), st.astuple()))
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+        t_wall = time.perf_counter() - t_wall0
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    tot_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([tot_ms], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        tot_ms = float(t.item())
+    ms_per_step = tot_ms / args.steps
+    cells = float(m) * float(n)
+    value = world * cells / (ms_per_step * 1e-3) / 1e9
+    assert len(results) == 1, f"non-deterministic results {results}"
+    (best, start) = results.pop()
+    rows_per_step = sink_rows[0] // max(1, args.steps)
+
+    # ---- e2e through the host API from pinned host memory
+    e2e = None
+    if not args.no_e2e:
+        hA = torch.from_numpy(A).pin_memory()
+        hB = torch.from_numpy(B).pin_memory()
+        import ctypes
+
+        def e2e_step():
+            r, _ = ctx.align_stage1(np.ctypeslib.as_array((ctypes.c_uint8 * m).from_address(hA.data_ptr())),
+                                    np.ctypeslib.as_array((ctypes.c_uint8 * n).from_address(hB.data_ptr())),
+                                    *SCORING, k=k, sink=sink)
+            st = ctx.reverse_goal(np.ctypeslib.as_array((ctypes.c_uint8 * m).from_address(hA.data_ptr())), r.i,
+                                  np.ctypeslib.as_array((ctypes.c_uint8 * n).from_address(hB.data_ptr())), r.j,
+                                  r.score, *SCORING)
+            return r, st
+
+        e2e_step()
+        torch.cuda.synchronize()
+        ts = []
+        for s in range(args.steps):
+            flush.fill_(s & 0xFF)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            r, st = e2e_step()
+            ts.append(time.perf_counter() - t0)
+            assert (r.astuple(), st.astuple()) == (best, start)
+        e2e_s = sum(ts) / len(ts)
+        if world > 1:
+            t = torch.tensor([e2e_s], device=dev, dtype=torch.float64)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            e2e_s = float(t.item())
+        h2d = m + n + best[1] + best[2]
+        d2h = sp_bytes // args.steps + 3 * 16
+        e2e = {"value": round(world * cells / e2e_s / 1e9, 3), "unit": "GCUPS", "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": round(1e3 * e2e_s, 3)}
+
+    if rank != 0:
+        return 0
+
+    clocks = clk.summary()
+    # ---- roofline of the dominant kernel (the fill), from live CUDA events on its stream
+    fill_avg = statistics.mean(fill_ms)
+    achieved = cells / (fill_avg * 1e-3) / 1e9
+    sm_max = clocks.get("sm_max_mhz") or 1965.0
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        sm_max = float(peaks.get("sm_max_mhz", sm_max))
+    except Exception:
+        pass
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    peak = nsm * ROOF_CELLS_PER_CLK_SM * sm_max * 1e6 / 1e9
+    traffic = None
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        if tr.get("workload") == cfg.name:
+            traffic = tr.get("fill_dram_bytes_per_launch")
+    except Exception:
+        pass
+    roofline = {"bound": "alu", "achieved": round(achieved, 2), "peak": round(peak, 1), "unit": "GCUPS",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "peak_basis": f"{nsm} SM x {ROOF_CELLS_PER_CLK_SM} cells/clk/SM x {sm_max:.0f} MHz (measured pipe rates, DESIGN.md 5)",
+                "fill_ms": round(fill_avg, 3),
+                "peak_at_measured_clock": round(nsm * ROOF_CELLS_PER_CLK_SM * (clocks.get('sm_mhz') or sm_max) * 1e-3, 1)}
+
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        v, sample, _ = oracle_sample(A, B, k, target_s=12.0)
+        cpu = {"value": round(v, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": sample}
+
+    line = {
+        "metric": METRIC, "value": round(value, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": (round(value / PAPER_GCUPS[cfg.name], 2) if cfg.name in PAPER_GCUPS and world == 1 else None),
+        "dtype": "int32", "data": "synthetic",
+        "config": {"workload": cfg.name, "m": m, "n": n, "k": k, "scoring": list(SCORING),
+                   "step": "encode + Stage-1 fill + special rows to host sink + reverse goal pass",
+                   "l2": "flushed between timed steps (256 MiB write)",
+                   "parallelism": "single" if world == 1 else f"replicas x{world}",
+                   "kernel": {"alpha": s1["alpha"], "warps": s1["warps"], "width": s1["width"], "grid": s1["grid"]},
+                   "baseline_note": "vs_baseline = value / paper Table IV 543Kx536K flush (21.419 GCUPS, GTX 285, real DNA)"},
+        "result": {"best": list(best), "start": list(start), "special_rows_per_step": rows_per_step},
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "replays_per_step": replays // args.steps,
+        "clocks": clocks,
+        "wall_s_timed": round(t_wall, 3),
+    }
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

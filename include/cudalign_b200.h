@@ -99,8 +99,9 @@ int sw_align_stage1(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, 
 
 /* Same as sw_align_stage1 but the sequences are DEVICE pointers (bytes of
  * ACGTacgt already resident in HBM on the context's device) and the work is
- * ordered after `stream` (a cudaStream_t, or NULL for the library stream).
- * Returns when the result is on the host. */
+ * launched on `stream` (a cudaStream_t, or NULL for the library stream), so
+ * the caller's CUDA events on that stream bracket the kernels.  Special-row
+ * copies use the library's side stream.  Returns when the result is on the host. */
 int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
                         int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
                         int64_t special_row_interval, sw_row_sink sink, void *user, void *stream,
@@ -116,10 +117,11 @@ int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, const char *se
                     int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
                     int32_t goal, sw_result *start_out);
 
-/* sw_reverse_goal on DEVICE pointers (bytes of ACGTacgt resident in HBM). */
+/* sw_reverse_goal on DEVICE pointers (bytes of ACGTacgt resident in HBM),
+ * kernels launched on `stream` (a cudaStream_t, or NULL for the library's). */
 int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end, const char *dseqB, int64_t j_end,
                         int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
-                        int32_t goal, sw_result *start_out);
+                        int32_t goal, void *stream, sw_result *start_out);
 
 /* Rows per thread strip (alpha): special_row_interval multiples of this take
  * the fast special-row path. */

@@ -107,7 +107,7 @@ def load_library(path: str = LIB_PATH):
     lib.sw_align_stage1_dev.restype = ctypes.c_int
     lib.sw_reverse_goal.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, R]
     lib.sw_reverse_goal.restype = ctypes.c_int
-    lib.sw_reverse_goal_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, R]
+    lib.sw_reverse_goal_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, vp, R]
     lib.sw_reverse_goal_dev.restype = ctypes.c_int
     lib.sw_row_granularity.argtypes = [vp]
     lib.sw_row_granularity.restype = i64
@@ -221,9 +221,11 @@ class Context:
         self._check(rc, "sw_reverse_goal")
         return Result(out.score, out.i, out.j)
 
-    def reverse_goal_dev(self, dA_ptr, i_end, dB_ptr, j_end, goal, match=1, mismatch=-3, gap_open=3, gap_ext=2):
+    def reverse_goal_dev(self, dA_ptr, i_end, dB_ptr, j_end, goal, match=1, mismatch=-3, gap_open=3, gap_ext=2,
+                         stream: int = 0):
         out = _Result()
-        rc = self._lib.sw_reverse_goal_dev(self._h, dA_ptr, i_end, dB_ptr, j_end, match, mismatch, gap_open, gap_ext, goal, ctypes.byref(out))
+        rc = self._lib.sw_reverse_goal_dev(self._h, dA_ptr, i_end, dB_ptr, j_end, match, mismatch, gap_open, gap_ext,
+                                           goal, stream or None, ctypes.byref(out))
         self._check(rc, "sw_reverse_goal_dev")
         return Result(out.score, out.i, out.j)
 

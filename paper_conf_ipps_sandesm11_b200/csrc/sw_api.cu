@@ -118,9 +118,9 @@ static Variant make_variant()
 static const Variant &variant_for(int idx)
 {
     static const Variant vs[] = {
-        make_variant<16, 4, 32>(),
-        make_variant<16, 8, 32>(),
-        make_variant<8, 4, 32>(),
+        make_variant<16, 4, 64>(),
+        make_variant<16, 8, 64>(),
+        make_variant<8, 8, 64>(),
     };
     const int n = sizeof(vs) / sizeof(vs[0]);
     return vs[idx < 0 ? 0 : idx >= n ? n - 1 : idx];
@@ -364,12 +364,9 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         }
     }
 
-    cudaStream_t st = ctx->stream;
-    if (user_stream) {
-        // order our work after the caller's stream
-        CK(cudaEventRecord(ctx->ev[5], user_stream));
-        CK(cudaStreamWaitEvent(st, ctx->ev[5], 0));
-    }
+    // With a caller stream, every kernel of the call is launched on it (so the
+    // caller's CUDA events bracket them); otherwise on the library stream.
+    cudaStream_t st = user_stream ? user_stream : ctx->stream;
     char *misc = (char *)ctx->misc.p;
     int *d_err = (int *)(misc + 0);
     int *d_ticket = (int *)(misc + 4);
@@ -403,6 +400,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     a.go = J.go;
     a.ge = J.ge;
     a.gf = J.go + J.ge;
+    a.one = 1;
     for (int x = 0; x < 4; x++) {
         uint32_t w = 0;
         for (int y = 0; y < 4; y++) {
@@ -589,7 +587,7 @@ extern "C" int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, co
 // hit among rows <= L; L grows geometrically until a hit appears or L = i_end.
 static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, const unsigned char *dB,
                           int64_t j_end, int32_t ma, int32_t mi, int32_t go, int32_t ge, int32_t goal,
-                          sw_result *out)
+                          cudaStream_t us, sw_result *out)
 {
     const long long pmax = std::max(ma, mi);
     const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0);
@@ -618,7 +616,7 @@ static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, c
         J.local = false;
         J.goal = goal;
         int4 r;
-        const int rc = run_job(ctx, J, nullptr, &r);
+        const int rc = run_job(ctx, J, us, &r);
         if (rc) return rc;
         if (r.w) {
             out->score = goal;
@@ -651,7 +649,7 @@ extern "C" int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, con
     CK(cudaEventRecord(ctx->ev[4], ctx->stream));
     if ((rc = upload(ctx, seqA, i_end, seqB, j_end))) return rc;
     rc = reverse_common(ctx, (const unsigned char *)ctx->seq.p, i_end, (const unsigned char *)ctx->seq.p + i_end,
-                        j_end, match, mismatch, gap_open, gap_ext, goal, start_out);
+                        j_end, match, mismatch, gap_open, gap_ext, goal, nullptr, start_out);
     if (rc) return rc;
     ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     return SW_OK;
@@ -659,7 +657,7 @@ extern "C" int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, con
 
 extern "C" int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end, const char *dseqB, int64_t j_end,
                                    int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext, int32_t goal,
-                                   sw_result *start_out)
+                                   void *stream, sw_result *start_out)
 {
     if (!ctx || !start_out || i_end < 0 || j_end < 0 || goal < 0) return SW_EINVAL;
     if ((i_end && !dseqA) || (j_end && !dseqB)) return SW_EINVAL;
@@ -673,5 +671,5 @@ extern "C" int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end
     }
     if (i_end == 0 || j_end == 0) return SW_ENOTFOUND;
     return reverse_common(ctx, (const unsigned char *)dseqA, i_end, (const unsigned char *)dseqB, j_end, match,
-                          mismatch, gap_open, gap_ext, goal, start_out);
+                          mismatch, gap_open, gap_ext, goal, (cudaStream_t)stream, start_out);
 }

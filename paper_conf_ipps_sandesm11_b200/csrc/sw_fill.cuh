@@ -16,11 +16,13 @@
 //  * Lane = ALPHA consecutive rows whose (E, t = H - G_first) live in
 //    registers; the substitution score p(i,j)+G_first for the lane's rows is a
 //    per-row int8x4 "profile" word selected with one PRMT per cell by the
-//    column's 2-bit code.  Lanes of a warp form a wavefront skewed by one column;
-//    (t, F) of a lane's bottom row passes to the next lane by SHFL, to the next
-//    warp through a shared-memory ring, to the next band through the row border
-//    in global memory (in place, n x 8 B), gated by a per-band progress counter
-//    (release/acquire at gpu scope).
+//    column's 2-bit code.  A lane handles TWO columns per step, the second one
+//    row behind the first, so its vertical dependency chain (F -> H -> t ->
+//    next row) runs as two interleaved chains (ILP 2).  Lanes of a warp form
+//    a wavefront skewed by two columns; (t, F) of a lane's bottom row passes
+//    to the next lane by SHFL, to the next warp through a shared-memory ring,
+//    to the next band through the row border in global memory (in place,
+//    n x 8 B), gated by a per-band progress counter (release/acquire, gpu).
 //  * Warps of a CTA are skewed by 2 tiles of W columns and advance in lockstep
 //    intervals separated by __syncthreads.  A dedicated I/O warp loads the top
 //    border and column codes one tile ahead and drains the bottom row one tile
@@ -38,6 +40,7 @@ namespace swb {
 
 constexpr int NEG = -(1 << 30);            // E(i,0), F(0,j) = "-infinity" (reading S3)
 constexpr uint32_t PADPROF = 0x80808080u;  // profile of padding rows / padding column: -128
+constexpr int LANE_SKEW = 2;               // columns per lane step
 
 struct FillArgs {
     int m, n;            // real sizes (rows of S0, columns of S1)
@@ -45,6 +48,7 @@ struct FillArgs {
     int NT;              // tiles each warp runs per band = ncols_pad / W + 1
     int nb;              // number of bands
     int go, ge, gf;      // G_open, G_ext, G_first = go + ge
+    int one;             // always 1 (see imad())
     uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
     const uint32_t *A2;  // S0 codes, 2 bits each, 16 per word
     const uint32_t *B2;  // S1 codes
@@ -80,6 +84,15 @@ __device__ __forceinline__ int prmt(uint32_t a, uint32_t b, uint32_t sel)
     return r;
 }
 
+// x * one + y through the FMA pipe (IMAD); `one` is a runtime 1 so ptxas
+// cannot fold the add into an ALU-pipe VIADDMNMX.
+__device__ __forceinline__ int imad(int x, int one, int y)
+{
+    int r;
+    asm("mad.lo.s32 %0, %1, %2, %3;" : "=r"(r) : "r"(x), "r"(one), "r"(y));
+    return r;
+}
+
 __device__ __forceinline__ int ld_acquire(const int *p)
 {
     int v;
@@ -110,8 +123,8 @@ __device__ __forceinline__ bool better(int s, int i, int j, int bs, int bi, int 
 template <int W, int NW>
 struct Smem {
     static constexpr int RING = 4 * W;
-    static constexpr int SRING_MIN = 2 * NW * W + 32;
-    static constexpr int SRING = SRING_MIN <= 256 ? 256 : SRING_MIN <= 512 ? 512 : SRING_MIN <= 1024 ? 1024 : 2048;
+    static constexpr int SRING_MIN = 2 * NW * W + 2 * 32 * LANE_SKEW;
+    static constexpr int SRING = SRING_MIN <= 256 ? 256 : SRING_MIN <= 512 ? 512 : SRING_MIN <= 1024 ? 1024 : SRING_MIN <= 2048 ? 2048 : 4096;
 };
 
 template <int ALPHA, int NW, int W, bool LOCAL>
@@ -119,8 +132,10 @@ struct Fill {
     static constexpr int BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
     static constexpr int SRING = Smem<W, NW>::SRING;
-    static constexpr int NSAVE = 2 * ALPHA + 3;
-    static_assert(W % 32 == 0 && W >= 32, "W multiple of 32");
+    static constexpr int NSAVE = 2 * ALPHA + 5;
+    static constexpr int SKEW = 31 * LANE_SKEW;  // columns lane 31 lags lane 0
+    static constexpr int STEPS = W / LANE_SKEW;  // lane steps per tile
+    static_assert(W % 64 == 0 && W > SKEW, "W multiple of 64, larger than the warp skew");
     static_assert(ALPHA % 2 == 0 && ALPHA <= 16, "ALPHA even, <= 16");
 
     static size_t smem_bytes()
@@ -131,131 +146,130 @@ struct Fill {
     // ---------------------------------------------------------------- per-lane state
     struct Lane {
         uint32_t P[ALPHA];
-        int e[ALPHA];
-        int t[ALPHA];
-        int tprev;         // t of the row above this strip at the previous column (diagonal input)
-        int out_t, out_f;  // (t, F) of this strip's bottom row at the last column done
-        __device__ __forceinline__ void P_copy_from(const Lane &o)
-        {
-#pragma unroll
-            for (int r = 0; r < ALPHA; r++) P[r] = o.P[r];
-        }
+        int e[ALPHA];      // E(r, j-1) of the last column done
+        int t[ALPHA];      // t = H - G_first at (r, j-1)
+        int tprev;         // t of the row above this strip at the last column done (diagonal input)
+        int out_t0, out_f0, out_t1, out_f1;  // (t, F) of the strip's bottom row at the two last columns
     };
 
-    // One column step of one lane (warp-synchronous).  k = warp step; the lane
-    // handles 0-based column j = k - lane.  TRACK: exact best/hit tracking.
-    // SPM: 0 = no special rows, 1 = special row is the strip's bottom row,
+    // One lane step (warp-synchronous): the lane handles 0-based columns
+    // j0 = 2 (k - lane) and j0 + 1.  TRACK: exact best / first-hit tracking.
+    // SPM: 0 = no special rows, 1 = special rows are strip-bottom rows,
     // 2 = special rows anywhere in the strip (bitmask).
     template <bool GUARD, bool TRACK, int SPM>
     static __device__ __forceinline__ int step(const FillArgs &a, Lane &L, int k, int lane, const int2 *ring_in,
                                                int2 *ring_out, const uint32_t *selr, int tmax, int row1,
                                                int &bs, int &bi, int &bj, int *sp_ptr, uint32_t smask)
     {
-        int in_t = __shfl_up_sync(0xffffffffu, L.out_t, 1);
-        int in_f = __shfl_up_sync(0xffffffffu, L.out_f, 1);
-        const int j = k - lane;
+        int a_t = __shfl_up_sync(0xffffffffu, L.out_t0, 1);
+        int a_f = __shfl_up_sync(0xffffffffu, L.out_f0, 1);
+        int b_t = __shfl_up_sync(0xffffffffu, L.out_t1, 1);
+        int b_f = __shfl_up_sync(0xffffffffu, L.out_f1, 1);
+        const int j0 = LANE_SKEW * (k - lane);
         if (lane == 0) {
-            const int2 v = ring_in[j & (RING - 1)];
-            in_t = v.x;
-            in_f = v.y;
+            const int4 v = *reinterpret_cast<const int4 *>(ring_in + (j0 & (RING - 1)));
+            a_t = v.x; a_f = v.y; b_t = v.z; b_f = v.w;
         }
-        if (GUARD && j < 0) return tmax;
-        const uint32_t sel = selr[j & (SRING - 1)];
-        int td = L.tprev;
-        L.tprev = in_t;
-        int tu = in_t, fu = in_f;
+        if (GUARD && j0 < 0) return tmax;
+        const uint2 sl = *reinterpret_cast<const uint2 *>(selr + (j0 & (SRING - 1)));
+        int tdA = L.tprev;  // t(r0-1, j0-1)
+        int tdB = a_t;      // t(r0-1, j0)
+        L.tprev = b_t;
+        int tuA = a_t, fuA = a_f, tuB = b_t, fuB = b_f;
         const int nge = -a.ge;
         const int gf = a.gf;
         int *spp = sp_ptr;
 #pragma unroll
-        for (int r = 0; r < ALPHA; r += 2) {
-            // row r: Eq. 2, Eq. 3, Eq. 1 (with p' = p + G_first applied to t = H - G_first)
-            L.e[r] = __viaddmax_s32(L.e[r], nge, L.t[r]);
-            fu = max(fu - a.ge, tu);
-            int p = prmt(L.P[r], PADPROF, sel);
-            int mx = max(L.e[r], fu);
-            int h0 = LOCAL ? __viaddmax_s32_relu(td, p, mx) : __viaddmax_s32(td, p, mx);
-            td = L.t[r];
-            L.t[r] = h0 - gf;
-            tu = L.t[r];
+        for (int r = 0; r < ALPHA; r++) {
+            // column j0: Eq. 2, Eq. 3, Eq. 1 (p' = p + G_first applied to t = H - G_first).
+            // Instruction mix balanced over the ALU pipe (DPX max, PRMT) and the
+            // FMA pipe (the adds, as IMAD with a runtime 1): DESIGN.md section 5.
+            const int eA = __viaddmax_s32(L.e[r], nge, L.t[r]);
+            fuA = max(imad(fuA, a.one, nge), tuA);
+            const int pA = prmt(L.P[r], PADPROF, sl.x);
+            const int xA = imad(tdA, a.one, pA);
+            const int hA = LOCAL ? __vimax3_s32_relu(eA, fuA, xA) : __vimax3_s32(eA, fuA, xA);
+            tdA = L.t[r];
+            const int tA = imad(hA, a.one, -gf);
+            tuA = tA;
+            // column j0 + 1 (one row behind column j0 in the dependency chain)
+            const int eB = __viaddmax_s32(eA, nge, tA);
+            fuB = max(imad(fuB, a.one, nge), tuB);
+            const int pB = prmt(L.P[r], PADPROF, sl.y);
+            const int xB = imad(tdB, a.one, pB);
+            const int hB = LOCAL ? __vimax3_s32_relu(eB, fuB, xB) : __vimax3_s32(eB, fuB, xB);
+            tdB = tA;
+            const int tB = imad(hB, a.one, -gf);
+            tuB = tB;
+            L.e[r] = eB;
+            L.t[r] = tB;
+            tmax = __vimax3_s32(tmax, hA, hB);
             if (SPM == 2) {
                 if (smask & (1u << r)) {
-                    if (j < a.n) { spp[j] = h0; spp[a.sp_ld + j] = fu; }
+                    if (j0 < a.n) { spp[j0] = hA; spp[a.sp_ld + j0] = fuA; }
+                    if (j0 + 1 < a.n) { spp[j0 + 1] = hB; spp[a.sp_ld + j0 + 1] = fuB; }
                     spp += a.sp_stride;
                 }
             }
             if (TRACK) {
-                const int row = row1 + r, col = j + 1;
-                if (row <= a.m && col <= a.n) {
-                    if (LOCAL) {
-                        if (better(h0, row, col, bs, bi, bj)) { bs = h0; bi = row; bj = col; }
-                    } else if (h0 == a.goal && (row < bi || (row == bi && col < bj))) {
-                        bi = row; bj = col;
+                const int row = row1 + r;
+                if (row <= a.m) {
+                    if (j0 + 1 <= a.n) {
+                        if (LOCAL) {
+                            if (better(hA, row, j0 + 1, bs, bi, bj)) { bs = hA; bi = row; bj = j0 + 1; }
+                        } else if (hA == a.goal && (row < bi || (row == bi && j0 + 1 < bj))) {
+                            bi = row; bj = j0 + 1;
+                        }
+                    }
+                    if (j0 + 2 <= a.n) {
+                        if (LOCAL) {
+                            if (better(hB, row, j0 + 2, bs, bi, bj)) { bs = hB; bi = row; bj = j0 + 2; }
+                        } else if (hB == a.goal && (row < bi || (row == bi && j0 + 2 < bj))) {
+                            bi = row; bj = j0 + 2;
+                        }
                     }
                 }
             }
-            // row r + 1
-            L.e[r + 1] = __viaddmax_s32(L.e[r + 1], nge, L.t[r + 1]);
-            fu = max(fu - a.ge, tu);
-            p = prmt(L.P[r + 1], PADPROF, sel);
-            mx = max(L.e[r + 1], fu);
-            int h1 = LOCAL ? __viaddmax_s32_relu(td, p, mx) : __viaddmax_s32(td, p, mx);
-            td = L.t[r + 1];
-            L.t[r + 1] = h1 - gf;
-            tu = L.t[r + 1];
-            if (SPM == 2) {
-                if (smask & (2u << r)) {
-                    if (j < a.n) { spp[j] = h1; spp[a.sp_ld + j] = fu; }
-                    spp += a.sp_stride;
-                }
-            }
-            if (TRACK) {
-                const int row = row1 + r + 1, col = j + 1;
-                if (row <= a.m && col <= a.n) {
-                    if (LOCAL) {
-                        if (better(h1, row, col, bs, bi, bj)) { bs = h1; bi = row; bj = col; }
-                    } else if (h1 == a.goal && (row < bi || (row == bi && col < bj))) {
-                        bi = row; bj = col;
-                    }
-                }
-            }
-            tmax = __vimax3_s32(tmax, h0, h1);
         }
-        L.out_t = tu;
-        L.out_f = fu;
-        if (SPM == 1 && sp_ptr != nullptr && j < a.n) {
-            sp_ptr[j] = tu + gf;  // H = t + G_first
-            sp_ptr[a.sp_ld + j] = fu;
+        L.out_t0 = tuA; L.out_f0 = fuA;
+        L.out_t1 = tuB; L.out_f1 = fuB;
+        if (SPM == 1 && sp_ptr != nullptr) {
+            if (j0 < a.n) { sp_ptr[j0] = tuA + gf; sp_ptr[a.sp_ld + j0] = fuA; }  // H = t + G_first
+            if (j0 + 1 < a.n) { sp_ptr[j0 + 1] = tuB + gf; sp_ptr[a.sp_ld + j0 + 1] = fuB; }
         }
-        if (!TRACK && lane == 31) ring_out[j & (RING - 1)] = make_int2(tu, fu);
+        if (!TRACK && lane == 31) *reinterpret_cast<int4 *>(ring_out + (j0 & (RING - 1))) = make_int4(tuA, fuA, tuB, fuB);
         return tmax;
     }
 
+    // Rare tiles (tile 0 with its lane guard, exact replays, generic special
+    // rows): inlined so the lane state stays in registers, but not unrolled.
     template <bool GUARD, bool TRACK, int SPM>
-    static __device__ __noinline__ int tile(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
-                                            int2 *ring_out, const uint32_t *selr, int row1, int &bs, int &bi,
-                                            int &bj, int *sp_ptr, uint32_t smask)
+    static __device__ __forceinline__ int tile(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
+                                               int2 *ring_out, const uint32_t *selr, int row1, int &bs, int &bi,
+                                               int &bj, int *sp_ptr, uint32_t smask)
     {
         int tmax = INT_MIN;
-        const int k0 = c * W;
-#pragma unroll 2
-        for (int kk = 0; kk < W; kk++)
+        const int k0 = c * STEPS;
+#pragma unroll 1
+        for (int kk = 0; kk < STEPS; kk++)
             tmax = step<GUARD, TRACK, SPM>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1, bs, bi, bj,
                                            sp_ptr, smask);
         return tmax;
     }
 
-    // The hot path: no guard, no tracking, no special rows; inlined.
+    // The hot path: no guard, no tracking; SP1 = this warp holds special rows
+    // that are strip-bottom rows (k a multiple of ALPHA): predicated stores.
+    template <bool SP1>
     static __device__ __forceinline__ int tile_fast(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
-                                                    int2 *ring_out, const uint32_t *selr)
+                                                    int2 *ring_out, const uint32_t *selr, int *sp_ptr)
     {
         int tmax = INT_MIN;
         int d0 = 0, d1 = 0, d2 = 0;
-        const int k0 = c * W;
-#pragma unroll 4
-        for (int kk = 0; kk < W; kk++)
-            tmax = step<false, false, 0>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, 0, d0, d1, d2, nullptr,
-                                         0u);
+        const int k0 = c * STEPS;
+#pragma unroll 2
+        for (int kk = 0; kk < STEPS; kk++)
+            tmax = step<false, false, SP1 ? 1 : 0>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, 0, d0, d1, d2,
+                                                   sp_ptr, 0u);
         return tmax;
     }
 
@@ -267,8 +281,10 @@ struct Fill {
             sv[(ALPHA + r) * 32 + lane] = L.t[r];
         }
         sv[(2 * ALPHA) * 32 + lane] = L.tprev;
-        sv[(2 * ALPHA + 1) * 32 + lane] = L.out_t;
-        sv[(2 * ALPHA + 2) * 32 + lane] = L.out_f;
+        sv[(2 * ALPHA + 1) * 32 + lane] = L.out_t0;
+        sv[(2 * ALPHA + 2) * 32 + lane] = L.out_f0;
+        sv[(2 * ALPHA + 3) * 32 + lane] = L.out_t1;
+        sv[(2 * ALPHA + 4) * 32 + lane] = L.out_f1;
     }
     static __device__ __forceinline__ void restore(Lane &L, const int *sv, int lane)
     {
@@ -278,8 +294,10 @@ struct Fill {
             L.t[r] = sv[(ALPHA + r) * 32 + lane];
         }
         L.tprev = sv[(2 * ALPHA) * 32 + lane];
-        L.out_t = sv[(2 * ALPHA + 1) * 32 + lane];
-        L.out_f = sv[(2 * ALPHA + 2) * 32 + lane];
+        L.out_t0 = sv[(2 * ALPHA + 1) * 32 + lane];
+        L.out_f0 = sv[(2 * ALPHA + 2) * 32 + lane];
+        L.out_t1 = sv[(2 * ALPHA + 3) * 32 + lane];
+        L.out_f1 = sv[(2 * ALPHA + 4) * 32 + lane];
     }
 };
 
@@ -296,15 +314,15 @@ template <int ALPHA, int NW, int W, bool LOCAL>
 __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a)
 {
     using F = Fill<ALPHA, NW, W, LOCAL>;
-    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH;
+    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    int2 *rings = reinterpret_cast<int2 *>(smem_raw);                    // (NW+1) x RING
+    int2 *rings = reinterpret_cast<int2 *>(smem_raw);                        // (NW+1) x RING
     uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * RING);  // SRING
-    int *saves = reinterpret_cast<int *>(selr + SRING);                 // NW x NSAVE x 32
+    int *saves = reinterpret_cast<int *>(selr + SRING);                     // NW x NSAVE x 32
     __shared__ int s_band, s_abort;
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    int bs = LOCAL ? 0 : 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
+    int bs = 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
     long long nrep = 0;
     if (*a.err) return;
 
@@ -335,8 +353,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
                 L.t[r] = LOCAL ? -a.gf : -(a.go + (row0 + r + 1) * a.ge) - a.gf;  // H(i,0) - G_first
             }
             L.tprev = LOCAL ? -a.gf : (row0 == 0 ? -a.gf : -(a.go + row0 * a.ge) - a.gf);
-            L.out_t = 0;
-            L.out_f = 0;
+            L.out_t0 = L.out_f0 = L.out_t1 = L.out_f1 = 0;
             if (LOCAL && a.k > 0) {
                 // special rows among DP rows row0+1 .. row0+ALPHA (<= m)
                 for (int r = 0; r < ALPHA; r++) {
@@ -352,9 +369,8 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
         }
         const int spm = (a.k > 0 && a.k % ALPHA == 0) ? 1 : 2;
 
-        // prologue: I/O warp loads tile 0
         auto io_load = [&](int c) {
-            const int need = min((c + 1) * W, a.NT * W - 31);
+            const int need = min((c + 1) * W, a.NT * W - SKEW);
             if (b > 0) {
                 if (lane == 0) {
                     while (ld_acquire(a.progress + b - 1) < need) {
@@ -379,12 +395,12 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
             const int2 *ringN = rings + NW * RING;
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
-                const int col = cd * W - 31 + x;
+                const int col = cd * W - SKEW + x;
                 if (col >= 0) __stcg(a.rowb + col, ringN[col & (RING - 1)]);
             }
             __threadfence();
             __syncwarp();
-            if (lane == 0) st_release(a.progress + b, cd * W + W - 31);
+            if (lane == 0) st_release(a.progress + b, cd * W + W - SKEW);
         };
 
         if (warp == NW) io_load(0);
@@ -402,23 +418,18 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
                     else thr = a.goal;
                     F::save(L, sv, lane);
                     int tmax;
-                    if (c == 0 || warp_sp) {
-                        // slow tiles work on a copy so that L itself never has its address taken
-                        typename F::Lane T = L;
-                        if (!warp_sp) tmax = F::template tile<true, false, 0>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, nullptr, 0u);
-                        else if (spm == 1) tmax = F::template tile<true, false, 1>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, sp_ptr, smask);
-                        else tmax = F::template tile<true, false, 2>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, sp_ptr, smask);
-                        L = T;
+                    if (c == 0 || (warp_sp && spm == 2)) {
+                        tmax = F::template tile<true, false, 2>(a, L, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, sp_ptr, smask);
+                    } else if (warp_sp) {
+                        tmax = F::template tile_fast<true>(a, L, c, lane, rin, rout, selr, sp_ptr);
                     } else {
-                        tmax = F::tile_fast(a, L, c, lane, rin, rout, selr);
+                        tmax = F::template tile_fast<false>(a, L, c, lane, rin, rout, selr, nullptr);
                     }
                     if (__any_sync(0xffffffffu, tmax >= thr)) {
                         // exact replay of this tile from the saved state (rare)
-                        typename F::Lane T;
-                        F::restore(T, sv, lane);
-                        T.P_copy_from(L);
+                        F::restore(L, sv, lane);
                         const int obs = bs, obi = bi, obj = bj;
-                        F::template tile<true, true, 0>(a, T, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, nullptr, 0u);
+                        F::template tile<true, true, 0>(a, L, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, nullptr, 0u);
                         if (lane == 0) nrep++;
                         if (LOCAL) {
                             if (bs > obs) atomicMax(a.gbest, bs);
@@ -437,7 +448,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
             __syncthreads();
             if (!LOCAL && s_abort) break;
         }
-        if (warp == NW && lane == 0) st_release(a.progress + b, INT_MAX);
+        if (warp == NW && lane == 0 && !s_abort) st_release(a.progress + b, INT_MAX);
         if (LOCAL && a.k > 0) {
             // publish this band's special rows to the host
             __threadfence();
