@@ -115,6 +115,8 @@ static Variant make_variant()
     return v;
 }
 
+static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
+
 static const Variant &variant_for(int idx)
 {
     static const Variant vs[] = {
@@ -249,7 +251,7 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
 extern "C" int64_t sw_row_granularity(const sw_ctx *ctx)
 {
     if (!ctx) return 0;
-    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0).alpha;
+    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT).alpha;
 }
 
 extern "C" int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int64_t bh, int64_t sra_bytes)
@@ -304,7 +306,7 @@ struct Job {
 
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
 {
-    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0);
+    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT);
     const int W = V.w;
     const int BH = V.alpha * 32 * V.nw;
     const int m = (int)J.m, n = (int)J.n;
@@ -590,7 +592,7 @@ static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, c
                           cudaStream_t us, sw_result *out)
 {
     const long long pmax = std::max(ma, mi);
-    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : 0);
+    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT);
     const long long BH = (long long)V.alpha * 32 * V.nw;
     long long L = std::max<long long>(BH, pmax > 0 ? (goal + pmax - 1) / pmax : i_end);
     for (;;) {

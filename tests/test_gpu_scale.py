@@ -1,0 +1,114 @@
+"""Parity at BASELINE.json sizes, in the launch configuration bench.py times.
+
+The oracle cannot redo 1e11-1e13 cells in one thread inside a test, so the
+GPU's output is checked by band induction:
+row 0 is trivially correct; for every band [r, r + k) the oracle recomputes
+rows r+1..r+k from the GPU's special row r and must reproduce the GPU's
+special row r + k bit for bit, and the band maxima (oracle-computed) combine
+under (max, min i, min j) into the GPU's best cell.  Bands run in parallel on
+the host cores.  C2 is checked completely (every row, the global best); C3 is
+checked on a seeded sample of bands plus the band that holds the end cell.
+"""
+import multiprocessing as mp
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+PAPER = (1, -3, 3, 2)
+
+_G = {}
+
+
+def _band_job(args):
+    q, r0, r1 = args
+    A, B, rows = _G["A"], _G["B"], _G["rows"]
+    n = len(B)
+    if r0 == 0:
+        Ht = np.zeros(n + 1, np.int64)
+        Ft = np.full(n + 1, oracle.NEG, np.int64)
+    else:
+        h, f = rows[r0]
+        Ht = np.concatenate([[0], h.astype(np.int64)])
+        Ft = np.concatenate([[oracle.NEG], f.astype(np.int64)])
+    Hb, Fb, best = oracle.band(A, B, *PAPER, r0, r1, Ht, Ft)
+    ok = True
+    if r1 in rows:
+        h, f = rows[r1]
+        ok = bool(np.array_equal(Hb[1:], h) and np.array_equal(Fb[1:], f))
+    return q, ok, best
+
+
+def _run_bands(A, B, rows, jobs):
+    _G.update(A=A.tobytes(), B=B.tobytes(), rows=rows)
+    oracle.build()
+    ctx = mp.get_context("fork")
+    with ctx.Pool(min(len(jobs), os.cpu_count() or 4)) as pool:
+        return pool.map(_band_job, jobs, chunksize=1)
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    from paper_conf_ipps_sandesm11_b200 import Context, build
+
+    build.build()
+    c = Context(0)
+    yield c
+    c.close()
+
+
+def test_c2_full_band_induction(ctx):
+    """BASELINE configs[1] (543K x 536K, k = 4096): every special row and the
+    best cell, bit-exact, plus the reverse-pass start cell."""
+    cfg = synth.CONFIGS["C2"]
+    A, B = synth.make_pair(cfg)
+    rows = {}
+
+    def sink(row, H, F):
+        rows[row] = (H.copy(), F.copy())
+
+    got, _ = ctx.align_stage1(A, B, *PAPER, k=cfg.k, sink=sink)
+    assert sorted(rows) == list(range(cfg.k, cfg.m + 1, cfg.k))
+    bounds = list(range(0, cfg.m, cfg.k)) + [cfg.m]
+    jobs = [(q, bounds[q], bounds[q + 1]) for q in range(len(bounds) - 1)]
+    res = _run_bands(A, B, rows, jobs)
+    assert all(ok for _, ok, _ in res), [q for q, ok, _ in res if not ok]
+    bests = [b for _, _, b in res if b[0] > 0]
+    want = max(bests, key=lambda x: (x[0], -x[1], -x[2]))
+    assert got.astuple() == want
+    # the reverse pass from the end cell, against the oracle
+    st = ctx.reverse_goal(A, got.i, B, got.j, got.score, *PAPER)
+    assert st.astuple() == oracle.reverse_goal(A.tobytes(), got.i, B.tobytes(), got.j, *PAPER, got.score)
+    assert (st.i, st.j) == (cfg.params["a0"], cfg.params["b0"])  # the planted segment's start (Table III shape)
+
+
+@pytest.mark.skipif(not os.environ.get("SWB_SLOW"), reason="set SWB_SLOW=1 (several minutes of host CPU)")
+def test_c3_sampled_band_induction(ctx):
+    cfg = synth.CONFIGS["C3"]
+    A, B = synth.make_pair(cfg)
+    k = 2048  # verification spacing (the kernel configuration is the bench's)
+    rng = np.random.default_rng(3)
+    nbands = cfg.m // k
+    sample = set(int(x) for x in rng.choice(nbands, size=12, replace=False))
+    sample.update({nbands - 1, nbands})  # the last full band and the ragged tail (holds the end cell)
+    keep = set()
+    for q in sample:
+        keep.update({q * k, (q + 1) * k})
+    rows = {}
+
+    def sink(row, H, F):
+        if row in keep:
+            rows[row] = (H.copy(), F.copy())
+
+    got, _ = ctx.align_stage1(A, B, *PAPER, k=k, sink=sink)
+    jobs = [(q, q * k, min((q + 1) * k, cfg.m)) for q in sorted(sample) if q * k < cfg.m]
+    res = _run_bands(A, B, rows, jobs)
+    assert all(ok for _, ok, _ in res), [q for q, ok, _ in res if not ok]
+    qe = (got.i - 1) // k
+    assert qe in sample
+    band_best = {q: b for q, _, b in res}[qe]
+    assert band_best == got.astuple()

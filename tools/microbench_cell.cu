@@ -112,6 +112,86 @@ __global__ void kern(int *out, const uint32_t *prof, const uint32_t *sels, int g
     if (threadIdx.x == 0) cyc[blockIdx.x] = c1 - c0;
 }
 
+// Packed 16x2: each 32-bit register holds (row i, col j) and (row i+8, col j-1)
+// as biased unsigned 16-bit values; adds via IMAD (carry-free: halves stay in
+// [0, 65535]), maxima via VIMNMX(3).U16x2.  8 packed slots = 16 rows.
+template <int F>
+__global__ void kernp(int *out, const uint32_t *prof, const uint32_t *sels, int ge, int gf, int one, long long *cyc)
+{
+    uint32_t P[8], Q[8];
+    uint32_t e[8], t[8];
+    const uint32_t nge2 = (uint32_t)(0x10000 - ge) * 0x10001u;  // unused (adds of negatives avoided)
+    (void)nge2;
+    const uint32_t ge2 = (uint32_t)ge * 0x10001u, gf2 = (uint32_t)gf * 0x10001u, fl2 = 0x40004000u;
+#pragma unroll
+    for (int r = 0; r < 8; r++) {
+        P[r] = prof[(threadIdx.x + r) & 15];
+        Q[r] = prof[(threadIdx.x + r + 8) & 15];
+        e[r] = 0x40004000u;
+        t[r] = 0x40004000u;
+    }
+    uint32_t tprev = 0x40004000u, ot = 0x40004000u, of = 0x40004000u, tmax = 0;
+    long long c0 = clock64();
+    for (int k = 0; k < STEPS; k++) {
+        uint32_t up_t = __shfl_up_sync(0xffffffffu, ot, 1);
+        uint32_t up_f = __shfl_up_sync(0xffffffffu, of, 1);
+        const uint32_t sel = sels[k & 63];
+        // slot-0 inputs: lo half = upper lane's hi half, hi half = own slot-7 lo half
+        uint32_t tu = __byte_perm(up_t, t[7], 0x5432);
+        uint32_t fu = __byte_perm(up_f, of, 0x5432);
+        uint32_t td = tprev;
+        tprev = tu;
+#pragma unroll
+        for (int r = 0; r < 8; r++) {
+            // E: a = max(e - ge, t_left)
+            uint32_t ea = __vmaxu2(e[r] - ge2, t[r]);
+            // F: max(fu - ge, tu)
+            fu = __vmaxu2(fu - ge2, tu);
+            uint32_t p = prmt(P[r], Q[r], sel);
+            uint32_t x = (uint32_t)imad((int)td, one, (int)p);
+            uint32_t h = __vimax3_u16x2(ea, fu, x);
+            if (F == 1) h = __vmaxu2(h, fl2);
+            td = t[r];
+            uint32_t tt = (uint32_t)imad((int)h, one, -(int)gf2);
+            tu = tt;
+            e[r] = ea;
+            t[r] = tt;
+            if (r & 1) tmax = __vimax3_u16x2(tmax, h, tt);
+        }
+        ot = tu;
+        of = fu;
+    }
+    long long c1 = clock64();
+    uint32_t s = tmax ^ ot ^ of;
+#pragma unroll
+    for (int r = 0; r < 8; r++) s ^= e[r] + t[r];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+    if (threadIdx.x == 0) cyc[blockIdx.x] = c1 - c0;
+}
+
+template <int F>
+void runp(int sms, int threads, int ctas, const uint32_t *prof, const uint32_t *sels)
+{
+    int grid = sms * ctas;
+    int *out;
+    long long *cyc;
+    cudaMalloc(&out, sizeof(int) * grid * threads);
+    cudaMalloc(&cyc, sizeof(long long) * grid);
+    kernp<F><<<grid, threads>>>(out, prof, sels, 2, 5, 1, cyc);
+    cudaDeviceSynchronize();
+    kernp<F><<<grid, threads>>>(out, prof, sels, 2, 5, 1, cyc);
+    cudaDeviceSynchronize();
+    long long *h = new long long[grid];
+    cudaMemcpy(h, cyc, sizeof(long long) * grid, cudaMemcpyDeviceToHost);
+    long long mx = 0;
+    for (int i = 0; i < grid; i++) mx = h[i] > mx ? h[i] : mx;
+    double cells = (double)grid * threads * STEPS * 16;
+    printf("P%d threads=%4d ctas/sm=%d  cells/clk/SM=%6.2f\n", F, threads, ctas, cells / sms / mx);
+    delete[] h;
+    cudaFree(out);
+    cudaFree(cyc);
+}
+
 template <int F>
 void run(int sms, int threads, int ctas, const uint32_t *prof, const uint32_t *sels)
 {
@@ -162,6 +242,8 @@ int main()
         run<1>(sms, w, 1, prof, sels);
         run<2>(sms, w, 1, prof, sels);
         run<3>(sms, w, 1, prof, sels);
+        runp<0>(sms, w, 1, prof, sels);
+        runp<1>(sms, w, 1, prof, sels);
     }
     return 0;
 }
