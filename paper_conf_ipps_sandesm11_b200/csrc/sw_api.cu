@@ -140,7 +140,8 @@ struct sw_ctx {
     int num_sms = 0;
     cudaStream_t stream = nullptr, side = nullptr;
     cudaEvent_t ev[6] = {};
-    DevBuf seq, a2, b2, rowb, progress, misc, slots, sp;
+    DevBuf seq, a2, b2, rowb, progress, misc, slots, sp, dbg;
+    int dbg_n = 0;
     unsigned int *flags_h = nullptr, *flags_d = nullptr;
     size_t flags_cap = 0;
     int32_t *stage_h = nullptr;
@@ -236,7 +237,7 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->side) cudaStreamSynchronize(ctx->side);
-    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->rowb, &ctx->progress, &ctx->misc, &ctx->slots, &ctx->sp})
+    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->rowb, &ctx->progress, &ctx->misc, &ctx->slots, &ctx->sp, &ctx->dbg})
         if (b->p) cudaFree(b->p);
     if (ctx->flags_h) cudaFreeHost(ctx->flags_h);
     if (ctx->stage_h) cudaFreeHost(ctx->stage_h);
@@ -263,6 +264,15 @@ extern "C" int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int6
     unsigned __int128 q = (num + den - 1) / den;
     if (q < 1) q = 1;
     return (int64_t)(bh * (int64_t)q);
+}
+
+// Debug: copy the per-band timestamps of the last fill (SWB_DEBUG_TIMES set).
+extern "C" int64_t swb_debug_times(sw_ctx *ctx, unsigned long long *out, int64_t cap)
+{
+    if (!ctx || !ctx->dbg.p || !out) return 0;
+    const int64_t n = std::min<int64_t>(cap, (int64_t)ctx->dbg_n * 80);
+    cudaMemcpy(out, ctx->dbg.p, n * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+    return n;
 }
 
 extern "C" int sw_get_stats(const sw_ctx *ctx, sw_stats *out)
@@ -428,6 +438,14 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     a.hit_key = d_hit_key;
     a.hit_band = d_hit_band;
     a.replays = d_replays;
+    a.dbg = nullptr;
+    a.force_slow = getenv("SWB_FORCE_SLOW") ? 1 : 0;
+    if (getenv("SWB_DEBUG_TIMES")) {
+        if ((rc = grow(ctx, ctx->dbg, (size_t)nb * 80 * sizeof(unsigned long long)))) return rc;
+        CK(cudaMemsetAsync(ctx->dbg.p, 0, (size_t)nb * 80 * sizeof(unsigned long long), st));
+        a.dbg = (unsigned long long *)ctx->dbg.p;
+        ctx->dbg_n = nb;
+    }
     {
         void *args[] = {&a};
         CK(cudaLaunchKernel(J.local ? V.local_fn : V.global_fn, dim3(grid), dim3(V.nw * 32 + 32), args, V.smem, st));

@@ -69,7 +69,16 @@ struct FillArgs {
     unsigned long long *hit_key;  // min over hits of (i' << 32 | j')
     int *hit_band;       // min band containing a hit
     unsigned long long *replays;
+    int force_slow;           // unused (kept for ABI of FillArgs between host and kernels)
+    unsigned long long *dbg;  // optional: per band 80 x %globaltimer; slot 0 band start, 1 first tile, 15 band end
 };
+
+__device__ __forceinline__ unsigned long long gtimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 
 __device__ __forceinline__ uint32_t col_sel(uint32_t code)  // code 0..3, 4 = pad
 {
@@ -336,6 +345,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
         __syncthreads();
         const int b = s_band;
         if (b >= a.nb) break;
+        if (a.dbg && threadIdx.x == 0) a.dbg[80 * b] = gtimer();
 
         typename F::Lane L;
         const int row0 = b * BH + (warp * 32 + lane) * ALPHA;  // 0-based first row of the strip
@@ -405,6 +415,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
 
         if (warp == NW) io_load(0);
         __syncthreads();
+        if (a.dbg && threadIdx.x == 0) a.dbg[80 * b + 1] = gtimer();
         const int S_END = a.NT + 2 * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s <= S_END; ++s) {
@@ -449,6 +460,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
             if (!LOCAL && s_abort) break;
         }
         if (warp == NW && lane == 0 && !s_abort) st_release(a.progress + b, INT_MAX);
+        if (a.dbg && threadIdx.x == 0) a.dbg[80 * b + 15] = gtimer();
         if (LOCAL && a.k > 0) {
             // publish this band's special rows to the host
             __threadfence();

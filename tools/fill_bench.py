@@ -12,6 +12,26 @@ import torch  # noqa: E402
 import synth  # noqa: E402
 
 
+def band_times(ctx):
+    """Per-band timestamps (needs SWB_DEBUG_TIMES=1): returns an (nb, 4) array in us."""
+    import ctypes
+
+    import numpy as np
+
+    lib = ctx._lib
+    lib.swb_debug_times.restype = ctypes.c_int64
+    buf = (ctypes.c_uint64 * (80 * 40000))()
+    n = lib.swb_debug_times(ctx._h, buf, len(buf))
+    raw = np.frombuffer(buf, dtype=np.uint64, count=n).reshape(-1, 80)
+    for i in (0, 1, len(raw) // 2):
+        print("   band", i, "replays", raw[i, 9], "thr/tmax per warp,unit:", [(int(x >> 32), int(x & 0xffffffff) - (1 << 32 if (x & 0xffffffff) >= (1 << 31) else 0)) for x in raw[i, 64:80]])
+    a = raw[:, :64].astype(np.float64)
+    a[:, 9] = 0
+    t0 = a[a > 1e12].min()
+    a = np.where(a > 0, (a - t0) / 1e3, np.nan)
+    return a
+
+
 def main():
     args = [a for a in sys.argv[1:] if not a.startswith("--")]
     opts = dict(a[2:].split("=") for a in sys.argv[1:] if a.startswith("--"))
@@ -36,6 +56,15 @@ def main():
             if best is None or st["fill_ms"] < best["fill_ms"]:
                 best = st
         cells = len(A) * len(B)
+        if os.environ.get("SWB_DEBUG_TIMES"):
+            import numpy as np
+            t = band_times(ctx)
+            np.set_printoptions(linewidth=250, precision=1, suppress=True)
+            print("  slots: 0 start | 1..8 warp first chunk | 10 io first load | 11 io first drain | 12,13 chunk2 | 14 last warp done | 15 end")
+            for i in list(range(0, min(len(t), 3))) + [len(t) // 2]:
+                print("   band", i, t[i][:16])
+            lag = np.diff(t[:, 1])
+            print(f"  start lag us mean={np.nanmean(lag):.1f}; band dur us mean={np.nanmean(t[:,15]-t[:,1]):.0f}")
         print(f"{wl} v{v} k={k} result={r.astuple()} fill_ms={best['fill_ms']:.2f} total_ms={best['total_ms']:.2f} "
               f"GCUPS(fill)={cells / best['fill_ms'] / 1e6:.1f} alpha={best['alpha']} warps={best['warps']} "
               f"grid={best['grid']} replays={best['replays']}", flush=True)
@@ -44,3 +73,4 @@ def main():
 
 if __name__ == "__main__":
     main()
+
