@@ -127,6 +127,41 @@ int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end, const cha
  * the fast special-row path. */
 int64_t sw_row_granularity(const sw_ctx *ctx);
 
+/* Rows per band (alpha x 32 x warps): the unit of the band pipeline and of the
+ * multi-GPU border hand-off. */
+int64_t sw_band_height(const sw_ctx *ctx);
+
+/* ---- Column-stripe pipeline ----
+ * The matrix is split into column stripes; stripe g sweeps every band of its
+ * columns and hands the band's right-edge (t = H - G_first, E) column to stripe
+ * g+1, per (band, warp), with a release flag carrying the call's epoch.
+ *
+ * Virtual stripes on one GPU (testing / small m): the next sw_align_stage1*
+ * calls split [0, n) into `nstripes` (1..8) stripes run by one launch. */
+int sw_set_virtual_stripes(sw_ctx *ctx, int nstripes);
+
+/* One process per GPU.  Every rank except the first allocates its left-border
+ * receive area for up to `max_rows` rows and exports it as a CUDA IPC handle
+ * (64 bytes written to handle_out); the caller ships it to the left
+ * neighbour (e.g. torch.distributed).  The left neighbour maps it with
+ * sw_stripe_connect (NULL handle = last stripe).  Both must use the same band
+ * height (same library build and variant). */
+int sw_stripe_export(sw_ctx *ctx, int64_t max_rows, void *handle_out);
+int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t max_rows);
+
+/* Stage 1 on this rank's stripe: global columns [c_lo, c_hi) of S1 (0-based),
+ * all m rows.  dseqA / dseqB are the WHOLE sequences in this device's memory.
+ * `epoch` (>= 1) must be the same on all ranks for one alignment and grow by
+ * one per alignment.  `sink` receives this stripe's slice of each special row:
+ * H, F = columns c_lo+1 .. c_hi, n = c_hi - c_lo.  `out` is this stripe's best
+ * (score, i, j) in global coordinates; the global best is the maximum over
+ * ranks under the same order (score, then smallest i, then smallest j). */
+int sw_align_stage1_stripe(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                           int64_t c_lo, int64_t c_hi, int32_t epoch,
+                           int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                           int64_t special_row_interval, sw_row_sink sink, void *user, void *stream,
+                           sw_result *out);
+
 /* Flush-interval rule of P:178 as a helper: the special-row spacing in rows,
  * R = bh * ceil(8 m n / (bh * sra_bytes)), for a byte budget sra_bytes. */
 int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int64_t bh, int64_t sra_bytes);

@@ -38,6 +38,11 @@ EXPORTED = [
     "sw_reverse_goal",
     "sw_reverse_goal_dev",
     "sw_row_granularity",
+    "sw_band_height",
+    "sw_set_virtual_stripes",
+    "sw_stripe_export",
+    "sw_stripe_connect",
+    "sw_align_stage1_stripe",
     "sw_special_row_interval_for_budget",
     "sw_get_stats",
     "sw_shutdown",
@@ -111,6 +116,16 @@ def load_library(path: str = LIB_PATH):
     lib.sw_reverse_goal_dev.restype = ctypes.c_int
     lib.sw_row_granularity.argtypes = [vp]
     lib.sw_row_granularity.restype = i64
+    lib.sw_band_height.argtypes = [vp]
+    lib.sw_band_height.restype = i64
+    lib.sw_set_virtual_stripes.argtypes = [vp, ctypes.c_int]
+    lib.sw_set_virtual_stripes.restype = ctypes.c_int
+    lib.sw_stripe_export.argtypes = [vp, i64, vp]
+    lib.sw_stripe_export.restype = ctypes.c_int
+    lib.sw_stripe_connect.argtypes = [vp, vp, i64]
+    lib.sw_stripe_connect.restype = ctypes.c_int
+    lib.sw_align_stage1_stripe.argtypes = [vp, vp, i64, vp, i64, i64, i64, i32, i32, i32, i32, i32, i64, SINK, vp, vp, R]
+    lib.sw_align_stage1_stripe.restype = ctypes.c_int
     lib.sw_special_row_interval_for_budget.argtypes = [i64, i64, i64, i64]
     lib.sw_special_row_interval_for_budget.restype = i64
     lib.sw_get_stats.argtypes = [vp, ctypes.POINTER(Stats)]
@@ -231,6 +246,36 @@ class Context:
 
     def row_granularity(self) -> int:
         return int(self._lib.sw_row_granularity(self._h))
+
+    def band_height(self) -> int:
+        return int(self._lib.sw_band_height(self._h))
+
+    def set_virtual_stripes(self, nstripes: int):
+        """Split the next Stage-1 calls into `nstripes` column stripes on this GPU
+        (the multi-GPU border protocol, run inside one launch)."""
+        self._check(self._lib.sw_set_virtual_stripes(self._h, nstripes), "sw_set_virtual_stripes")
+
+    def stripe_export(self, max_rows: int) -> bytes:
+        """Allocate this rank's left-border receive area; returns its 64-byte CUDA IPC handle."""
+        buf = ctypes.create_string_buffer(64)
+        self._check(self._lib.sw_stripe_export(self._h, max_rows, buf), "sw_stripe_export")
+        return buf.raw
+
+    def stripe_connect(self, right_handle, max_rows: int):
+        """Map the right neighbour's receive area (None for the last stripe)."""
+        h = ctypes.create_string_buffer(bytes(right_handle), 64) if right_handle is not None else None
+        self._check(self._lib.sw_stripe_connect(self._h, h, max_rows), "sw_stripe_connect")
+
+    def align_stage1_stripe(self, dA_ptr, m, dB_ptr, n, c_lo, c_hi, epoch, match=1, mismatch=-3, gap_open=3,
+                            gap_ext=2, k=0, sink=None, keep_rows=False, stream: int = 0):
+        """This rank's stripe [c_lo, c_hi) of Stage 1 (device sequences, whole A and B)."""
+        rows = []
+        cb = self._make_sink(sink, keep_rows, rows) if k > 0 else SINK()
+        out = _Result()
+        rc = self._lib.sw_align_stage1_stripe(self._h, dA_ptr, m, dB_ptr, n, c_lo, c_hi, epoch, match, mismatch,
+                                              gap_open, gap_ext, k, cb, None, stream or None, ctypes.byref(out))
+        self._check(rc, "sw_align_stage1_stripe")
+        return Result(out.score, out.i, out.j), rows
 
     def stats(self) -> dict:
         s = Stats()

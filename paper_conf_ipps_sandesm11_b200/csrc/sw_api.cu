@@ -1,9 +1,10 @@
 // sw_api.cu -- C ABI (include/cudalign_b200.h) and host runtime of the
 // B200-native Stage-1 engine: parameter validation, sequence encode/pack,
 // persistent fill launch, special-row streaming to the host sink through
-// pinned memory on a side stream, best-cell reduction, and the
-// reverse goal pass.  No CPU fallback: every step runs in the
-// kernels below or in sw_fill.cuh.
+// pinned memory on a side stream, best-cell reduction, the
+// reverse goal pass, and the column-stripe pipeline (one stripe
+// per GPU over CUDA IPC / NVLink, or several virtual stripes on one GPU).
+// No CPU fallback: every step runs in the kernels below or in sw_fill.cuh.
 #include <algorithm>
 #include <chrono>
 #include <cstdarg>
@@ -11,6 +12,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <thread>
+#include <vector>
 
 #include "../../include/cudalign_b200.h"
 #include "sw_fill.cuh"
@@ -116,16 +118,16 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
+static constexpr int NVARIANTS = 3;
 
 static const Variant &variant_for(int idx)
 {
-    static const Variant vs[] = {
+    static const Variant vs[NVARIANTS] = {
         make_variant<16, 4, 64>(),
         make_variant<16, 8, 64>(),
         make_variant<8, 8, 64>(),
     };
-    const int n = sizeof(vs) / sizeof(vs[0]);
-    return vs[idx < 0 ? 0 : idx >= n ? n - 1 : idx];
+    return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
 
 // ---------------------------------------------------------------- context
@@ -135,21 +137,42 @@ struct DevBuf {
     size_t cap = 0;
 };
 
+struct HostBuf {
+    void *p = nullptr;
+    size_t cap = 0;
+    bool mapped = false;
+};
+
+// Border receive area of one stripe: (t, E) per DP row, then per (band, warp) epoch flags.
+struct RecvArea {
+    void *base = nullptr;  // device allocation (IPC-exportable)
+    size_t rows = 0, flags = 0;
+    int2 *lb() const { return (int2 *)base; }
+    int *lready() const { return (int *)((char *)base + rows * sizeof(int2)); }
+};
+
 struct sw_ctx {
     int device = 0;
     int num_sms = 0;
     cudaStream_t stream = nullptr, side = nullptr;
     cudaEvent_t ev[6] = {};
-    DevBuf seq, a2, b2, rowb, progress, misc, slots, sp, dbg;
+    DevBuf seq, a2, b2, misc, slots, dbg;
+    DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
+    HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
+    HostBuf stage;               // pinned staging for one special row (H then F)
+    RecvArea vrecv[MAX_STRIPES]; // receive areas of virtual stripes 1..S-1
+    // multi-GPU stripe (one per process): own receive area (exported), right neighbour's (imported)
+    RecvArea recv;
+    void *right_base = nullptr;
+    size_t right_rows = 0;
+    int epoch = 0;
     int dbg_n = 0;
-    unsigned int *flags_h = nullptr, *flags_d = nullptr;
-    size_t flags_cap = 0;
-    int32_t *stage_h = nullptr;
-    size_t stage_cap = 0;
-    int4 *res_h = nullptr;  // pinned: result + err
+    int4 *res_h = nullptr;  // pinned: result + err + replays
     sw_stats stats{};
     char errbuf[512] = {0};
     int variant_override = -1;
+    int vstripes = 1;           // virtual stripes for the single-process calls
+    long long timeout_ns = 120ll * 1000000000ll;
 };
 
 static int cuda_fail(sw_ctx *c, cudaError_t e, const char *what)
@@ -178,6 +201,39 @@ static int grow(sw_ctx *ctx, DevBuf &b, size_t bytes)
         return SW_ENOMEM;
     }
     b.cap = want;
+    return SW_OK;
+}
+
+static int grow_host(sw_ctx *ctx, HostBuf &b, size_t bytes, bool mapped)
+{
+    if (b.cap >= bytes && b.p) return SW_OK;
+    if (b.p) cudaFreeHost(b.p);
+    b.p = nullptr;
+    b.cap = 0;
+    if (cudaHostAlloc(&b.p, std::max<size_t>(bytes, 64), mapped ? cudaHostAllocMapped : cudaHostAllocDefault) != cudaSuccess) {
+        cudaGetLastError();
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "cudaHostAlloc(%zu) failed", bytes);
+        return SW_ENOMEM;
+    }
+    b.cap = std::max<size_t>(bytes, 64);
+    b.mapped = mapped;
+    return SW_OK;
+}
+
+static int grow_recv(sw_ctx *ctx, RecvArea &r, size_t rows, size_t flags)
+{
+    if (r.base && r.rows >= rows && r.flags >= flags) return SW_OK;
+    if (r.base) cudaFree(r.base);
+    r.base = nullptr;
+    const size_t bytes = rows * sizeof(int2) + flags * sizeof(int);
+    if (cudaMalloc(&r.base, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "cudaMalloc(%zu) for a border area failed", bytes);
+        return SW_ENOMEM;
+    }
+    cudaMemset(r.base, 0, bytes);  // flags start at epoch 0; calls use epochs >= 1
+    r.rows = rows;
+    r.flags = flags;
     return SW_OK;
 }
 
@@ -217,14 +273,15 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
             if ((e = cudaEventCreate(&ev)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
         if (rc) break;
         if ((e = cudaHostAlloc(&ctx->res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
-        for (int i = 0; i < 3; i++) {
+        for (int i = 0; i < NVARIANTS; i++) {
             const Variant &v = variant_for(i);
             cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
             cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaFuncSetAttribute"); break; }
-        const char *ov = getenv("SWB_VARIANT");
-        if (ov) ctx->variant_override = atoi(ov);
+        if (const char *ov = getenv("SWB_VARIANT")) ctx->variant_override = atoi(ov);
+        if (const char *vs = getenv("SWB_VSTRIPES")) ctx->vstripes = std::max(1, std::min(MAX_STRIPES, atoi(vs)));
+        if (const char *to = getenv("SWB_TIMEOUT_S")) ctx->timeout_ns = (long long)(atof(to) * 1e9);
     } while (0);
     if (rc) { sw_shutdown(ctx); return rc; }
     *out = ctx;
@@ -237,10 +294,17 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->side) cudaStreamSynchronize(ctx->side);
-    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->rowb, &ctx->progress, &ctx->misc, &ctx->slots, &ctx->sp, &ctx->dbg})
+    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg})
         if (b->p) cudaFree(b->p);
-    if (ctx->flags_h) cudaFreeHost(ctx->flags_h);
-    if (ctx->stage_h) cudaFreeHost(ctx->stage_h);
+    for (int s = 0; s < MAX_STRIPES; s++) {
+        for (DevBuf *b : {&ctx->rowb[s], &ctx->progress[s], &ctx->sp[s]})
+            if (b->p) cudaFree(b->p);
+        if (ctx->flags[s].p) cudaFreeHost(ctx->flags[s].p);
+        if (ctx->vrecv[s].base) cudaFree(ctx->vrecv[s].base);
+    }
+    if (ctx->right_base) cudaIpcCloseMemHandle(ctx->right_base);
+    if (ctx->recv.base) cudaFree(ctx->recv.base);
+    if (ctx->stage.p) cudaFreeHost(ctx->stage.p);
     if (ctx->res_h) cudaFreeHost(ctx->res_h);
     for (auto &ev : ctx->ev)
         if (ev) cudaEventDestroy(ev);
@@ -249,10 +313,22 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     delete ctx;
 }
 
+static const Variant &ctx_variant(const sw_ctx *ctx)
+{
+    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT);
+}
+
 extern "C" int64_t sw_row_granularity(const sw_ctx *ctx)
 {
     if (!ctx) return 0;
-    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT).alpha;
+    return ctx_variant(ctx).alpha;
+}
+
+extern "C" int64_t sw_band_height(const sw_ctx *ctx)
+{
+    if (!ctx) return 0;
+    const Variant &v = ctx_variant(ctx);
+    return (int64_t)v.alpha * 32 * v.nw;
 }
 
 extern "C" int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int64_t bh, int64_t sra_bytes)
@@ -264,6 +340,13 @@ extern "C" int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int6
     unsigned __int128 q = (num + den - 1) / den;
     if (q < 1) q = 1;
     return (int64_t)(bh * (int64_t)q);
+}
+
+extern "C" int sw_set_virtual_stripes(sw_ctx *ctx, int nstripes)
+{
+    if (!ctx || nstripes < 1 || nstripes > MAX_STRIPES) return SW_EINVAL;
+    ctx->vstripes = nstripes;
+    return SW_OK;
 }
 
 // Debug: copy the per-band timestamps of the last fill (SWB_DEBUG_TIMES set).
@@ -311,69 +394,102 @@ struct Job {
     void *user;
     bool local;
     int32_t goal;
+    // stripes: either `nv` virtual stripes of [0, n) on this GPU, or (rank mode)
+    // one stripe [c_lo, c_hi) whose borders come from / go to other GPUs.
+    int nv = 1;
+    bool rank_mode = false;
+    int64_t c_lo = 0, c_hi = 0;
+    int epoch = 0;
 };
 }  // namespace
 
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
 {
-    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT);
+    const Variant &V = ctx_variant(ctx);
     const int W = V.w;
     const int BH = V.alpha * 32 * V.nw;
     const int m = (int)J.m, n = (int)J.n;
-    const int ncols_pad = ((n + W - 1) / W) * W;
-    const int NT = ncols_pad / W + 1;
     const int nb = (m + BH - 1) / BH;
     const long long wa = (J.m + 15) / 16 + 2, wb = (J.n + 15) / 16 + 2;
+    const int NS = J.rank_mode ? 1 : J.nv;
     int rc;
+
+    // stripe geometry
+    long long col0[MAX_STRIPES], wid[MAX_STRIPES];
+    if (J.rank_mode) {
+        col0[0] = J.c_lo;
+        wid[0] = J.c_hi - J.c_lo;
+    } else {
+        for (int s = 0; s < NS; s++) {
+            col0[s] = (long long)n * s / NS;
+            wid[s] = (long long)n * (s + 1) / NS - col0[s];
+        }
+    }
+    for (int s = 0; s < NS; s++)
+        if (wid[s] <= 0) {
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe %d is empty (n=%d, stripes=%d)", s, n, NS);
+            return SW_EINVAL;
+        }
+
     if ((rc = grow(ctx, ctx->a2, wa * 4))) return rc;
     if ((rc = grow(ctx, ctx->b2, wb * 4))) return rc;
-    if ((rc = grow(ctx, ctx->rowb, (size_t)(NT * W + 2 * W) * sizeof(int2)))) return rc;
-    if ((rc = grow(ctx, ctx->progress, (size_t)(nb + 1) * sizeof(int)))) return rc;
-    // misc: err, ticket, gbest, hit_band, (pad), hit_key(8B), replays(8B)
-    if ((rc = grow(ctx, ctx->misc, 64))) return rc;
+    if ((rc = grow(ctx, ctx->misc, 256))) return rc;
+    const size_t border_rows = (size_t)nb * BH + 2;
+    const size_t border_flags = (size_t)nb * V.nw + 1;
+    for (int s = 0; s < NS; s++) {
+        const int npad = (int)((wid[s] + W - 1) / W) * W;
+        const int NT = npad / W + 1;
+        if ((rc = grow(ctx, ctx->rowb[s], (size_t)(NT * W + 2 * W) * sizeof(int2)))) return rc;
+        if ((rc = grow(ctx, ctx->progress[s], (size_t)(nb + 1) * sizeof(int)))) return rc;
+        if (!J.rank_mode && s > 0)
+            if ((rc = grow_recv(ctx, ctx->vrecv[s], border_rows, border_flags))) return rc;
+    }
+    if (J.rank_mode) {
+        if (J.c_lo > 0 && (!ctx->recv.base || ctx->recv.rows < border_rows || ctx->recv.flags < border_flags)) {
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe receive area missing or too small (sw_stripe_export)");
+            return SW_EINVAL;
+        }
+        if (J.c_hi < n && (!ctx->right_base || ctx->right_rows < border_rows)) {
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "right neighbour not connected (sw_stripe_connect)");
+            return SW_EINVAL;
+        }
+    }
     int blocks_per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, J.local ? V.local_fn : V.global_fn, V.nw * 32 + 32, V.smem);
     if (blocks_per_sm < 1) blocks_per_sm = 1;
-    int grid = std::min(nb, blocks_per_sm * ctx->num_sms);
-    if (const char *g = getenv("SWB_GRID")) grid = std::max(1, std::min(nb, atoi(g)));
+    // every CTA of every stripe must be co-resident (stripes wait on each other)
+    int per_stripe = std::max(1, std::min(nb, blocks_per_sm * ctx->num_sms / NS));
+    if (const char *g = getenv("SWB_GRID")) per_stripe = std::max(1, std::min(per_stripe, atoi(g) / NS));
+    const int grid = per_stripe * NS;
     if ((rc = grow(ctx, ctx->slots, (size_t)grid * sizeof(int4)))) return rc;
 
     // special rows: all of them stay resident on the device (180 GB HBM) and
     // are streamed to the host as bands complete.
     const long long nsp = (J.local && J.k > 0) ? J.m / J.k : 0;
-    const int ld = ((n + 31) / 32) * 32;
-    const long long stride = 2ll * ld;
+    int ld[MAX_STRIPES];
+    long long stride[MAX_STRIPES];
+    size_t row_ints = 0;
+    for (int s = 0; s < NS; s++) {
+        ld[s] = (int)((wid[s] + 31) / 32) * 32;
+        stride[s] = 2ll * ld[s];
+        row_ints += (size_t)stride[s];
+    }
     if (nsp > 0) {
         size_t freeb = 0, totb = 0;
         cudaMemGetInfo(&freeb, &totb);
-        const size_t need = (size_t)nsp * stride * sizeof(int);
-        if (need > ctx->sp.cap && need > (size_t)(0.8 * (double)(freeb + ctx->sp.cap))) {
+        size_t have = 0;
+        for (int s = 0; s < NS; s++) have += ctx->sp[s].cap;
+        const size_t need = (size_t)nsp * row_ints * sizeof(int);
+        if (need > have && need > (size_t)(0.8 * (double)(freeb + have))) {
             snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special rows need %zu bytes on the device", need);
             return SW_ENOMEM;
         }
-        if ((rc = grow(ctx, ctx->sp, need))) return rc;
-        if ((size_t)nsp > ctx->flags_cap) {
-            if (ctx->flags_h) cudaFreeHost(ctx->flags_h);
-            ctx->flags_h = nullptr;
-            ctx->flags_cap = 0;
-            if (cudaHostAlloc(&ctx->flags_h, nsp * sizeof(unsigned int), cudaHostAllocMapped) != cudaSuccess) {
-                cudaGetLastError();
-                return SW_ENOMEM;
-            }
-            ctx->flags_cap = nsp;
-            CK(cudaHostGetDevicePointer((void **)&ctx->flags_d, ctx->flags_h, 0));
+        for (int s = 0; s < NS; s++) {
+            if ((rc = grow(ctx, ctx->sp[s], (size_t)nsp * stride[s] * sizeof(int)))) return rc;
+            if ((rc = grow_host(ctx, ctx->flags[s], nsp * sizeof(unsigned int), true))) return rc;
+            memset(ctx->flags[s].p, 0, nsp * sizeof(unsigned int));
         }
-        memset(ctx->flags_h, 0, nsp * sizeof(unsigned int));
-        if ((size_t)stride > ctx->stage_cap) {
-            if (ctx->stage_h) cudaFreeHost(ctx->stage_h);
-            ctx->stage_h = nullptr;
-            ctx->stage_cap = 0;
-            if (cudaHostAlloc(&ctx->stage_h, stride * sizeof(int32_t), cudaHostAllocDefault) != cudaSuccess) {
-                cudaGetLastError();
-                return SW_ENOMEM;
-            }
-            ctx->stage_cap = stride;
-        }
+        if ((rc = grow_host(ctx, ctx->stage, (size_t)2 * (n + 32) * sizeof(int32_t), false))) return rc;
     }
 
     // With a caller stream, every kernel of the call is launched on it (so the
@@ -381,19 +497,20 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     cudaStream_t st = user_stream ? user_stream : ctx->stream;
     char *misc = (char *)ctx->misc.p;
     int *d_err = (int *)(misc + 0);
-    int *d_ticket = (int *)(misc + 4);
     int *d_gbest = (int *)(misc + 8);
     int *d_hit_band = (int *)(misc + 12);
     unsigned long long *d_hit_key = (unsigned long long *)(misc + 16);
     unsigned long long *d_replays = (unsigned long long *)(misc + 24);
     int4 *d_res = (int4 *)(misc + 32);
+    int *d_tickets = (int *)(misc + 64);  // MAX_STRIPES
 
     CK(cudaEventRecord(ctx->ev[0], st));
     CK(cudaMemsetAsync(misc, 0, 16, st));
     CK(cudaMemsetAsync(d_hit_band, 0x7f, 4, st));
     CK(cudaMemsetAsync(d_hit_key, 0xff, 8, st));
     CK(cudaMemsetAsync(d_replays, 0, 8, st));
-    CK(cudaMemsetAsync(ctx->progress.p, 0, (size_t)(nb + 1) * sizeof(int), st));
+    CK(cudaMemsetAsync(d_tickets, 0, MAX_STRIPES * sizeof(int), st));
+    for (int s = 0; s < NS; s++) CK(cudaMemsetAsync(ctx->progress[s].p, 0, (size_t)(nb + 1) * sizeof(int), st));
     {
         const long long words = wa + wb;
         const int tpb = 256;
@@ -406,8 +523,6 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     FillArgs a{};
     a.m = m;
     a.n = n;
-    a.ncols_pad = ncols_pad;
-    a.NT = NT;
     a.nb = nb;
     a.go = J.go;
     a.ge = J.ge;
@@ -424,27 +539,53 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     a.A2 = (const uint32_t *)ctx->a2.p;
     a.B2 = (const uint32_t *)ctx->b2.p;
     a.err = d_err;
-    a.rowb = (int2 *)ctx->rowb.p;
-    a.progress = (int *)ctx->progress.p;
-    a.ticket = d_ticket;
     a.k = (int)(nsp > 0 ? J.k : 0);
-    a.sp = (int *)ctx->sp.p;
-    a.sp_stride = stride;
-    a.sp_ld = ld;
-    a.row_done = ctx->flags_d;
     a.gbest = d_gbest;
     a.slots = (int4 *)ctx->slots.p;
     a.goal = J.goal;
     a.hit_key = d_hit_key;
     a.hit_band = d_hit_band;
     a.replays = d_replays;
+    a.epoch = J.epoch;
+    a.timeout_ns = ctx->timeout_ns;
+    a.nstripes = NS;
+    a.force_slow = 0;
     a.dbg = nullptr;
-    a.force_slow = getenv("SWB_FORCE_SLOW") ? 1 : 0;
     if (getenv("SWB_DEBUG_TIMES")) {
         if ((rc = grow(ctx, ctx->dbg, (size_t)nb * 80 * sizeof(unsigned long long)))) return rc;
         CK(cudaMemsetAsync(ctx->dbg.p, 0, (size_t)nb * 80 * sizeof(unsigned long long), st));
         a.dbg = (unsigned long long *)ctx->dbg.p;
         ctx->dbg_n = nb;
+    }
+    for (int s = 0; s < NS; s++) {
+        StripeArgs &S = a.st[s];
+        S.col0 = (int)col0[s];
+        S.w = (int)wid[s];
+        S.ncols_pad = (int)((wid[s] + W - 1) / W) * W;
+        S.NT = S.ncols_pad / W + 1;
+        S.rowb = (int2 *)ctx->rowb[s].p;
+        S.progress = (int *)ctx->progress[s].p;
+        S.ticket = d_tickets + s;
+        S.sp = nsp > 0 ? (int *)ctx->sp[s].p : nullptr;
+        S.sp_stride = stride[s];
+        S.sp_ld = ld[s];
+        unsigned int *fd = nullptr;
+        if (nsp > 0) CK(cudaHostGetDevicePointer((void **)&fd, ctx->flags[s].p, 0));
+        S.row_done = fd;
+        if (J.rank_mode) {
+            S.lb = J.c_lo > 0 ? ctx->recv.lb() : nullptr;
+            S.lready = J.c_lo > 0 ? ctx->recv.lready() : nullptr;
+            RecvArea right;
+            right.base = ctx->right_base;
+            right.rows = ctx->right_rows;
+            S.rb = J.c_hi < n ? right.lb() : nullptr;
+            S.rready = J.c_hi < n ? right.lready() : nullptr;
+        } else {
+            S.lb = s > 0 ? ctx->vrecv[s].lb() : nullptr;
+            S.lready = s > 0 ? ctx->vrecv[s].lready() : nullptr;
+            S.rb = s + 1 < NS ? ctx->vrecv[s + 1].lb() : nullptr;
+            S.rready = s + 1 < NS ? ctx->vrecv[s + 1].lready() : nullptr;
+        }
     }
     {
         void *args[] = {&a};
@@ -458,37 +599,50 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     CK(cudaMemcpyAsync(ctx->res_h + 2, d_replays, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     CK(cudaEventRecord(ctx->ev[3], st));
 
-    // stream special rows to the sink in ascending order while the fill runs
+    // stream special rows to the sink in ascending order while the fill runs;
+    // a row is complete when every stripe of this launch has published it
     int sink_rc = 0;
     long long bytes = 0;
+    const int64_t nrow_out = J.rank_mode ? wid[0] : n;
+    int32_t *stage = (int32_t *)ctx->stage.p;
+    const int64_t sld = nrow_out + 32;
     for (long long q = 0; q < nsp; q++) {
-        volatile unsigned int *f = ctx->flags_h + q;
-        while (*f == 0) {
-            const cudaError_t qe = cudaEventQuery(ctx->ev[2]);
-            if (qe == cudaSuccess) {
-                if (*f == 0) {
-                    // fill finished without publishing: only legitimate on an alphabet error
-                    CK(cudaStreamSynchronize(st));
-                    if (ctx->res_h[1].x) return SW_EALPHABET;
-                    snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published", q);
-                    return SW_ECUDA;
+        for (int s = 0; s < NS; s++) {
+            volatile unsigned int *f = (volatile unsigned int *)ctx->flags[s].p + q;
+            while (*f == 0) {
+                const cudaError_t qe = cudaEventQuery(ctx->ev[2]);
+                if (qe == cudaSuccess) {
+                    if (*f == 0) {
+                        CK(cudaStreamSynchronize(st));
+                        if (ctx->res_h[1].x == 1) return SW_EALPHABET;
+                        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", q,
+                                 ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
+                        return SW_ECUDA;
+                    }
+                    break;
+                } else if (qe != cudaErrorNotReady) {
+                    return cuda_fail(ctx, qe, "fill kernel");
                 }
-                break;
-            } else if (qe != cudaErrorNotReady) {
-                return cuda_fail(ctx, qe, "fill kernel");
+                std::this_thread::yield();
             }
-            std::this_thread::yield();
         }
         if (sink_rc) continue;  // aborted: drain flags, skip copies
-        const int32_t *src = (const int32_t *)ctx->sp.p + q * stride;
-        CK(cudaMemcpyAsync(ctx->stage_h, src, (size_t)n * 4, cudaMemcpyDeviceToHost, ctx->side));
-        CK(cudaMemcpyAsync(ctx->stage_h + ld, src + ld, (size_t)n * 4, cudaMemcpyDeviceToHost, ctx->side));
+        for (int s = 0; s < NS; s++) {
+            const int32_t *src = (const int32_t *)ctx->sp[s].p + q * stride[s];
+            const int64_t off = J.rank_mode ? 0 : col0[s];
+            CK(cudaMemcpyAsync(stage + off, src, (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+            CK(cudaMemcpyAsync(stage + sld + off, src + ld[s], (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+        }
         CK(cudaStreamSynchronize(ctx->side));
-        bytes += 8ll * n;
-        if (J.sink && J.sink(J.user, (q + 1) * J.k, ctx->stage_h, ctx->stage_h + ld, J.n)) sink_rc = SW_EABORTED;
+        bytes += 8ll * nrow_out;
+        if (J.sink && J.sink(J.user, (q + 1) * J.k, stage, stage + sld, nrow_out)) sink_rc = SW_EABORTED;
     }
     CK(cudaStreamSynchronize(st));
-    if (ctx->res_h[1].x) return SW_EALPHABET;
+    if (ctx->res_h[1].x == 1) return SW_EALPHABET;
+    if (ctx->res_h[1].x == 2) {
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "fill kernel: border wait timeout (a neighbour stripe did not progress)");
+        return SW_ECUDA;
+    }
     if (sink_rc) return sink_rc;
     *res = ctx->res_h[0];
 
@@ -521,6 +675,8 @@ static int stage1_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const 
     J.k = k; J.sink = sink; J.user = user;
     J.local = true;
     J.goal = 0;
+    J.nv = (int)std::max<int64_t>(1, std::min<int64_t>(ctx->vstripes, n));
+    J.epoch = ++ctx->epoch;
     int4 r;
     const int rc = run_job(ctx, J, us, &r);
     if (rc) return rc;
@@ -533,7 +689,7 @@ static int stage1_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const 
 static bool valid_common(sw_ctx *ctx, int64_t m, int64_t n, int64_t k, sw_row_sink sink, sw_result *out)
 {
     if (!ctx || !out || m < 0 || n < 0 || k < 0) return false;
-    if (m >= (1ll << 31) - 1024 || n >= (1ll << 31) - 1024) return false;
+    if (m >= (1ll << 31) - (1 << 16) || n >= (1ll << 31) - (1 << 16)) return false;
     if (k > 0 && !sink) return false;
     return true;
 }
@@ -599,18 +755,86 @@ extern "C" int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, co
     return SW_OK;
 }
 
-// Reverse pass.  Exact pruning: a cell (i', j')
-// of the reverse matrix scores at most pmax*min(i',j') - [i' != j'](G_open +
-// |i'-j'| G_ext), so a hit in rows <= L lies in columns <= J(L) = L +
-// (pmax*L - G_open - goal)/G_ext.  The rectangle [1..L] x [1..J(L)] is closed
-// under the recurrence's dependencies, so filling it exactly finds the first
-// hit among rows <= L; L grows geometrically until a hit appears or L = i_end.
+// ---------------------------------------------------------------- multi-GPU column stripes
+
+extern "C" int sw_stripe_export(sw_ctx *ctx, int64_t max_rows, void *handle_out)
+{
+    if (!ctx || max_rows < 0 || !handle_out) return SW_EINVAL;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const Variant &V = ctx_variant(ctx);
+    const int64_t BH = (int64_t)V.alpha * 32 * V.nw;
+    const int64_t nb = (max_rows + BH - 1) / BH;
+    int rc = grow_recv(ctx, ctx->recv, (size_t)(nb * BH + 2), (size_t)(nb * V.nw + 1));
+    if (rc) return rc;
+    cudaIpcMemHandle_t h;
+    CK(cudaIpcGetMemHandle(&h, ctx->recv.base));
+    memcpy(handle_out, &h, sizeof(h));
+    return SW_OK;
+}
+
+extern "C" int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t max_rows)
+{
+    if (!ctx) return SW_EINVAL;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    if (ctx->right_base) {
+        cudaIpcCloseMemHandle(ctx->right_base);
+        ctx->right_base = nullptr;
+    }
+    if (!right_handle) return SW_OK;
+    cudaIpcMemHandle_t h;
+    memcpy(&h, right_handle, sizeof(h));
+    CK(cudaIpcOpenMemHandle(&ctx->right_base, h, cudaIpcMemLazyEnablePeerAccess));
+    const Variant &V = ctx_variant(ctx);
+    const int64_t BH = (int64_t)V.alpha * 32 * V.nw;
+    ctx->right_rows = (size_t)(((max_rows + BH - 1) / BH) * BH + 2);
+    return SW_OK;
+}
+
+extern "C" int sw_align_stage1_stripe(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                                      int64_t c_lo, int64_t c_hi, int32_t epoch, int32_t match, int32_t mismatch,
+                                      int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
+                                      sw_row_sink sink, void *user, void *stream, sw_result *out)
+{
+    if (!valid_common(ctx, m, n, special_row_interval, sink, out)) return SW_EINVAL;
+    if (!dseqA || !dseqB || m <= 0 || c_lo < 0 || c_hi > n || c_hi <= c_lo || epoch <= 0) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    Job J{};
+    J.dA = (const unsigned char *)dseqA; J.m = m; J.dB = (const unsigned char *)dseqB; J.n = n;
+    J.ma = match; J.mi = mismatch; J.go = gap_open; J.ge = gap_ext;
+    J.k = special_row_interval; J.sink = sink; J.user = user;
+    J.local = true;
+    J.rank_mode = true;
+    J.c_lo = c_lo;
+    J.c_hi = c_hi;
+    J.epoch = epoch;
+    int4 r;
+    rc = run_job(ctx, J, (cudaStream_t)stream, &r);
+    if (rc) return rc;
+    out->score = r.x;
+    out->i = r.y;
+    out->j = r.z;
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return SW_OK;
+}
+
+// ---------------------------------------------------------------- reverse pass
+
+// Exact pruning: a cell (i', j') of the reverse matrix scores
+// at most pmax*min(i',j') - [i' != j'](G_open + |i'-j'| G_ext), so a hit in rows
+// <= L lies in columns <= J(L) = L + (pmax*L - G_open - goal)/G_ext.  The
+// rectangle [1..L] x [1..J(L)] is closed under the recurrence's dependencies,
+// so filling it exactly finds the first hit among rows <= L; L grows
+// geometrically until a hit appears or L = i_end.
 static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, const unsigned char *dB,
                           int64_t j_end, int32_t ma, int32_t mi, int32_t go, int32_t ge, int32_t goal,
                           cudaStream_t us, sw_result *out)
 {
     const long long pmax = std::max(ma, mi);
-    const Variant &V = variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT);
+    const Variant &V = ctx_variant(ctx);
     const long long BH = (long long)V.alpha * 32 * V.nw;
     long long L = std::max<long long>(BH, pmax > 0 ? (goal + pmax - 1) / pmax : i_end);
     for (;;) {
@@ -635,6 +859,8 @@ static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, c
         J.k = 0; J.sink = nullptr; J.user = nullptr;
         J.local = false;
         J.goal = goal;
+        J.nv = 1;
+        J.epoch = ++ctx->epoch;
         int4 r;
         const int rc = run_job(ctx, J, us, &r);
         if (rc) return rc;
@@ -655,7 +881,7 @@ extern "C" int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, con
 {
     if (!ctx || !start_out || i_end < 0 || j_end < 0 || goal < 0) return SW_EINVAL;
     if ((i_end && !seqA) || (j_end && !seqB)) return SW_EINVAL;
-    if (i_end >= (1ll << 31) - 1024 || j_end >= (1ll << 31) - 1024) return SW_EINVAL;
+    if (i_end >= (1ll << 31) - (1 << 16) || j_end >= (1ll << 31) - (1 << 16)) return SW_EINVAL;
     int rc = check_scoring(match, mismatch, gap_open, gap_ext, i_end, j_end);
     if (rc) return rc;
     if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;

@@ -42,35 +42,62 @@ constexpr int NEG = -(1 << 30);            // E(i,0), F(0,j) = "-infinity" (read
 constexpr uint32_t PADPROF = 0x80808080u;  // profile of padding rows / padding column: -128
 constexpr int LANE_SKEW = 2;               // columns per lane step
 
-struct FillArgs {
-    int m, n;            // real sizes (rows of S0, columns of S1)
-    int ncols_pad;       // n rounded up to a multiple of W
+constexpr int MAX_STRIPES = 8;
+
+// One column stripe [col0, col0 + w) of the matrix.  A launch
+// runs nstripes stripes (CTA -> stripe = blockIdx.x % nstripes): 1 per GPU in
+// the multi-GPU pipeline, several "virtual" stripes on one GPU for testing.
+struct StripeArgs {
+    int col0;            // first global 0-based column
+    int w;               // real columns of the stripe
+    int ncols_pad;       // w rounded up to a multiple of W
     int NT;              // tiles each warp runs per band = ncols_pad / W + 1
+    int2 *rowb;          // row border: (t, F) per local column, >= NT*W + W entries
+    int *progress;       // per band: number of leading columns of its bottom row published
+    int *ticket;         // band ticket of this stripe
+    int *sp;             // special rows (this stripe's slice): slot q at sp + q*sp_stride: H, then F at + sp_ld
+    long long sp_stride;
+    int sp_ld;
+    unsigned int *row_done;  // mapped host flags, one per special row
+    const int2 *lb;      // left border (t, E) per DP row 0..m at column col0 - 1 (null: column-0 boundary)
+    const int *lready;   // per (band, warp) epoch flags guarding lb
+    int2 *rb;            // right neighbour's lb (null: last stripe); a peer-GPU pointer across GPUs
+    int *rready;         // right neighbour's lready
+};
+
+struct FillArgs {
+    int m;               // rows of S0
+    int n;               // columns of S1 (all stripes)
     int nb;              // number of bands
     int go, ge, gf;      // G_open, G_ext, G_first = go + ge
     int one;             // always 1 (see imad())
     uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
     const uint32_t *A2;  // S0 codes, 2 bits each, 16 per word
-    const uint32_t *B2;  // S1 codes
-    const int *err;      // non-zero: encode found a bad byte -> do nothing
-    int2 *rowb;          // row border: (t, F) per column, >= NT*W + W entries
-    int *progress;       // per band: number of leading columns of its bottom row published
-    int *ticket;         // band ticket
-    // special rows (LOCAL only)
-    int k;               // interval (0 = none)
-    int *sp;             // device rows: slot q at sp + q*sp_stride: H[0..n), then F at + sp_ld
-    long long sp_stride;
-    int sp_ld;
-    unsigned int *row_done;  // mapped host flags, one per special row
-    // best (LOCAL) / goal (GLOBAL)
+    const uint32_t *B2;  // S1 codes (global columns)
+    int *err;            // non-zero: encode found a bad byte -> do nothing; kernel sets 2 on a wait timeout
+    int k;               // special-row interval (0 = none)
     int *gbest;          // running best-score hint
     int4 *slots;         // per-CTA (score, i, j, 0)
-    int goal;
+    int goal;            // GLOBAL mode
     unsigned long long *hit_key;  // min over hits of (i' << 32 | j')
     int *hit_band;       // min band containing a hit
     unsigned long long *replays;
-    int force_slow;           // unused (kept for ABI of FillArgs between host and kernels)
+    int epoch;           // value written to the border flags by this call
+    long long timeout_ns;  // spin-wait watchdog
+    int nstripes;
+    int force_slow;      // unused
     unsigned long long *dbg;  // optional: per band 80 x %globaltimer; slot 0 band start, 1 first tile, 15 band end
+    StripeArgs st[MAX_STRIPES];
+};
+
+// Per-CTA view of the stripe fields the cell step needs.
+struct StepInfo {
+    int w;               // stripe width (pad columns are >= w)
+    int col0;            // global column of local column 0
+    int sp_ld;
+    long long sp_stride;
+    int jcap;            // local column whose (t, E) goes to the right neighbour
+    int2 *rbrow;         // right-border destination for this lane's first row
 };
 
 __device__ __forceinline__ unsigned long long gtimer()
@@ -91,6 +118,39 @@ __device__ __forceinline__ int prmt(uint32_t a, uint32_t b, uint32_t sel)
     int r;
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
     return r;
+}
+
+// Shared-memory accesses through 32-bit shared-window addresses (kept in
+// registers; avoids re-deriving the generic window inside the hot loop).
+__device__ __forceinline__ int4 lds_v4(uint32_t addr)
+{
+    int4 v;
+    asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint2 lds_v2u(uint32_t addr)
+{
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(addr) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sts_v4(uint32_t addr, int4 v)
+{
+    asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+// An opaque copy: the result cannot be rematerialised by the compiler, so a
+// value computed once outside a loop stays in a register inside it.
+__device__ __forceinline__ uint32_t pin(uint32_t x)
+{
+    uint32_t y;
+    asm volatile("mov.b32 %0, %1;" : "=r"(y) : "r"(x));
+    return y;
+}
+__device__ __forceinline__ int lane_id()
+{
+    int l;
+    asm volatile("mov.u32 %0, %%laneid;" : "=r"(l));
+    return l;
 }
 
 // x * one + y through the FMA pipe (IMAD); `one` is a runtime 1 so ptxas
@@ -165,10 +225,10 @@ struct Fill {
     // j0 = 2 (k - lane) and j0 + 1.  TRACK: exact best / first-hit tracking.
     // SPM: 0 = no special rows, 1 = special rows are strip-bottom rows,
     // 2 = special rows anywhere in the strip (bitmask).
-    template <bool GUARD, bool TRACK, int SPM>
-    static __device__ __forceinline__ int step(const FillArgs &a, Lane &L, int k, int lane, const int2 *ring_in,
-                                               int2 *ring_out, const uint32_t *selr, int tmax, int row1,
-                                               int &bs, int &bi, int &bj, int *sp_ptr, uint32_t smask)
+    template <bool GUARD, bool TRACK, int SPM, bool CAP = false>
+    static __device__ __forceinline__ int step(const FillArgs &a, const StepInfo &X, Lane &L, int k, int lane,
+                                               uint32_t ring_in, uint32_t ring_out, uint32_t selr, int tmax,
+                                               int row1, int &bs, int &bi, int &bj, int *sp_ptr, uint32_t smask)
     {
         int a_t = __shfl_up_sync(0xffffffffu, L.out_t0, 1);
         int a_f = __shfl_up_sync(0xffffffffu, L.out_f0, 1);
@@ -176,11 +236,11 @@ struct Fill {
         int b_f = __shfl_up_sync(0xffffffffu, L.out_f1, 1);
         const int j0 = LANE_SKEW * (k - lane);
         if (lane == 0) {
-            const int4 v = *reinterpret_cast<const int4 *>(ring_in + (j0 & (RING - 1)));
+            const int4 v = lds_v4(ring_in + (uint32_t)(j0 & (RING - 1)) * 8u);
             a_t = v.x; a_f = v.y; b_t = v.z; b_f = v.w;
         }
         if (GUARD && j0 < 0) return tmax;
-        const uint2 sl = *reinterpret_cast<const uint2 *>(selr + (j0 & (SRING - 1)));
+        const uint2 sl = lds_v2u(selr + (uint32_t)(j0 & (SRING - 1)) * 4u);
         int tdA = L.tprev;  // t(r0-1, j0-1)
         int tdB = a_t;      // t(r0-1, j0)
         L.tprev = b_t;
@@ -215,26 +275,31 @@ struct Fill {
             tmax = __vimax3_s32(tmax, hA, hB);
             if (SPM == 2) {
                 if (smask & (1u << r)) {
-                    if (j0 < a.n) { spp[j0] = hA; spp[a.sp_ld + j0] = fuA; }
-                    if (j0 + 1 < a.n) { spp[j0 + 1] = hB; spp[a.sp_ld + j0 + 1] = fuB; }
-                    spp += a.sp_stride;
+                    if (j0 < X.w) { spp[j0] = hA; spp[X.sp_ld + j0] = fuA; }
+                    if (j0 + 1 < X.w) { spp[j0 + 1] = hB; spp[X.sp_ld + j0 + 1] = fuB; }
+                    spp += X.sp_stride;
                 }
+            }
+            if (CAP) {  // the stripe's last column: hand (t, E) to the right neighbour
+                if (j0 == X.jcap) X.rbrow[r] = make_int2(tA, eA);
+                if (j0 + 1 == X.jcap) X.rbrow[r] = make_int2(tB, eB);
             }
             if (TRACK) {
                 const int row = row1 + r;
                 if (row <= a.m) {
-                    if (j0 + 1 <= a.n) {
+                    const int cA = X.col0 + j0 + 1, cB = cA + 1;  // global DP columns
+                    if (j0 + 1 <= X.w) {
                         if (LOCAL) {
-                            if (better(hA, row, j0 + 1, bs, bi, bj)) { bs = hA; bi = row; bj = j0 + 1; }
-                        } else if (hA == a.goal && (row < bi || (row == bi && j0 + 1 < bj))) {
-                            bi = row; bj = j0 + 1;
+                            if (better(hA, row, cA, bs, bi, bj)) { bs = hA; bi = row; bj = cA; }
+                        } else if (hA == a.goal && (row < bi || (row == bi && cA < bj))) {
+                            bi = row; bj = cA;
                         }
                     }
-                    if (j0 + 2 <= a.n) {
+                    if (j0 + 2 <= X.w) {
                         if (LOCAL) {
-                            if (better(hB, row, j0 + 2, bs, bi, bj)) { bs = hB; bi = row; bj = j0 + 2; }
-                        } else if (hB == a.goal && (row < bi || (row == bi && j0 + 2 < bj))) {
-                            bi = row; bj = j0 + 2;
+                            if (better(hB, row, cB, bs, bi, bj)) { bs = hB; bi = row; bj = cB; }
+                        } else if (hB == a.goal && (row < bi || (row == bi && cB < bj))) {
+                            bi = row; bj = cB;
                         }
                     }
                 }
@@ -243,42 +308,43 @@ struct Fill {
         L.out_t0 = tuA; L.out_f0 = fuA;
         L.out_t1 = tuB; L.out_f1 = fuB;
         if (SPM == 1 && sp_ptr != nullptr) {
-            if (j0 < a.n) { sp_ptr[j0] = tuA + gf; sp_ptr[a.sp_ld + j0] = fuA; }  // H = t + G_first
-            if (j0 + 1 < a.n) { sp_ptr[j0 + 1] = tuB + gf; sp_ptr[a.sp_ld + j0 + 1] = fuB; }
+            if (j0 < X.w) { sp_ptr[j0] = tuA + gf; sp_ptr[X.sp_ld + j0] = fuA; }  // H = t + G_first
+            if (j0 + 1 < X.w) { sp_ptr[j0 + 1] = tuB + gf; sp_ptr[X.sp_ld + j0 + 1] = fuB; }
         }
-        if (!TRACK && lane == 31) *reinterpret_cast<int4 *>(ring_out + (j0 & (RING - 1))) = make_int4(tuA, fuA, tuB, fuB);
+        if (!TRACK && lane == 31) sts_v4(ring_out + (uint32_t)(j0 & (RING - 1)) * 8u, make_int4(tuA, fuA, tuB, fuB));
         return tmax;
     }
 
     // Rare tiles (tile 0 with its lane guard, exact replays, generic special
     // rows): inlined so the lane state stays in registers, but not unrolled.
-    template <bool GUARD, bool TRACK, int SPM>
-    static __device__ __forceinline__ int tile(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
-                                               int2 *ring_out, const uint32_t *selr, int row1, int &bs, int &bi,
-                                               int &bj, int *sp_ptr, uint32_t smask)
+    template <bool GUARD, bool TRACK, int SPM, bool CAP = false>
+    static __device__ __forceinline__ int tile(const FillArgs &a, const StepInfo &X, Lane &L, int c, int lane,
+                                               uint32_t ring_in, uint32_t ring_out, uint32_t selr, int row1,
+                                               int &bs, int &bi, int &bj, int *sp_ptr, uint32_t smask)
     {
         int tmax = INT_MIN;
         const int k0 = c * STEPS;
 #pragma unroll 1
         for (int kk = 0; kk < STEPS; kk++)
-            tmax = step<GUARD, TRACK, SPM>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1, bs, bi, bj,
-                                           sp_ptr, smask);
+            tmax = step<GUARD, TRACK, SPM, CAP>(a, X, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1, bs, bi,
+                                                bj, sp_ptr, smask);
         return tmax;
     }
 
     // The hot path: no guard, no tracking; SP1 = this warp holds special rows
     // that are strip-bottom rows (k a multiple of ALPHA): predicated stores.
     template <bool SP1>
-    static __device__ __forceinline__ int tile_fast(const FillArgs &a, Lane &L, int c, int lane, const int2 *ring_in,
-                                                    int2 *ring_out, const uint32_t *selr, int *sp_ptr)
+    static __device__ __forceinline__ int tile_fast(const FillArgs &a, const StepInfo &X, Lane &L, int c, int lane,
+                                                    uint32_t ring_in, uint32_t ring_out, uint32_t selr,
+                                                    int *sp_ptr)
     {
         int tmax = INT_MIN;
         int d0 = 0, d1 = 0, d2 = 0;
         const int k0 = c * STEPS;
 #pragma unroll 2
         for (int kk = 0; kk < STEPS; kk++)
-            tmax = step<false, false, SP1 ? 1 : 0>(a, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, 0, d0, d1, d2,
-                                                   sp_ptr, 0u);
+            tmax = step<false, false, SP1 ? 1 : 0>(a, X, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, 0, d0, d1,
+                                                   d2, sp_ptr, 0u);
         return tmax;
     }
 
@@ -311,7 +377,8 @@ struct Fill {
 };
 
 // Boundary values of row 0 / column 0 as t = H - G_first (reading S3, and the
-// global initialisation of reading S9): column index j is 0-based (DP j+1).
+// global initialisation of reading S9): column index j is the GLOBAL 0-based
+// column (DP column j+1).
 template <bool LOCAL>
 __device__ __forceinline__ int2 top_boundary(const FillArgs &a, int j)
 {
@@ -319,39 +386,71 @@ __device__ __forceinline__ int2 top_boundary(const FillArgs &a, int j)
     return make_int2(-(a.go + (j + 1) * a.ge) - a.gf, NEG);  // H(0, j+1) = -(G_open + (j+1) G_ext)
 }
 
+__device__ __forceinline__ int ld_acquire_sys(const int *p)
+{
+    int v;
+    asm volatile("ld.acquire.sys.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys_s32(int *p, int v)
+{
+    asm volatile("st.release.sys.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ int2 ld_sys_int2(const int2 *p)
+{
+    int2 v;
+    asm volatile("ld.relaxed.sys.global.v2.s32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
+    return v;
+}
+
 template <int ALPHA, int NW, int W, bool LOCAL>
-__global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a)
+__global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_constant__ FillArgs a)
 {
     using F = Fill<ALPHA, NW, W, LOCAL>;
-    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW;
+    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int2 *rings = reinterpret_cast<int2 *>(smem_raw);                        // (NW+1) x RING
     uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * RING);  // SRING
     int *saves = reinterpret_cast<int *>(selr + SRING);                     // NW x NSAVE x 32
     __shared__ int s_band, s_abort;
 
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const uint32_t selr_base = (uint32_t)__cvta_generic_to_shared(selr);
+    const StripeArgs &S = a.st[blockIdx.x % a.nstripes];
+    const int NT = S.NT;
+    const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr;
     int bs = 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
     long long nrep = 0;
     if (*a.err) return;
+    StepInfo X;
+    X.w = S.w;
+    X.col0 = S.col0;
+    X.sp_ld = S.sp_ld;
+    X.sp_stride = S.sp_stride;
+    X.jcap = S.w - 1;
+    X.rbrow = nullptr;
+    // tiles in which a lane meets the capture column jcap (lane l at step jcap/2 + l)
+    const int cap_t0 = (X.jcap >> 1) / STEPS, cap_t1 = ((X.jcap >> 1) + 31) / STEPS;
 
     for (;;) {
         if (threadIdx.x == 0) {
-            int b = atomicAdd(a.ticket, 1);
+            int b = atomicAdd(S.ticket, 1);
             if (!LOCAL && b > ld_relaxed(a.hit_band)) b = a.nb;
+            if (ld_relaxed(a.err)) b = a.nb;
             s_band = b;
             s_abort = 0;
         }
         __syncthreads();
         const int b = s_band;
         if (b >= a.nb) break;
-        if (a.dbg && threadIdx.x == 0) a.dbg[80 * b] = gtimer();
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b] = gtimer();
 
         typename F::Lane L;
         const int row0 = b * BH + (warp * 32 + lane) * ALPHA;  // 0-based first row of the strip
         int *sp_ptr = nullptr;
         uint32_t smask = 0;
         bool warp_sp = false;
+        X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
         if (warp < NW) {
             const uint32_t w = row0 < a.m ? a.A2[row0 >> 4] : 0u;
             const int sh = (row0 & 15) * 2;
@@ -372,7 +471,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
                 }
                 if (smask) {
                     const int first = __ffs(smask) - 1;
-                    sp_ptr = a.sp + (long long)((row0 + first + 1) / a.k - 1) * a.sp_stride;
+                    sp_ptr = S.sp + (long long)((row0 + first + 1) / a.k - 1) * S.sp_stride;
                 }
             }
             warp_sp = __any_sync(0xffffffffu, smask != 0);
@@ -380,11 +479,13 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
         const int spm = (a.k > 0 && a.k % ALPHA == 0) ? 1 : 2;
 
         auto io_load = [&](int c) {
-            const int need = min((c + 1) * W, a.NT * W - SKEW);
+            const int need = min((c + 1) * W, NT * W - SKEW);
             if (b > 0) {
                 if (lane == 0) {
-                    while (ld_acquire(a.progress + b - 1) < need) {
+                    const unsigned long long t0 = gtimer();
+                    while (ld_acquire(S.progress + b - 1) < need) {
                         if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
+                        if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                         __nanosleep(64);
                     }
                 }
@@ -394,10 +495,13 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = c * W + x;
-                int2 v = (b == 0) ? top_boundary<LOCAL>(a, col) : __ldcg(a.rowb + col);
+                int2 v = (b == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb + col);
                 ring0[col & (RING - 1)] = v;
                 uint32_t code = 4u;
-                if (col < a.n) code = (__ldg(a.B2 + (col >> 4)) >> ((col & 15) * 2)) & 3u;
+                if (col < S.w) {
+                    const int gc = S.col0 + col;
+                    code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
+                }
                 selr[col & (SRING - 1)] = col_sel(code);
             }
         };
@@ -406,41 +510,73 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = cd * W - SKEW + x;
-                if (col >= 0) __stcg(a.rowb + col, ringN[col & (RING - 1)]);
+                if (col >= 0) __stcg(S.rowb + col, ringN[col & (RING - 1)]);
             }
             __threadfence();
             __syncwarp();
-            if (lane == 0) st_release(a.progress + b, cd * W + W - SKEW);
+            if (lane == 0) st_release(S.progress + b, cd * W + W - SKEW);
+        };
+        // left border of this warp's rows (stripes after the first): wait for the
+        // left neighbour's flags, then take (t, E) at column col0 - 1 as the state.
+        auto load_left = [&]() {
+            if (lane == 0) {
+                const int fi = b * NW + warp;
+                const unsigned long long t0 = gtimer();
+                while (ld_acquire_sys(S.lready + fi) != a.epoch || (fi > 0 && ld_acquire_sys(S.lready + fi - 1) != a.epoch)) {
+                    if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); break; }
+                    __nanosleep(64);
+                }
+            }
+            __syncwarp();
+#pragma unroll
+            for (int r = 0; r < ALPHA; r++) {
+                const int2 v = ld_sys_int2(S.lb + row0 + 1 + r);  // rows past m read padding, never used
+                L.t[r] = v.x;
+                L.e[r] = v.y;
+            }
+            if (row0 > 0) L.tprev = ld_sys_int2(S.lb + row0).x;
+            else L.tprev = LOCAL ? -a.gf : -(a.go + S.col0 * a.ge) - a.gf;  // t(0, col0 - 1)
         };
 
         if (warp == NW) io_load(0);
         __syncthreads();
-        if (a.dbg && threadIdx.x == 0) a.dbg[80 * b + 1] = gtimer();
-        const int S_END = a.NT + 2 * (NW - 1);
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 1] = gtimer();
+        const int S_END = NT + 2 * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s <= S_END; ++s) {
             if (warp < NW) {
                 const int c = s - 2 * warp;
-                if (c >= 0 && c < a.NT) {
-                    const int2 *rin = rings + warp * RING;
-                    int2 *rout = rings + (warp + 1) * RING;
+                if (c >= 0 && c < NT) {
+                    const uint32_t rin = pin((uint32_t)__cvta_generic_to_shared(rings + warp * RING));
+                    const uint32_t rout = pin((uint32_t)__cvta_generic_to_shared(rings + (warp + 1) * RING));
+                    const uint32_t selr_s = pin(selr_base);
+                    if (c == 0 && has_left) load_left();
                     int thr;
                     if (LOCAL) thr = max(max(bs, ld_relaxed(a.gbest)), 1);
                     else thr = a.goal;
                     F::save(L, sv, lane);
                     int tmax;
-                    if (c == 0 || (warp_sp && spm == 2)) {
-                        tmax = F::template tile<true, false, 2>(a, L, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, sp_ptr, smask);
+                    const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
+                    if (cap) {
+                        tmax = F::template tile<true, false, 2, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, smask);
+                        if (c == cap_t1) {
+                            // this warp's rows are complete at the stripe's last column
+                            __threadfence_system();
+                            __syncwarp();
+                            if (lane == 0) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
+                        }
+                    } else if (c == 0 || (warp_sp && spm == 2)) {
+                        tmax = F::template tile<true, false, 2>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, smask);
                     } else if (warp_sp) {
-                        tmax = F::template tile_fast<true>(a, L, c, lane, rin, rout, selr, sp_ptr);
+                        tmax = F::template tile_fast<true>(a, X, L, c, lane, rin, rout, selr_s, sp_ptr);
                     } else {
-                        tmax = F::template tile_fast<false>(a, L, c, lane, rin, rout, selr, nullptr);
+                        tmax = F::template tile_fast<false>(a, X, L, c, lane, rin, rout, selr_s, nullptr);
                     }
                     if (__any_sync(0xffffffffu, tmax >= thr)) {
                         // exact replay of this tile from the saved state (rare)
                         F::restore(L, sv, lane);
                         const int obs = bs, obi = bi, obj = bj;
-                        F::template tile<true, true, 0>(a, L, c, lane, rin, rout, selr, row0 + 1, bs, bi, bj, nullptr, 0u);
+                        F::template tile<true, true, 0>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr, 0u);
                         if (lane == 0) nrep++;
                         if (LOCAL) {
                             if (bs > obs) atomicMax(a.gbest, bs);
@@ -451,18 +587,18 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
                     }
                 }
             } else {
-                if (s + 1 < a.NT) io_load(s + 1);
+                if (s + 1 < NT) io_load(s + 1);
                 const int cd = s - 1 - 2 * (NW - 1);
                 if (cd >= 0) io_drain(cd);
                 if (!LOCAL && lane == 0 && ld_relaxed(a.hit_band) < b) s_abort = 1;
             }
             __syncthreads();
-            if (!LOCAL && s_abort) break;
+            if (s_abort) break;
         }
-        if (warp == NW && lane == 0 && !s_abort) st_release(a.progress + b, INT_MAX);
-        if (a.dbg && threadIdx.x == 0) a.dbg[80 * b + 15] = gtimer();
+        if (warp == NW && lane == 0 && !s_abort) st_release(S.progress + b, INT_MAX);
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 15] = gtimer();
         if (LOCAL && a.k > 0) {
-            // publish this band's special rows to the host
+            // publish this band's special rows (this stripe's slice) to the host
             __threadfence();
             __syncthreads();
             if (threadIdx.x == 0) {
@@ -470,7 +606,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const FillArgs a
                 long long q = (lo + a.k - 1) / a.k;
                 if (q * a.k <= hi) {
                     __threadfence_system();
-                    for (; q * a.k <= hi; q++) st_release_sys(a.row_done + (q - 1), 1u);
+                    for (; q * a.k <= hi; q++) st_release_sys(S.row_done + (q - 1), 1u);
                 }
             }
         }
