@@ -8,9 +8,12 @@ pass to the start cell (a8).  GCUPS = m n / (t 10^9).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl ours|reference]
 
-N > 1 (torchrun, one process per GPU): round 1 runs one independent replica
-of the workload per GPU (weak scaling, no data-path collective); the
-column-stripe exchange of 8(e) is not built yet.
+N > 1 (torchrun, one process per GPU): the column-stripe pipeline (a7): rank g
+owns columns [g n / N, (g+1) n / N) and hands each band's right-edge column to
+rank g+1 by peer stores over NVLink (CUDA IPC); strong scaling (the same
+matrix on N GPUs).  Special-row slices stay with their rank's sink; the
+reverse pass (tiny for C2) runs on rank 0.  SWB_SAME_DEVICE=1 maps every rank
+to cuda:0 with gloo (a functional check of the N > 1 path on one GPU).
 
 --impl reference: the CPU oracle (oracle/, single-threaded plain C) timed on a
 bounded row-band sample of the same workload on the host cores.
@@ -107,7 +110,7 @@ class ClockSampler:
 
 # ---------------------------------------------------------------- oracle (CPU) timing
 
-def oracle_sample(A, B, k, target_s=12.0):
+def oracle_sample(A, B, target_s=12.0):
     """Time the oracle's band recompute (the same loop as its Stage 1) on a
     bounded sample of rows of the workload: single-threaded, as it stands."""
     import numpy as np
@@ -115,7 +118,6 @@ def oracle_sample(A, B, k, target_s=12.0):
     import oracle
 
     n = len(B)
-    # calibrate on a small band, then size the sample for ~target_s seconds
     ma, mi, go, ge = SCORING
     Htop = np.zeros(n + 1, np.int64)
     Ftop = np.full(n + 1, oracle.NEG, np.int64)
@@ -132,6 +134,35 @@ def oracle_sample(A, B, k, target_s=12.0):
     return cells / dt / 1e9, f"oracle.band rows 1..{rows} x all {n} columns of the workload ({cells:.3g} cells, {dt:.1f} s, 1 thread)", dt
 
 
+def reference_arm(args, cfg, k, rank, world):
+    if rank != 0:
+        return 0  # rank 0 alone runs the CPU oracle
+    import synth
+    import oracle
+
+    A, B = synth.make_pair(cfg)
+    oracle.build()
+    vals, samples, times = [], "", []
+    for _ in range(args.warmup):
+        oracle_sample(A, B, target_s=2.0)
+    for _ in range(args.steps):
+        v, samples, dt = oracle_sample(A, B, target_s=10.0)
+        vals.append(v)
+        times.append(dt)
+    value = statistics.median(vals)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GCUPS",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
+        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": {"workload": cfg.name, "m": cfg.m, "n": cfg.n, "k": k, "scoring": list(SCORING)},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": samples},
+        "e2e": {"value": round(value, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 # ---------------------------------------------------------------- main
 
 def main():
@@ -146,48 +177,37 @@ def main():
 
     cfg = synth.CONFIGS[args.workload]
     k = cfg.k if args.k is None else args.k
-
     if args.impl == "reference":
-        if rank != 0:
-            return 0  # rank 0 alone runs the CPU oracle
-        A, B = synth.make_pair(cfg)
-        import oracle
-
-        oracle.build()
-        vals, samples = [], ""
-        for _ in range(args.warmup):
-            oracle_sample(A, B, k, target_s=2.0)
-        times = []
-        for _ in range(args.steps):
-            v, samples, dt = oracle_sample(A, B, k, target_s=10.0)
-            vals.append(v)
-            times.append(dt)
-        value = statistics.median(vals)
-        line = {
-            "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GCUPS",
-            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-            "config": {"workload": cfg.name, "m": cfg.m, "n": cfg.n, "k": k, "scoring": list(SCORING)},
-            "cpu_baseline": {"value": round(value, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": samples},
-            "e2e": {"value": round(value, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-        }
-        print(json.dumps(line), flush=True)
-        return 0
+        return reference_arm(args, cfg, k, rank, world)
 
     import torch
 
+    same_dev = bool(os.environ.get("SWB_SAME_DEVICE"))
+    dev_index = 0 if same_dev else local_rank
+    torch.cuda.set_device(dev_index)
+    dev = torch.device("cuda", dev_index)
+    dist = None
     if world > 1:
         import torch.distributed as dist
 
-        torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    else:
-        torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
+        if same_dev:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if same_dev else dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
 
     from paper_conf_ipps_sandesm11_b200 import Context, build
 
+    if rank == 0:
+        build.build()
+    if world > 1:
+        dist.barrier()
     build.build()
     A, B = synth.make_pair(cfg)
     m, n = len(A), len(B)
@@ -195,8 +215,13 @@ def main():
     dB = torch.from_numpy(B).to(dev)
     stream = torch.cuda.current_stream(dev)
     sptr = stream.cuda_stream
-    ctx = Context(local_rank)
+    ctx = Context(dev_index)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    grp = None
+    if world > 1:
+        from paper_conf_ipps_sandesm11_b200.parallel import StripeGroup
+
+        grp = StripeGroup(ctx, rank, world, max_rows=m)
 
     sink_rows = [0]
 
@@ -205,50 +230,54 @@ def main():
         return False
 
     def step():
-        r, _ = ctx.align_stage1_dev(dA.data_ptr(), m, dB.data_ptr(), n, *SCORING, k=k, sink=sink, stream=sptr)
+        """One step on this rank; returns (best, start, stage-1 stats, launches)."""
+        if grp is None:
+            r, _ = ctx.align_stage1_dev(dA.data_ptr(), m, dB.data_ptr(), n, *SCORING, k=k, sink=sink, stream=sptr)
+            best = r.astuple()
+        else:
+            best, _, _ = grp.align_stage1(dA.data_ptr(), m, dB.data_ptr(), n, SCORING, k=k, sink=sink, stream=sptr)
         s1 = ctx.stats()
-        st = ctx.reverse_goal_dev(dA.data_ptr(), r.i, dB.data_ptr(), r.j, r.score, *SCORING, stream=sptr)
-        s2 = ctx.stats()
-        return r, st, s1, s2
+        launches = s1["kernel_launches"]
+        start = None
+        if rank == 0 and best[0] > 0:
+            st = ctx.reverse_goal_dev(dA.data_ptr(), best[1], dB.data_ptr(), best[2], best[0], *SCORING, stream=sptr)
+            start = st.astuple()
+            launches += ctx.stats()["kernel_launches"]
+        return best, start, s1, launches
 
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     if world > 1:
-        torch.distributed.barrier()
+        dist.barrier()
 
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     fill_ms, launches, replays, sp_bytes = [], 0, 0, 0
     results = set()
     sink_rows[0] = 0
-    with ClockSampler(local_rank) as clk:
+    with ClockSampler(dev_index) as clk:
         torch.cuda.synchronize()
         if world > 1:
-            torch.distributed.barrier()
+            dist.barrier()
         t_wall0 = time.perf_counter()
         for s in range(args.steps):
             flush.fill_(s & 0xFF)  # evict L2 between timed steps (outside the events)
             ev[s][0].record(stream)
-            r, st, s1, s2 = step()
+            best, start, s1, nl = step()
             ev[s][1].record(stream)
             fill_ms.append(s1["fill_ms"])
-            launches += s1["kernel_launches"] + s2["kernel_launches"]
+            launches += nl
             replays += s1["replays"]
             sp_bytes += s1["special_bytes_d2h"]
-            results.add((r.astuple(), st.astuple()))
+            results.add((best, start))
         torch.cuda.synchronize()
         if world > 1:
-            torch.distributed.barrier()
+            dist.barrier()
         t_wall = time.perf_counter() - t_wall0
     step_ms = [a.elapsed_time(b) for a, b in ev]
-    tot_ms = sum(step_ms)
-    if world > 1:
-        t = torch.tensor([tot_ms], device=dev, dtype=torch.float64)
-        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-        tot_ms = float(t.item())
-    ms_per_step = tot_ms / args.steps
+    ms_per_step = max_over_ranks(sum(step_ms) / args.steps)
     cells = float(m) * float(n)
-    value = world * cells / (ms_per_step * 1e-3) / 1e9
+    value = cells / (ms_per_step * 1e-3) / 1e9
     assert len(results) == 1, f"non-deterministic results {results}"
     (best, start) = results.pop()
     rows_per_step = sink_rows[0] // max(1, args.steps)
@@ -260,14 +289,23 @@ def main():
         hB = torch.from_numpy(B).pin_memory()
         import ctypes
 
+        def host_view(t, size):
+            return np.ctypeslib.as_array((ctypes.c_uint8 * size).from_address(t.data_ptr()))
+
         def e2e_step():
-            r, _ = ctx.align_stage1(np.ctypeslib.as_array((ctypes.c_uint8 * m).from_address(hA.data_ptr())),
-                                    np.ctypeslib.as_array((ctypes.c_uint8 * n).from_address(hB.data_ptr())),
-                                    *SCORING, k=k, sink=sink)
-            st = ctx.reverse_goal(np.ctypeslib.as_array((ctypes.c_uint8 * m).from_address(hA.data_ptr())), r.i,
-                                  np.ctypeslib.as_array((ctypes.c_uint8 * n).from_address(hB.data_ptr())), r.j,
-                                  r.score, *SCORING)
-            return r, st
+            if grp is None:
+                r, _ = ctx.align_stage1(host_view(hA, m), host_view(hB, n), *SCORING, k=k, sink=sink)
+                b = r.astuple()
+                st = ctx.reverse_goal(host_view(hA, m), b[1], host_view(hB, n), b[2], b[0], *SCORING).astuple() if b[0] > 0 else None
+                return b, st
+            # multi-GPU: copy this step's inputs host -> device, then the stripe call
+            dA.copy_(hA, non_blocking=True)
+            dB.copy_(hB, non_blocking=True)
+            b, _, _ = grp.align_stage1(dA.data_ptr(), m, dB.data_ptr(), n, SCORING, k=k, sink=sink, stream=sptr)
+            st = None
+            if rank == 0 and b[0] > 0:
+                st = ctx.reverse_goal(host_view(hA, m), b[1], host_view(hB, n), b[2], b[0], *SCORING).astuple()
+            return b, st
 
         e2e_step()
         torch.cuda.synchronize()
@@ -275,27 +313,29 @@ def main():
         for s in range(args.steps):
             flush.fill_(s & 0xFF)
             torch.cuda.synchronize()
+            if world > 1:
+                dist.barrier()
             t0 = time.perf_counter()
-            r, st = e2e_step()
+            b, st = e2e_step()
+            torch.cuda.synchronize()
             ts.append(time.perf_counter() - t0)
-            assert (r.astuple(), st.astuple()) == (best, start)
-        e2e_s = sum(ts) / len(ts)
-        if world > 1:
-            t = torch.tensor([e2e_s], device=dev, dtype=torch.float64)
-            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            e2e_s = float(t.item())
-        h2d = m + n + best[1] + best[2]
+            assert (b, st) == (best, start)
+        e2e_s = max_over_ranks(sum(ts) / len(ts))
+        h2d = m + n + ((best[1] + best[2]) if rank == 0 else 0)
         d2h = sp_bytes // args.steps + 3 * 16
-        e2e = {"value": round(world * cells / e2e_s / 1e9, 3), "unit": "GCUPS", "h2d_bytes_per_step": int(h2d),
+        e2e = {"value": round(cells / e2e_s / 1e9, 3), "unit": "GCUPS", "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h), "ms_per_step": round(1e3 * e2e_s, 3)}
 
+    fill_avg = max_over_ranks(statistics.mean(fill_ms))
     if rank != 0:
+        ctx.close()
+        if world > 1:
+            dist.destroy_process_group()
         return 0
 
     clocks = clk.summary()
     # ---- roofline of the dominant kernel (the fill), from live CUDA events on its stream
-    fill_avg = statistics.mean(fill_ms)
-    achieved = cells / (fill_avg * 1e-3) / 1e9
+    achieved = cells / (fill_avg * 1e-3) / 1e9 / world  # per GPU
     sm_max = clocks.get("sm_max_mhz") or 1965.0
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -307,33 +347,35 @@ def main():
     traffic = None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        if tr.get("workload") == cfg.name:
+        if tr.get("workload") == cfg.name and world == 1:
             traffic = tr.get("fill_dram_bytes_per_launch")
     except Exception:
         pass
     roofline = {"bound": "alu", "achieved": round(achieved, 2), "peak": round(peak, 1), "unit": "GCUPS",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
                 "peak_basis": f"{nsm} SM x {ROOF_CELLS_PER_CLK_SM} cells/clk/SM x {sm_max:.0f} MHz (measured pipe rates, DESIGN.md 5)",
-                "fill_ms": round(fill_avg, 3),
+                "fill_ms": round(fill_avg, 3), "per": "GPU",
                 "peak_at_measured_clock": round(nsm * ROOF_CELLS_PER_CLK_SM * (clocks.get('sm_mhz') or sm_max) * 1e-3, 1)}
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
-        v, sample, _ = oracle_sample(A, B, k, target_s=12.0)
+        v, sample, _ = oracle_sample(A, B, target_s=12.0)
         cpu = {"value": round(v, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": sample}
 
     line = {
         "metric": METRIC, "value": round(value, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": (round(value / PAPER_GCUPS[cfg.name], 2) if cfg.name in PAPER_GCUPS and world == 1 else None),
+        "scaling": "strong" if world > 1 else "weak",
+        "vs_baseline": (round(value / PAPER_GCUPS[cfg.name], 2) if cfg.name in PAPER_GCUPS else None),
         "dtype": "int32", "data": "synthetic",
         "config": {"workload": cfg.name, "m": m, "n": n, "k": k, "scoring": list(SCORING),
                    "step": "encode + Stage-1 fill + special rows to host sink + reverse goal pass",
                    "l2": "flushed between timed steps (256 MiB write)",
-                   "parallelism": "single" if world == 1 else f"replicas x{world}",
+                   "parallelism": "single" if world == 1 else f"column stripes x{world} (NVLink border hand-off)"
+                   + (" [same device, functional check]" if same_dev else ""),
                    "kernel": {"alpha": s1["alpha"], "warps": s1["warps"], "width": s1["width"], "grid": s1["grid"]},
                    "baseline_note": "vs_baseline = value / paper Table IV 543Kx536K flush (21.419 GCUPS, GTX 285, real DNA)"},
-        "result": {"best": list(best), "start": list(start), "special_rows_per_step": rows_per_step},
+        "result": {"best": list(best), "start": list(start) if start else None, "special_rows_per_step": rows_per_step},
         "roofline": roofline,
         "cpu_baseline": cpu,
         "e2e": e2e,
@@ -345,7 +387,7 @@ def main():
     print(json.dumps(line), flush=True)
     ctx.close()
     if world > 1:
-        torch.distributed.destroy_process_group()
+        dist.destroy_process_group()
     return 0
 
 
