@@ -12,7 +12,9 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libcudalign_b200.so")
 SOURCES = [os.path.join(HERE, "csrc", "sw_api.cu")]
-DEPS = SOURCES + [os.path.join(HERE, "csrc", "sw_fill.cuh"), os.path.join(ROOT, "include", "cudalign_b200.h")]
+import glob
+
+DEPS = sorted(glob.glob(os.path.join(HERE, "csrc", "*"))) + [os.path.join(ROOT, "include", "cudalign_b200.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",

@@ -16,6 +16,7 @@
 
 #include "../../include/cudalign_b200.h"
 #include "sw_fill.cuh"
+#include "sw_fill16.cuh"
 
 using namespace swb;
 
@@ -102,6 +103,8 @@ struct Variant {
     int alpha, nw, w;
     const void *local_fn, *global_fn;
     size_t smem;
+    const void *packed_fn;  // packed 16x2 Stage-1 kernel with the same band geometry (alpha 16 only)
+    size_t smem16;
 };
 
 template <int ALPHA, int NW, int W>
@@ -114,6 +117,12 @@ static Variant make_variant()
     v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
     v.global_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, false>;
     v.smem = Fill<ALPHA, NW, W, true>::smem_bytes();
+    v.packed_fn = nullptr;
+    v.smem16 = 0;
+    if constexpr (ALPHA == 16) {
+        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W>;
+        v.smem16 = Fill16<NW, W>::smem_bytes();
+    }
     return v;
 }
 
@@ -172,6 +181,7 @@ struct sw_ctx {
     char errbuf[512] = {0};
     int variant_override = -1;
     int vstripes = 1;           // virtual stripes for the single-process calls
+    int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
     long long timeout_ns = 120ll * 1000000000ll;
 };
 
@@ -277,11 +287,13 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
             const Variant &v = variant_for(i);
             cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
             cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+            if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaFuncSetAttribute"); break; }
         if (const char *ov = getenv("SWB_VARIANT")) ctx->variant_override = atoi(ov);
         if (const char *vs = getenv("SWB_VSTRIPES")) ctx->vstripes = std::max(1, std::min(MAX_STRIPES, atoi(vs)));
         if (const char *to = getenv("SWB_TIMEOUT_S")) ctx->timeout_ns = (long long)(atof(to) * 1e9);
+        if (const char *pk = getenv("SWB_PACKED")) ctx->packed = atoi(pk);
     } while (0);
     if (rc) { sw_shutdown(ctx); return rc; }
     *out = ctx;
@@ -403,9 +415,40 @@ struct Job {
 };
 }  // namespace
 
+// Kernel choice per call: the packed 16x2 kernel with the
+// 4-warp geometry when it applies and the band pipeline runs for >= 2 waves
+// (steady state dominates); otherwise the int32 kernel with 8 warps (best when
+// all bands are in flight at once and the pipeline skew dominates, e.g. C2).
+// Deterministic in (m, n, k, scoring), so all ranks of a stripe group agree.
+static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
+{
+    const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
+    const bool packed_ok = ctx->packed && J.local && (J.k == 0 || J.k % 16 == 0) &&
+                           650ll * (pmax_abs + J.go + J.ge) + 1024 < 30000;
+    if (ctx->variant_override >= 0) {
+        const Variant &V = variant_for(ctx->variant_override);
+        *use16 = packed_ok && V.packed_fn;
+        return V;
+    }
+    const Variant &V0 = variant_for(0);
+    if (packed_ok && V0.packed_fn) {
+        int per_sm = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, V0.packed_fn, V0.nw * 32 + 32, V0.smem16);
+        const long long bh = (long long)V0.alpha * 32 * V0.nw;
+        const long long nb = (J.m + bh - 1) / bh;
+        if (nb >= 2ll * std::max(1, per_sm) * ctx->num_sms) {
+            *use16 = true;
+            return V0;
+        }
+    }
+    *use16 = false;
+    return variant_for(DEFAULT_VARIANT);
+}
+
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
 {
-    const Variant &V = ctx_variant(ctx);
+    bool use16 = false;
+    const Variant &V = choose_variant(ctx, J, &use16);
     const int W = V.w;
     const int BH = V.alpha * 32 * V.nw;
     const int m = (int)J.m, n = (int)J.n;
@@ -454,8 +497,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             return SW_EINVAL;
         }
     }
+    const void *fill_fn = use16 ? V.packed_fn : (J.local ? V.local_fn : V.global_fn);
+    const size_t fill_smem = use16 ? V.smem16 : V.smem;
     int blocks_per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, J.local ? V.local_fn : V.global_fn, V.nw * 32 + 32, V.smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, fill_fn, V.nw * 32 + 32, fill_smem);
     if (blocks_per_sm < 1) blocks_per_sm = 1;
     // every CTA of every stripe must be co-resident (stripes wait on each other)
     int per_stripe = std::max(1, std::min(nb, blocks_per_sm * ctx->num_sms / NS));
@@ -589,7 +634,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     }
     {
         void *args[] = {&a};
-        CK(cudaLaunchKernel(J.local ? V.local_fn : V.global_fn, dim3(grid), dim3(V.nw * 32 + 32), args, V.smem, st));
+        CK(cudaLaunchKernel(fill_fn, dim3(grid), dim3(V.nw * 32 + 32), args, fill_smem, st));
     }
     CK(cudaEventRecord(ctx->ev[2], st));
     sw_reduce_kernel<<<1, 256, 0, st>>>((const int4 *)ctx->slots.p, grid, J.local ? 1 : 0, d_hit_key, J.goal, d_res);
@@ -657,7 +702,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     ctx->stats.replays += (long long)*(unsigned long long *)(ctx->res_h + 2);
     ctx->stats.special_rows += nsp;
     ctx->stats.special_bytes_d2h += bytes;
-    ctx->stats.alpha = V.alpha;
+    ctx->stats.alpha = use16 ? -V.alpha : V.alpha;  // negative: packed 16x2 kernel
     ctx->stats.warps = V.nw;
     ctx->stats.width = W;
     ctx->stats.grid = grid;
@@ -757,14 +802,35 @@ extern "C" int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, co
 
 // ---------------------------------------------------------------- multi-GPU column stripes
 
+// Receive-area geometry valid for every kernel variant: rows cover the padded
+// last band of the tallest band height, flags (band, warp) the finest split.
+static size_t recv_rows(int64_t max_rows)
+{
+    int64_t bh_max = 0;
+    for (int i = 0; i < NVARIANTS; i++) bh_max = std::max<int64_t>(bh_max, (int64_t)variant_for(i).alpha * 32 * variant_for(i).nw);
+    return (size_t)(((max_rows + bh_max - 1) / bh_max) * bh_max + 2);
+}
+static size_t recv_flags(int64_t max_rows)
+{
+    size_t f = 0;
+    for (int i = 0; i < NVARIANTS; i++) {
+        const Variant &v = variant_for(i);
+        const int64_t bh = (int64_t)v.alpha * 32 * v.nw;
+        f = std::max<size_t>(f, (size_t)(((max_rows + bh - 1) / bh) * v.nw + 1));
+    }
+    return f;
+}
+
 extern "C" int sw_stripe_export(sw_ctx *ctx, int64_t max_rows, void *handle_out)
 {
     if (!ctx || max_rows < 0 || !handle_out) return SW_EINVAL;
     if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
-    const Variant &V = ctx_variant(ctx);
-    const int64_t BH = (int64_t)V.alpha * 32 * V.nw;
-    const int64_t nb = (max_rows + BH - 1) / BH;
-    int rc = grow_recv(ctx, ctx->recv, (size_t)(nb * BH + 2), (size_t)(nb * V.nw + 1));
+    // exact geometry: the left neighbour locates the flags from max_rows alone
+    if (ctx->recv.base && (ctx->recv.rows != recv_rows(max_rows) || ctx->recv.flags != recv_flags(max_rows))) {
+        cudaFree(ctx->recv.base);
+        ctx->recv = RecvArea{};
+    }
+    int rc = grow_recv(ctx, ctx->recv, recv_rows(max_rows), recv_flags(max_rows));
     if (rc) return rc;
     cudaIpcMemHandle_t h;
     CK(cudaIpcGetMemHandle(&h, ctx->recv.base));
@@ -784,9 +850,7 @@ extern "C" int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t 
     cudaIpcMemHandle_t h;
     memcpy(&h, right_handle, sizeof(h));
     CK(cudaIpcOpenMemHandle(&ctx->right_base, h, cudaIpcMemLazyEnablePeerAccess));
-    const Variant &V = ctx_variant(ctx);
-    const int64_t BH = (int64_t)V.alpha * 32 * V.nw;
-    ctx->right_rows = (size_t)(((max_rows + BH - 1) / BH) * BH + 2);
+    ctx->right_rows = recv_rows(max_rows);
     return SW_OK;
 }
 

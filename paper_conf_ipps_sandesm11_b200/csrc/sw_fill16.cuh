@@ -1,0 +1,469 @@
+// sw_fill16.cuh -- packed 16x2 Stage-1 fill.
+//
+// Same band pipeline, I/O warp, row border, special rows, stripes and exact
+// best-cell replay as sw_fill.cuh (read that first); what changes is the lane:
+//
+//  * A lane owns 16 rows as 8 packed slots: slot s holds row s in its low
+//    half at column j and row s+8 in its high half at column j-1, so ONE
+//    instruction updates two cells that do not depend on each other.  Slot 0's
+//    high half takes row 7's values of the previous step (a PRMT), so the
+//    vertical chain is 8 slots long instead of 16.
+//  * Values are biased unsigned 16-bit numbers in a warp-uniform frame
+//    q = x - B + 32768 (x the int32 value), re-based at every tile.  Within a
+//    warp all live values lie within ~650 (p_max + G_first) of each other
+//    (|H(i,j) - H(i-1,j)| <= p_max + G_first), far inside
+//    16 bits for the supported scorings, so the frame never wraps.
+//  * Adds that cannot borrow across halves use IMAD on the FMA pipe
+//    (q - G_ext, q - G_first); the signed substitution score is added with the
+//    per-half VIADDMNMX.U16x2; maxima use VIMNMX(3).U16x2.  The local 0 floor
+//    is the frame's image of 0.
+//  * Everything that leaves the lane (warp ring, special rows, the right
+//    border of a stripe, replay tracking) is converted back to int32.
+//
+// Results are bit-identical to the int32 kernel at every real cell; the two
+// differences are internal and exact: E(i,0) and F(0,j) start at t instead of
+// -infinity (both give E(i,1) = t(i,0), F(1,j) = t(0,j)), and pad columns use
+// base code 0 (they only feed pad cells; tracking ignores them).
+#pragma once
+#include "sw_fill.cuh"
+
+namespace swb {
+
+constexpr int BIAS16 = 32768;
+
+__device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(lo & 0xffff) | ((uint32_t)hi << 16); }
+__device__ __forceinline__ int lo16(uint32_t v) { return (int)(v & 0xffffu); }
+__device__ __forceinline__ int hi16(uint32_t v) { return (int)(v >> 16); }
+
+// Per-column selector parts for the packed PRMT: low byte = nibbles selecting
+// P[c] with sign replication (low half), high byte = nibbles selecting Q[c]
+// (bytes 4..7) for the high half.
+__device__ __forceinline__ uint32_t col_sel16(uint32_t code)
+{
+    const uint32_t lo = code | ((code | 8u) << 4);
+    const uint32_t hi = (code + 4u) | (((code + 4u) | 8u) << 4);
+    return lo | (hi << 8);
+}
+
+template <int NW, int W>
+struct Fill16 {
+    static constexpr int ALPHA = 16, BH = ALPHA * 32 * NW;
+    static constexpr int RING = Smem<W, NW>::RING;
+    static constexpr int SRING = Smem<W, NW>::SRING;
+    static constexpr int SKEW = 63;     // lane 31's output column lags lane 0's by 2*31 + 1
+    static constexpr int STEPS = W;     // one column per lane step
+    static constexpr int NSAVE = 20;
+    static_assert(W % 64 == 0 && W > SKEW, "W multiple of 64, larger than the warp skew");
+
+    static size_t smem_bytes()
+    {
+        return sizeof(int2) * RING * (NW + 1) + sizeof(uint32_t) * SRING + sizeof(int) * NSAVE * 32 * NW;
+    }
+
+    struct Lane {
+        uint32_t P[8], Q[8];  // int8x4 profiles of rows s (low halves) and s+8 (high halves)
+        uint32_t e[8], t[8];  // packed E and t = H - G_first of the previous column of each half
+        uint32_t tprev;       // packed diagonal input of slot 0
+        uint32_t f7;          // packed F of slot 7 after the last step (row 15 in the high half)
+        uint32_t selhi;       // high-half selector part of the previous column
+        int B;                // warp-uniform frame base
+        uint32_t FL;          // packed frame image of the local floor 0
+    };
+
+    static __device__ __forceinline__ int toabs(const Lane &L, int q) { return q - BIAS16 + L.B; }
+    static __device__ __forceinline__ int tofr(const Lane &L, int x) { return x - L.B + BIAS16; }
+
+    // One lane step: low half at local column jl = k - 2 lane, high half at jl - 1.
+    template <bool GUARD, bool TRACK, bool SP1, bool CAP>
+    static __device__ __forceinline__ uint32_t step(const FillArgs &a, const StepInfo &X, Lane &L, int k, int lane,
+                                                    uint32_t ring_in, uint32_t ring_out, uint32_t selr, uint32_t tmax,
+                                                    int row1, int &bs, int &bi, int &bj, int *sp_ptr)
+    {
+        uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[7], 1);
+        uint32_t up_f = __shfl_up_sync(0xffffffffu, L.f7, 1);
+        const int jl = k - 2 * lane;
+        if (lane == 0) {
+            int2 v;
+            asm volatile("ld.shared.v2.s32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(ring_in + (uint32_t)(jl & (RING - 1)) * 8u) : "memory");
+            // F_in only enters as max(F_in - G_ext, t_in): clamping it to >= t_in is exact
+            up_t = (uint32_t)tofr(L, v.x) << 16;
+            up_f = (uint32_t)tofr(L, max(v.y, v.x)) << 16;
+        }
+        Lane S;
+        if (GUARD) S = L;
+        const uint32_t tmax_in = tmax;
+        // slot-0 inputs: low = upper lane's row 15 (its high half), high = own row 7 (low half of slot 7)
+        uint32_t tu = __byte_perm(up_t, L.t[7], 0x5432);
+        uint32_t fu = __byte_perm(up_f, L.f7, 0x5432);
+        uint32_t td = L.tprev;
+        L.tprev = tu;
+        const uint32_t sw = lds_v2u(selr + (uint32_t)(jl & (SRING - 1)) * 4u).x;
+        const uint32_t sel = (sw & 0xffu) | L.selhi;
+        L.selhi = sw & 0xff00u;  // nibbles 2,3 (bytes 2,3 of the result) for the next column
+        const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
+#pragma unroll
+        for (int s = 0; s < 8; s += 2) {
+            const uint32_t e0 = __vmaxu2((uint32_t)imad((int)L.e[s], a.one, nge2), L.t[s]);
+            fu = __vmaxu2((uint32_t)imad((int)fu, a.one, nge2), tu);
+            const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
+            const uint32_t h0 = __viaddmax_u16x2(td, p0, __vimax3_u16x2(e0, fu, L.FL));
+            td = L.t[s];
+            const uint32_t t0 = (uint32_t)imad((int)h0, a.one, ngf2);
+            tu = t0;
+            L.e[s] = e0;
+            L.t[s] = t0;
+            const uint32_t e1 = __vmaxu2((uint32_t)imad((int)L.e[s + 1], a.one, nge2), L.t[s + 1]);
+            fu = __vmaxu2((uint32_t)imad((int)fu, a.one, nge2), tu);
+            const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
+            const uint32_t h1 = __viaddmax_u16x2(td, p1, __vimax3_u16x2(e1, fu, L.FL));
+            td = L.t[s + 1];
+            const uint32_t t1 = (uint32_t)imad((int)h1, a.one, ngf2);
+            tu = t1;
+            L.e[s + 1] = e1;
+            L.t[s + 1] = t1;
+            tmax = __vimax3_u16x2(tmax, h0, h1);
+            if (TRACK) {
+                const uint32_t hs[2] = {h0, h1};
+#pragma unroll
+                for (int q = 0; q < 2; q++) {
+                    const int rlo = row1 + s + q, rhi = rlo + 8;
+                    if (jl >= 0 && jl < X.w && rlo <= a.m) {
+                        const int v = toabs(L, lo16(hs[q])), c = X.col0 + jl + 1;
+                        if (better(v, rlo, c, bs, bi, bj)) { bs = v; bi = rlo; bj = c; }
+                    }
+                    if (jl >= 1 && jl - 1 < X.w && rhi <= a.m) {
+                        const int v = toabs(L, hi16(hs[q])), c = X.col0 + jl;
+                        if (better(v, rhi, c, bs, bi, bj)) { bs = v; bi = rhi; bj = c; }
+                    }
+                }
+            }
+            if (CAP) {
+                if (jl == X.jcap) {
+                    X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
+                    X.rbrow[s + 1] = make_int2(toabs(L, lo16(t1)), toabs(L, lo16(e1)));
+                }
+                if (jl - 1 == X.jcap) {
+                    X.rbrow[s + 8] = make_int2(toabs(L, hi16(t0)), toabs(L, hi16(e0)));
+                    X.rbrow[s + 9] = make_int2(toabs(L, hi16(t1)), toabs(L, hi16(e1)));
+                }
+            }
+        }
+        L.f7 = fu;
+        if (GUARD) {
+            // lanes left of column 0 keep their state; at jl == 0 only the high half waits
+            const uint32_t keep = (jl >= 0 ? 0x0000ffffu : 0u) | (jl >= 1 ? 0xffff0000u : 0u);
+#pragma unroll
+            for (int s = 0; s < 8; s++) {
+                L.e[s] = (L.e[s] & keep) | (S.e[s] & ~keep);
+                L.t[s] = (L.t[s] & keep) | (S.t[s] & ~keep);
+            }
+            if (jl < 0) {
+                L.tprev = S.tprev;
+                L.f7 = S.f7;
+                L.selhi = S.selhi;
+            }
+            tmax = (tmax & keep) | (tmax_in & ~keep);
+        }
+        const int jo = jl - 1;  // row 15's column (high half of slot 7)
+        if (SP1 && sp_ptr != nullptr && jo >= 0 && jo < X.w) {
+            sp_ptr[jo] = toabs(L, hi16(L.t[7])) + a.gf;  // H = t + G_first
+            sp_ptr[X.sp_ld + jo] = toabs(L, hi16(L.f7));
+        }
+        if (!TRACK && lane == 31 && (!GUARD || jo >= 0)) {
+            // (t, F) of row 15 at column jo for the next warp (int32, absolute)
+            asm volatile("st.shared.v2.s32 [%0], {%1, %2};" ::"r"(ring_out + (uint32_t)(jo & (RING - 1)) * 8u),
+                         "r"(toabs(L, hi16(L.t[7]))), "r"(toabs(L, hi16(L.f7))) : "memory");
+        }
+        return tmax;
+    }
+
+    template <bool GUARD, bool TRACK, bool SP1, bool CAP>
+    static __device__ __forceinline__ uint32_t tile(const FillArgs &a, const StepInfo &X, Lane &L, int c, int lane,
+                                                    uint32_t ring_in, uint32_t ring_out, uint32_t selr, int row1,
+                                                    int &bs, int &bi, int &bj, int *sp_ptr)
+    {
+        uint32_t tmax = 0;
+        const int k0 = c * STEPS;
+        if (GUARD || TRACK || CAP) {
+#pragma unroll 1
+            for (int kk = 0; kk < STEPS; kk++)
+                tmax = step<GUARD, TRACK, SP1, CAP>(a, X, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1, bs,
+                                                   bi, bj, sp_ptr);
+        } else {
+#pragma unroll 4
+            for (int kk = 0; kk < STEPS; kk++)
+                tmax = step<false, false, SP1, false>(a, X, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1,
+                                                      bs, bi, bj, sp_ptr);
+        }
+        return tmax;
+    }
+
+    // Re-base the frame to lane 0's slot-0 low value (warp-uniform shift).
+    static __device__ __forceinline__ void rebase(const FillArgs &a, Lane &L)
+    {
+        const int d = __shfl_sync(0xffffffffu, lo16(L.t[0]), 0) - BIAS16;
+        const int d2 = -(d * 0x10001);
+#pragma unroll
+        for (int s = 0; s < 8; s++) {
+            L.e[s] = (uint32_t)imad((int)L.e[s], a.one, d2);
+            L.t[s] = (uint32_t)imad((int)L.t[s], a.one, d2);
+        }
+        L.tprev = (uint32_t)imad((int)L.tprev, a.one, d2);
+        L.f7 = (uint32_t)imad((int)L.f7, a.one, d2);
+        L.B += d;
+        const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
+        L.FL = (uint32_t)fl * 0x10001u;
+    }
+
+    static __device__ __forceinline__ void save(const Lane &L, int *sv, int lane)
+    {
+#pragma unroll
+        for (int s = 0; s < 8; s++) {
+            sv[s * 32 + lane] = (int)L.e[s];
+            sv[(8 + s) * 32 + lane] = (int)L.t[s];
+        }
+        sv[16 * 32 + lane] = (int)L.tprev;
+        sv[17 * 32 + lane] = (int)L.f7;
+        sv[18 * 32 + lane] = (int)L.selhi;
+        sv[19 * 32 + lane] = L.B;
+    }
+    static __device__ __forceinline__ void restore(Lane &L, const int *sv, int lane)
+    {
+#pragma unroll
+        for (int s = 0; s < 8; s++) {
+            L.e[s] = (uint32_t)sv[s * 32 + lane];
+            L.t[s] = (uint32_t)sv[(8 + s) * 32 + lane];
+        }
+        L.tprev = (uint32_t)sv[16 * 32 + lane];
+        L.f7 = (uint32_t)sv[17 * 32 + lane];
+        L.selhi = (uint32_t)sv[18 * 32 + lane];
+        L.B = sv[19 * 32 + lane];
+        const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
+        L.FL = (uint32_t)fl * 0x10001u;
+    }
+};
+
+template <int NW, int W>
+__global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
+{
+    using F = Fill16<NW, W>;
+    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    int2 *rings = reinterpret_cast<int2 *>(smem_raw);
+    uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * RING);
+    int *saves = reinterpret_cast<int *>(selr + SRING);
+    __shared__ int s_band, s_abort;
+
+    const int warp = threadIdx.x >> 5, lane = lane_id();
+    const uint32_t selr_base = (uint32_t)__cvta_generic_to_shared(selr);
+    const StripeArgs &S = a.st[blockIdx.x % a.nstripes];
+    const int NT = S.NT;
+    const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr;
+    int bs = 0, bi = 0, bj = 0;
+    long long nrep = 0;
+    if (*a.err) return;
+    StepInfo X;
+    X.w = S.w;
+    X.col0 = S.col0;
+    X.sp_ld = S.sp_ld;
+    X.sp_stride = S.sp_stride;
+    X.jcap = S.w - 1;
+    X.rbrow = nullptr;
+    // steps at which a lane meets the capture column: low half at k = jcap + 2 lane, high at +1
+    const int cap_t0 = X.jcap / STEPS, cap_t1 = (X.jcap + 63) / STEPS;
+
+    for (;;) {
+        if (threadIdx.x == 0) {
+            int b = atomicAdd(S.ticket, 1);
+            if (ld_relaxed(a.err)) b = a.nb;
+            s_band = b;
+            s_abort = 0;
+        }
+        __syncthreads();
+        const int b = s_band;
+        if (b >= a.nb) break;
+
+        typename F::Lane L;
+        const int row0 = b * BH + (warp * 32 + lane) * 16;
+        int *sp_ptr = nullptr;
+        bool warp_sp = false;
+        X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
+        auto init_state = [&](bool from_left) {
+            // state at the column left of the stripe: the column-0 boundary or the left border
+            int tv[16], ev[16];
+            if (from_left) {
+#pragma unroll
+                for (int r = 0; r < 16; r++) {
+                    const int2 v = ld_sys_int2(S.lb + row0 + 1 + r);
+                    tv[r] = v.x;
+                    ev[r] = v.y;
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < 16; r++) { tv[r] = -a.gf; ev[r] = -a.gf; }  // E(i,0) := t(i,0), exact
+            }
+            int tp;
+            if (from_left && row0 > 0) tp = ld_sys_int2(S.lb + row0).x;
+            else tp = -a.gf;
+            L.B = __shfl_sync(0xffffffffu, tv[0], 0);
+#pragma unroll
+            for (int s = 0; s < 8; s++) {
+                L.e[s] = pk(F::tofr(L, ev[s]), F::tofr(L, ev[s + 8]));
+                L.t[s] = pk(F::tofr(L, tv[s]), F::tofr(L, tv[s + 8]));
+            }
+            L.tprev = pk(F::tofr(L, tp), F::tofr(L, tp));
+            L.f7 = L.t[7];
+            const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
+            L.FL = (uint32_t)fl * 0x10001u;
+        };
+        if (warp < NW) {
+            const uint32_t w = row0 < a.m ? a.A2[row0 >> 4] : 0u;
+#pragma unroll
+            for (int s = 0; s < 8; s++) {
+                L.P[s] = (row0 + s < a.m) ? a.prof[(w >> (2 * s)) & 3u] : PADPROF;
+                L.Q[s] = (row0 + s + 8 < a.m) ? a.prof[(w >> (2 * (s + 8))) & 3u] : PADPROF;
+            }
+            L.selhi = 0;
+            init_state(false);
+            if (a.k > 0) {
+                // special rows are strip-bottom rows (k a multiple of 16): row0 + 16
+                const int row = row0 + 16;
+                if (row <= a.m && row % a.k == 0) sp_ptr = S.sp + (long long)(row / a.k - 1) * S.sp_stride;
+            }
+            warp_sp = __any_sync(0xffffffffu, sp_ptr != nullptr);
+        }
+
+        auto io_load = [&](int c) {
+            const int need = min((c + 1) * W, NT * W - SKEW);
+            if (b > 0) {
+                if (lane == 0) {
+                    const unsigned long long t0 = gtimer();
+                    while (ld_acquire(S.progress + b - 1) < need) {
+                        if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
+                        __nanosleep(64);
+                    }
+                }
+                __syncwarp();
+            }
+#pragma unroll
+            for (int x = lane; x < W; x += 32) {
+                const int col = c * W + x;
+                rings[col & (RING - 1)] = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
+                uint32_t code = 0u;  // pad columns: code 0 (harmless, see header)
+                if (col < S.w) {
+                    const int gc = S.col0 + col;
+                    code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
+                }
+                selr[col & (SRING - 1)] = col_sel16(code);
+            }
+        };
+        auto io_drain = [&](int cd) {
+            const int2 *ringN = rings + NW * RING;
+#pragma unroll
+            for (int x = lane; x < W; x += 32) {
+                const int col = cd * W - SKEW + x;
+                if (col >= 0) __stcg(S.rowb + col, ringN[col & (RING - 1)]);
+            }
+            __threadfence();
+            __syncwarp();
+            if (lane == 0) st_release(S.progress + b, cd * W + W - SKEW);
+        };
+        auto wait_left = [&]() {
+            if (lane == 0) {
+                const int fi = b * NW + warp;
+                const unsigned long long t0 = gtimer();
+                while (ld_acquire_sys(S.lready + fi) != a.epoch || (fi > 0 && ld_acquire_sys(S.lready + fi - 1) != a.epoch)) {
+                    if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); break; }
+                    __nanosleep(64);
+                }
+            }
+            __syncwarp();
+        };
+
+        if (warp == NW) io_load(0);
+        __syncthreads();
+        const int S_END = NT + 2 * (NW - 1);
+        int *sv = saves + warp * F::NSAVE * 32;
+        for (int s = 0; s < S_END + 1; ++s) {
+            if (warp < NW) {
+                const int c = s - 2 * warp;
+                if (c >= 0 && c < NT) {
+                    const uint32_t rin = pin((uint32_t)__cvta_generic_to_shared(rings + warp * RING));
+                    const uint32_t rout = pin((uint32_t)__cvta_generic_to_shared(rings + (warp + 1) * RING));
+                    const uint32_t selr_s = pin(selr_base);
+                    if (c == 0 && has_left) {
+                        wait_left();
+                        init_state(true);
+                    }
+                    if (c > 0) F::rebase(a, L);
+                    const int thr = max(max(bs, ld_relaxed(a.gbest)), 1);
+                    F::save(L, sv, lane);
+                    uint32_t tm;
+                    const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
+                    if (cap) {
+                        tm = warp_sp ? F::template tile<true, false, true, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr)
+                                     : F::template tile<true, false, false, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr);
+                        if (c == cap_t1) {
+                            __threadfence_system();
+                            __syncwarp();
+                            if (lane == 0) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
+                        }
+                    } else if (c == 0) {
+                        tm = warp_sp ? F::template tile<true, false, true, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr)
+                                     : F::template tile<true, false, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr);
+                    } else if (warp_sp) {
+                        tm = F::template tile<false, false, true, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr);
+                    } else {
+                        tm = F::template tile<false, false, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
+                    }
+                    const int tmax = F::toabs(L, max(lo16(tm), hi16(tm)));
+                    if (__any_sync(0xffffffffu, tmax >= thr)) {
+                        F::restore(L, sv, lane);
+                        const int obs = bs;
+                        F::template tile<true, true, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
+                        if (lane == 0) nrep++;
+                        if (bs > obs) atomicMax(a.gbest, bs);
+                    }
+                }
+            } else {
+                if (s + 1 < NT) io_load(s + 1);
+                const int cd = s - 1 - 2 * (NW - 1);
+                if (cd >= 0) io_drain(cd);
+            }
+            __syncthreads();
+            if (s_abort) break;
+        }
+        if (warp == NW && lane == 0 && !s_abort) st_release(S.progress + b, INT_MAX);
+        if (a.k > 0) {
+            __threadfence();
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                const long long lo = (long long)b * BH + 1, hi = min((long long)(b + 1) * BH, (long long)a.m);
+                long long q = (lo + a.k - 1) / a.k;
+                if (q * a.k <= hi) {
+                    __threadfence_system();
+                    for (; q * a.k <= hi; q++) st_release_sys(S.row_done + (q - 1), 1u);
+                }
+            }
+        }
+    }
+
+    if (lane == 0 && nrep) atomicAdd(a.replays, (unsigned long long)nrep);
+    __shared__ int4 red[NW + 1];
+    for (int o = 16; o > 0; o >>= 1) {
+        const int s2 = __shfl_down_sync(0xffffffffu, bs, o);
+        const int i2 = __shfl_down_sync(0xffffffffu, bi, o);
+        const int j2 = __shfl_down_sync(0xffffffffu, bj, o);
+        if (better(s2, i2, j2, bs, bi, bj)) { bs = s2; bi = i2; bj = j2; }
+    }
+    if (lane == 0) red[warp] = make_int4(bs, bi, bj, 0);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int4 r = make_int4(0, 0, 0, 0);
+        for (int w = 0; w < NW; w++)
+            if (red[w].x > 0 && better(red[w].x, red[w].y, red[w].z, r.x, r.y, r.z)) r = red[w];
+        a.slots[blockIdx.x] = r;
+    }
+}
+
+}  // namespace swb

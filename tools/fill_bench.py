@@ -36,7 +36,7 @@ def main():
     args = [a for a in sys.argv[1:] if not a.startswith("--")]
     opts = dict(a[2:].split("=") for a in sys.argv[1:] if a.startswith("--"))
     wl = args[0] if args else "C2"
-    variants = [int(v) for v in args[1:]] or [int(os.environ.get("SWB_VARIANT", "1"))]
+    variants = [int(v) for v in args[1:]] or [-1]  # -1: the library's automatic choice
     reps = int(opts.get("reps", 2))
     cfg = synth.CONFIGS[wl]
     k = int(opts.get("k", cfg.k))
@@ -46,7 +46,10 @@ def main():
     from paper_conf_ipps_sandesm11_b200 import Context
 
     for v in variants:
-        os.environ["SWB_VARIANT"] = str(v)
+        if v >= 0:
+            os.environ["SWB_VARIANT"] = str(v)
+        else:
+            os.environ.pop("SWB_VARIANT", None)
         ctx = Context(0)
         best = None
         for _ in range(reps):
