@@ -36,9 +36,12 @@ METRIC = "GCUPS at 1/2/4/8 B200 (33×47 MBP synthetic) + % of INT-pipe roofline"
 SCORING = (1, -3, 3, 2)  # match +1, mismatch -3, first gap -5 (G_open 3), extension -2
 # Paper Table IV 543K x 536K Stage 1 with flush (SRA 50M): 21,419 MCUPS on a GTX 285.
 PAPER_GCUPS = {"C2": 21.419}
-# Roofline: best instruction mix for one int32 cell update:
-# 3.5 half-rate (64 lanes/clk/SM) + 4 full-rate ops -> 17.07 cells/clk/SM.
-ROOF_CELLS_PER_CLK_SM = 17.07
+# Roofline: ALU-pipe cycles of each kernel's cell-update
+# mix with the measured rates (profiles/r01_microbench_int.txt; half-rate ops
+# occupy the ALU pipe 2 cycles per warp instruction, full-rate ops 1):
+#   int32 kernel: 8 ALU cycles per 32 cells  -> 16.0 cells/clk/SM
+#   packed 16x2 : 9 ALU cycles per 64 cells  -> 28.44 cells/clk/SM
+ROOF_CELLS_PER_CLK_SM = {"int32": 16.0, "int16x2": 28.44}
 
 
 def parse():
@@ -343,7 +346,9 @@ def main():
     except Exception:
         pass
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
-    peak = nsm * ROOF_CELLS_PER_CLK_SM * sm_max * 1e6 / 1e9
+    kdtype = "int16x2" if s1["alpha"] < 0 else "int32"  # stats.alpha < 0: the packed kernel ran
+    roof = ROOF_CELLS_PER_CLK_SM[kdtype]
+    peak = nsm * roof * sm_max * 1e6 / 1e9
     traffic = None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
@@ -353,9 +358,9 @@ def main():
         pass
     roofline = {"bound": "alu", "achieved": round(achieved, 2), "peak": round(peak, 1), "unit": "GCUPS",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
-                "peak_basis": f"{nsm} SM x {ROOF_CELLS_PER_CLK_SM} cells/clk/SM x {sm_max:.0f} MHz (measured pipe rates, DESIGN.md 5)",
+                "peak_basis": f"{kdtype} kernel: {nsm} SM x {roof} cells/clk/SM x {sm_max:.0f} MHz (measured pipe rates, DESIGN.md 5)",
                 "fill_ms": round(fill_avg, 3), "per": "GPU",
-                "peak_at_measured_clock": round(nsm * ROOF_CELLS_PER_CLK_SM * (clocks.get('sm_mhz') or sm_max) * 1e-3, 1)}
+                "peak_at_measured_clock": round(nsm * roof * (clocks.get('sm_mhz') or sm_max) * 1e-3, 1)}
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
@@ -367,13 +372,14 @@ def main():
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
         "scaling": "strong" if world > 1 else "weak",
         "vs_baseline": (round(value / PAPER_GCUPS[cfg.name], 2) if cfg.name in PAPER_GCUPS else None),
-        "dtype": "int32", "data": "synthetic",
+        "dtype": "int16x2" if s1["alpha"] < 0 else "int32", "data": "synthetic",
         "config": {"workload": cfg.name, "m": m, "n": n, "k": k, "scoring": list(SCORING),
                    "step": "encode + Stage-1 fill + special rows to host sink + reverse goal pass",
                    "l2": "flushed between timed steps (256 MiB write)",
                    "parallelism": "single" if world == 1 else f"column stripes x{world} (NVLink border hand-off)"
                    + (" [same device, functional check]" if same_dev else ""),
-                   "kernel": {"alpha": s1["alpha"], "warps": s1["warps"], "width": s1["width"], "grid": s1["grid"]},
+                   "kernel": {"alpha": abs(s1["alpha"]), "packed16x2": s1["alpha"] < 0, "warps": s1["warps"],
+                              "width": s1["width"], "grid": s1["grid"]},
                    "baseline_note": "vs_baseline = value / paper Table IV 543Kx536K flush (21.419 GCUPS, GTX 285, real DNA)"},
         "result": {"best": list(best), "start": list(start) if start else None, "special_rows_per_step": rows_per_step},
         "roofline": roofline,

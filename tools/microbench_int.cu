@@ -37,6 +37,9 @@ __global__ void kern(int *out, int a0, int b0, long long *cycles)
             if (KIND == 7) x[k] = __viaddmax_s16x2(x[k], b, c);          // VIADDMNMX.S16x2
             if (KIND == 8) x[k] = __vimax3_s16x2_relu(x[k], b, c);       // VIMNMX3.S16x2.RELU
             if (KIND == 9) { x[k] = max(x[k] + b, c); }                   // IADD+IMNMX (compiler's choice)
+            if (KIND == 11) x[k] = __vmaxu2(x[k], b);                      // VIMNMX.U16x2
+            if (KIND == 12) x[k] = __vimax3_u16x2(x[k], b, c);            // VIMNMX3.U16x2
+            if (KIND == 13) x[k] = __viaddmax_u16x2(x[k], b, c);          // VIADDMNMX.U16x2
         }
     }
     long long t1 = clock64();
@@ -98,6 +101,9 @@ int main()
         run<8>("VIMNMX3.S16x2.RELU", sms, thr, 1);
         run<9>("IADD+IMNMX", sms, thr, 1);
         run<10>("IMAD", sms, thr, 1);
+        run<11>("VIMNMX.U16x2", sms, thr, 1);
+        run<12>("VIMNMX3.U16x2", sms, thr, 1);
+        run<13>("VIADDMNMX.U16x2", sms, thr, 1);
     }
     return 0;
 }
