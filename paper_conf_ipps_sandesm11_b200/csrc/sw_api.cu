@@ -127,7 +127,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 3;
+static constexpr int NVARIANTS = 6;
 
 static const Variant &variant_for(int idx)
 {
@@ -135,6 +135,9 @@ static const Variant &variant_for(int idx)
         make_variant<16, 4, 64>(),
         make_variant<16, 8, 64>(),
         make_variant<8, 8, 64>(),
+        make_variant<16, 12, 64>(),
+        make_variant<16, 14, 64>(),
+        make_variant<16, 15, 64>(),
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -415,11 +418,18 @@ struct Job {
 };
 }  // namespace
 
-// Kernel choice per call: the packed 16x2 kernel with the
-// 4-warp geometry when it applies and the band pipeline runs for >= 2 waves
-// (steady state dominates); otherwise the int32 kernel with 8 warps (best when
-// all bands are in flight at once and the pipeline skew dominates, e.g. C2).
-// Deterministic in (m, n, k, scoring), so all ranks of a stripe group agree.
+// Kernel choice per call: a small cost model over candidate
+// (kernel, geometry) pairs.  A band takes a CTA one sweep; with P resident
+// CTAs the fill takes ceil(nb / P) sweeps of time ~ BH * P / rate, where
+// `rate` is the measured steady-state GCUPS of the candidate (R10Mx1M, one
+// B200, profiles/r01_variants.txt).  Deterministic in (m, n, k, scoring), so
+// all ranks of a stripe group agree.
+struct Candidate {
+    int variant;
+    bool packed;
+    double rate;
+};
+
 static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
 {
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
@@ -430,19 +440,35 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         *use16 = packed_ok && V.packed_fn;
         return V;
     }
-    const Variant &V0 = variant_for(0);
-    if (packed_ok && V0.packed_fn) {
+    static const Candidate cands[] = {
+        {DEFAULT_VARIANT, false, 2572.0},  // int32, 8 warps
+        {0, true, 2785.0},                 // packed, 4 warps, 3 CTAs/SM
+        {3, true, 2851.0},                 // packed, 12 warps
+        {5, true, 3178.0},                 // packed, 15 warps
+    };
+    double best_t = 1e300;
+    int best = 0;
+    for (int c = 0; c < (int)(sizeof(cands) / sizeof(cands[0])); c++) {
+        const Candidate &C = cands[c];
+        if (C.packed && !packed_ok) continue;
+        if (!C.packed && !J.local) { best = c; break; }  // reverse pass: int32 only
+        const Variant &V = variant_for(C.variant);
+        const void *fn = C.packed ? V.packed_fn : V.local_fn;
+        if (!fn) continue;
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, V0.packed_fn, V0.nw * 32 + 32, V0.smem16);
-        const long long bh = (long long)V0.alpha * 32 * V0.nw;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, V.nw * 32 + 32, C.packed ? V.smem16 : V.smem);
+        const long long P = (long long)std::max(1, per_sm) * ctx->num_sms;
+        const long long bh = (long long)V.alpha * 32 * V.nw;
         const long long nb = (J.m + bh - 1) / bh;
-        if (nb >= 2ll * std::max(1, per_sm) * ctx->num_sms) {
-            *use16 = true;
-            return V0;
+        // one sweep of one band takes bh * P / rate whether or not all P CTAs are busy
+        const double t = (double)((nb + P - 1) / P) * (double)bh * (double)P / C.rate;
+        if (t < best_t * 0.97) {  // prefer earlier (simpler) candidates on near-ties
+            best_t = t;
+            best = c;
         }
     }
-    *use16 = false;
-    return variant_for(DEFAULT_VARIANT);
+    *use16 = cands[best].packed;
+    return variant_for(cands[best].variant);
 }
 
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)

@@ -70,6 +70,15 @@ struct Fill16 {
         uint32_t FL;          // packed frame image of the local floor 0
     };
 
+    // Selector ring layout: even columns in the first half, odd in the second,
+    // so the 32 lanes of a step (columns k - 2 lane, all of one parity) read
+    // 32 consecutive words: no bank conflicts.
+    static __device__ __forceinline__ uint32_t sel_index(int col)
+    {
+        const uint32_t c = (uint32_t)col & (SRING - 1);
+        return (c >> 1) + (c & 1u) * (SRING / 2);
+    }
+
     static __device__ __forceinline__ int toabs(const Lane &L, int q) { return q - BIAS16 + L.B; }
     static __device__ __forceinline__ int tofr(const Lane &L, int x) { return x - L.B + BIAS16; }
 
@@ -97,7 +106,8 @@ struct Fill16 {
         uint32_t fu = __byte_perm(up_f, L.f7, 0x5432);
         uint32_t td = L.tprev;
         L.tprev = tu;
-        const uint32_t sw = lds_v2u(selr + (uint32_t)(jl & (SRING - 1)) * 4u).x;
+        uint32_t sw;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(sw) : "r"(selr + sel_index(jl) * 4u) : "memory");
         const uint32_t sel = (sw & 0xffu) | L.selhi;
         L.selhi = sw & 0xff00u;  // nibbles 2,3 (bytes 2,3 of the result) for the next column
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
@@ -354,7 +364,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_c
                     const int gc = S.col0 + col;
                     code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
                 }
-                selr[col & (SRING - 1)] = col_sel16(code);
+                selr[F::sel_index(col)] = col_sel16(code);
             }
         };
         auto io_drain = [&](int cd) {

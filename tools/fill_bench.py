@@ -38,9 +38,14 @@ def main():
     wl = args[0] if args else "C2"
     variants = [int(v) for v in args[1:]] or [-1]  # -1: the library's automatic choice
     reps = int(opts.get("reps", 2))
-    cfg = synth.CONFIGS[wl]
-    k = int(opts.get("k", cfg.k))
-    A, B = synth.make_pair(cfg)
+    if wl.startswith("R"):  # R<m>x<n>: random pair with one plant, e.g. R2000000x300000
+        mm, nn = (int(x) for x in wl[1:].split("x"))
+        k = int(opts.get("k", 0))
+        A, B = synth.random_pair(99, mm, nn, plant_len=min(mm, nn) // 4, s=0.02, g=0.002)
+    else:
+        cfg = synth.CONFIGS[wl]
+        k = int(opts.get("k", cfg.k))
+        A, B = synth.make_pair(cfg)
     dA = torch.from_numpy(A).cuda()
     dB = torch.from_numpy(B).cuda()
     from paper_conf_ipps_sandesm11_b200 import Context
