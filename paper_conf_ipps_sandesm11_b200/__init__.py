@@ -39,6 +39,7 @@ EXPORTED = [
     "sw_reverse_goal_dev",
     "sw_row_granularity",
     "sw_band_height",
+    "sw_set_kernel",
     "sw_set_virtual_stripes",
     "sw_stripe_export",
     "sw_stripe_connect",
@@ -118,6 +119,8 @@ def load_library(path: str = LIB_PATH):
     lib.sw_row_granularity.restype = i64
     lib.sw_band_height.argtypes = [vp]
     lib.sw_band_height.restype = i64
+    lib.sw_set_kernel.argtypes = [vp, ctypes.c_int, ctypes.c_int]
+    lib.sw_set_kernel.restype = ctypes.c_int
     lib.sw_set_virtual_stripes.argtypes = [vp, ctypes.c_int]
     lib.sw_set_virtual_stripes.restype = ctypes.c_int
     lib.sw_stripe_export.argtypes = [vp, i64, vp]
@@ -249,6 +252,10 @@ class Context:
 
     def band_height(self) -> int:
         return int(self._lib.sw_band_height(self._h))
+
+    def set_kernel(self, variant: int = -1, packed: bool = True):
+        """variant -1: automatic; 0..5: fixed geometry; packed: allow the 16x2 kernel."""
+        self._check(self._lib.sw_set_kernel(self._h, variant, int(bool(packed))), "sw_set_kernel")
 
     def set_virtual_stripes(self, nstripes: int):
         """Split the next Stage-1 calls into `nstripes` column stripes on this GPU

@@ -357,6 +357,14 @@ extern "C" int64_t sw_special_row_interval_for_budget(int64_t m, int64_t n, int6
     return (int64_t)(bh * (int64_t)q);
 }
 
+extern "C" int sw_set_kernel(sw_ctx *ctx, int variant, int packed)
+{
+    if (!ctx || variant < -1 || variant >= NVARIANTS || packed < 0 || packed > 1) return SW_EINVAL;
+    ctx->variant_override = variant;
+    ctx->packed = packed;
+    return SW_OK;
+}
+
 extern "C" int sw_set_virtual_stripes(sw_ctx *ctx, int nstripes)
 {
     if (!ctx || nstripes < 1 || nstripes > MAX_STRIPES) return SW_EINVAL;

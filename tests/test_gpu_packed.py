@@ -1,0 +1,90 @@
+"""The packed 16x2 Stage-1 kernel (N4) forced on, bit-exact against the oracle:
+every geometry that has a packed instantiation, special rows (k % 16 == 0),
+ragged shapes, several scorings within its value window, virtual stripes,
+and the int32 kernel on the same inputs."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+PAPER = (1, -3, 3, 2)
+PACKED_VARIANTS = [0, 3, 5]  # (16, 4), (16, 12), (16, 15) warps
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    from paper_conf_ipps_sandesm11_b200 import Context, build
+
+    build.build()
+    c = Context(0)
+    yield c
+    c.set_kernel(-1, True)
+    c.set_virtual_stripes(1)
+    c.close()
+
+
+def _s(x):
+    return x.tobytes().decode() if isinstance(x, np.ndarray) else x
+
+
+def check(ctx, A, B, scoring, k, variant, stripes=1, expect_packed=True):
+    ctx.set_kernel(variant, True)
+    ctx.set_virtual_stripes(stripes)
+    try:
+        got, rows = ctx.align_stage1(A, B, *scoring, k=k, keep_rows=True)
+        st = ctx.stats()
+    finally:
+        ctx.set_kernel(-1, True)
+        ctx.set_virtual_stripes(1)
+    assert (st["alpha"] < 0) == expect_packed, st
+    want, orows = oracle.stage1(_s(A), _s(B), *scoring, k=k)
+    assert got.astuple() == want, (len(A), len(B), scoring, k, variant, stripes)
+    assert [r for r, _, _ in rows] == [r for r, _, _ in orows]
+    for (r, h, f), (_, oh, of) in zip(rows, orows):
+        assert np.array_equal(h, oh), f"H row {r}"
+        assert np.array_equal(f, of), f"F row {r}"
+
+
+@pytest.mark.parametrize("variant", PACKED_VARIANTS)
+@pytest.mark.parametrize("m,n", [(1, 1), (17, 1), (16, 300), (1000, 999), (3000, 64), (5000, 2049)])
+def test_packed_shapes(ctx, variant, m, n):
+    A, B = synth.random_pair(m + 3 * n + variant, m, n, plant_len=min(m, n) // 2, s=0.05, g=0.01)
+    check(ctx, A, B, PAPER, 16, variant)
+
+
+@pytest.mark.parametrize("variant", PACKED_VARIANTS)
+def test_packed_scorings(ctx, variant):
+    A, B = synth.random_pair(5 + variant, 2500, 1700, plant_len=1500, s=0.06, g=0.01)
+    for scoring in (PAPER, (2, -1, 4, 1), (1, -1, 0, 2), (5, -4, 10, 1), (3, -2, 0, 1)):
+        check(ctx, A, B, scoring, 32, variant)
+    check(ctx, A, B, PAPER, 0, variant)
+
+
+def test_packed_falls_back_when_not_applicable(ctx):
+    A, B = synth.random_pair(8, 900, 700, plant_len=500)
+    check(ctx, A, B, PAPER, 7, 5, expect_packed=False)            # k not a multiple of 16
+    check(ctx, A, B, (100, -20, 20, 5), 16, 5, expect_packed=False)  # value window too wide
+
+
+def test_packed_ties_and_long_alignment(ctx):
+    X = synth.random_pair(3, 400, 1)[0]
+    XXX = np.concatenate([X, X, X])
+    check(ctx, XXX, X, PAPER, 16, 5)
+    check(ctx, X, XXX, PAPER, 16, 0)
+    A, B = synth.random_pair(21, 9000, 9000, plant_len=9000, s=0.01, g=0.002)  # whole-length: large scores
+    check(ctx, A, B, PAPER, 1024, 3)
+
+
+@pytest.mark.parametrize("stripes", [2, 3, 8])
+def test_packed_virtual_stripes(ctx, stripes):
+    A, B = synth.random_pair(60 + stripes, 6000, 1500, plant_len=1200, s=0.04, g=0.01)
+    check(ctx, A, B, PAPER, 16, 0, stripes=stripes)
+    check(ctx, A, B, PAPER, 0, 5, stripes=stripes)
+
+
+def test_packed_config_c1(ctx):
+    cfg = synth.CONFIGS["C1"]
+    A, B = synth.make_pair(cfg)
+    check(ctx, A, B, PAPER, cfg.k, 5)
