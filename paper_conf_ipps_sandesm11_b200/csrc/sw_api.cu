@@ -168,6 +168,8 @@ struct sw_ctx {
     int num_sms = 0;
     cudaStream_t stream = nullptr, side = nullptr;
     cudaEvent_t ev[6] = {};
+    cudaEvent_t ev_row[8] = {};  // staging-row copies (special rows)
+    int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
     DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
     HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
@@ -284,6 +286,8 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
         if ((e = cudaStreamCreateWithFlags(&ctx->side, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
         for (auto &ev : ctx->ev)
             if ((e = cudaEventCreate(&ev)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
+        for (auto &ev : ctx->ev_row)
+            if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
         if (rc) break;
         if ((e = cudaHostAlloc(&ctx->res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
         for (int i = 0; i < NVARIANTS; i++) {
@@ -322,6 +326,8 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     if (ctx->stage.p) cudaFreeHost(ctx->stage.p);
     if (ctx->res_h) cudaFreeHost(ctx->res_h);
     for (auto &ev : ctx->ev)
+        if (ev) cudaEventDestroy(ev);
+    for (auto &ev : ctx->ev_row)
         if (ev) cudaEventDestroy(ev);
     if (ctx->stream) cudaStreamDestroy(ctx->stream);
     if (ctx->side) cudaStreamDestroy(ctx->side);
@@ -568,7 +574,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             if ((rc = grow_host(ctx, ctx->flags[s], nsp * sizeof(unsigned int), true))) return rc;
             memset(ctx->flags[s].p, 0, nsp * sizeof(unsigned int));
         }
-        if ((rc = grow_host(ctx, ctx->stage, (size_t)2 * (n + 32) * sizeof(int32_t), false))) return rc;
+        // staging ring: up to 8 rows, at most ~1 GiB of pinned memory
+        const size_t row_bytes = (size_t)2 * (n + 64) * sizeof(int32_t);
+        ctx->nstage = (int)std::max<size_t>(2, std::min<size_t>(8, ((size_t)1 << 30) / row_bytes));
+        if ((rc = grow_host(ctx, ctx->stage, row_bytes * ctx->nstage, false))) return rc;
     }
 
     // With a caller stream, every kernel of the call is launched on it (so the
@@ -678,43 +687,71 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     CK(cudaMemcpyAsync(ctx->res_h + 2, d_replays, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     CK(cudaEventRecord(ctx->ev[3], st));
 
-    // stream special rows to the sink in ascending order while the fill runs;
-    // a row is complete when every stripe of this launch has published it
+    // Stream special rows to the sink in ascending order while the fill runs.
+    // A row is complete when every stripe of this launch has published it.
+    // Up to NSTAGE pinned staging rows: copies are issued as soon as rows are
+    // ready (bands of a short matrix finish in a burst), sinks run in order.
     int sink_rc = 0;
     long long bytes = 0;
     const int64_t nrow_out = J.rank_mode ? wid[0] : n;
-    int32_t *stage = (int32_t *)ctx->stage.p;
-    const int64_t sld = nrow_out + 32;
-    for (long long q = 0; q < nsp; q++) {
-        for (int s = 0; s < NS; s++) {
-            volatile unsigned int *f = (volatile unsigned int *)ctx->flags[s].p + q;
-            while (*f == 0) {
-                const cudaError_t qe = cudaEventQuery(ctx->ev[2]);
-                if (qe == cudaSuccess) {
-                    if (*f == 0) {
-                        CK(cudaStreamSynchronize(st));
-                        if (ctx->res_h[1].x == 1) return SW_EALPHABET;
-                        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", q,
-                                 ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
-                        return SW_ECUDA;
-                    }
-                    break;
-                } else if (qe != cudaErrorNotReady) {
-                    return cuda_fail(ctx, qe, "fill kernel");
-                }
-                std::this_thread::yield();
-            }
-        }
-        if (sink_rc) continue;  // aborted: drain flags, skip copies
+    const int64_t sld = (NS == 1) ? ld[0] : nrow_out + 32;  // H at [0, sld), F at [sld, 2 sld)
+    const int nstage = nsp > 0 ? ctx->nstage : 0;
+    auto row_ready = [&](long long q) -> bool {
+        for (int s = 0; s < NS; s++)
+            if (((volatile unsigned int *)ctx->flags[s].p)[q] == 0) return false;
+        return true;
+    };
+    auto issue_copy = [&](long long q) -> int {
+        int32_t *dst = (int32_t *)ctx->stage.p + (q % nstage) * 2 * sld;
         for (int s = 0; s < NS; s++) {
             const int32_t *src = (const int32_t *)ctx->sp[s].p + q * stride[s];
-            const int64_t off = J.rank_mode ? 0 : col0[s];
-            CK(cudaMemcpyAsync(stage + off, src, (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
-            CK(cudaMemcpyAsync(stage + sld + off, src + ld[s], (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+            if (NS == 1) {
+                CK(cudaMemcpyAsync(dst, src, (size_t)stride[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+            } else {
+                const int64_t off = J.rank_mode ? 0 : col0[s];
+                CK(cudaMemcpyAsync(dst + off, src, (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+                CK(cudaMemcpyAsync(dst + sld + off, src + ld[s], (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+            }
         }
-        CK(cudaStreamSynchronize(ctx->side));
-        bytes += 8ll * nrow_out;
-        if (J.sink && J.sink(J.user, (q + 1) * J.k, stage, stage + sld, nrow_out)) sink_rc = SW_EABORTED;
+        CK(cudaEventRecord(ctx->ev_row[q % nstage], ctx->side));
+        return SW_OK;
+    };
+    long long issued = 0, done = 0;
+    while (done < nsp) {
+        bool progress = false;
+        while (issued < nsp && issued - done < nstage && row_ready(issued)) {
+            if (!sink_rc && (rc = issue_copy(issued))) return rc;
+            issued++;
+            progress = true;
+        }
+        if (issued > done) {
+            const cudaError_t qe = sink_rc ? cudaSuccess : cudaEventQuery(ctx->ev_row[done % nstage]);
+            if (qe == cudaSuccess) {
+                if (!sink_rc) {
+                    bytes += 8ll * nrow_out;
+                    int32_t *row = (int32_t *)ctx->stage.p + (done % nstage) * 2 * sld;
+                    if (J.sink && J.sink(J.user, (done + 1) * J.k, row, row + sld, nrow_out)) sink_rc = SW_EABORTED;
+                }
+                done++;
+                progress = true;
+            } else if (qe != cudaErrorNotReady) {
+                return cuda_fail(ctx, qe, "special-row copy");
+            }
+        }
+        if (!progress) {
+            // nothing ready: make sure the fill is still running
+            const cudaError_t fe = cudaEventQuery(ctx->ev[2]);
+            if (fe == cudaSuccess && issued < nsp && !row_ready(issued)) {
+                CK(cudaStreamSynchronize(st));
+                if (ctx->res_h[1].x == 1) return SW_EALPHABET;
+                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", issued,
+                         ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
+                return SW_ECUDA;
+            } else if (fe != cudaSuccess && fe != cudaErrorNotReady) {
+                return cuda_fail(ctx, fe, "fill kernel");
+            }
+            std::this_thread::yield();
+        }
     }
     CK(cudaStreamSynchronize(st));
     if (ctx->res_h[1].x == 1) return SW_EALPHABET;

@@ -464,10 +464,12 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             L.tprev = LOCAL ? -a.gf : (row0 == 0 ? -a.gf : -(a.go + row0 * a.ge) - a.gf);
             L.out_t0 = L.out_f0 = L.out_t1 = L.out_f1 = 0;
             if (LOCAL && a.k > 0) {
-                // special rows among DP rows row0+1 .. row0+ALPHA (<= m)
+                // special rows among DP rows row0+1 .. row0+ALPHA (<= m); the band's
+                // bottom row is written by the I/O warp from its coalesced drain
+                const int bottom = (b + 1) * BH;
                 for (int r = 0; r < ALPHA; r++) {
                     const int row = row0 + r + 1;
-                    if (row <= a.m && row % a.k == 0) smask |= 1u << r;
+                    if (row <= a.m && row % a.k == 0 && row != bottom) smask |= 1u << r;
                 }
                 if (smask) {
                     const int first = __ffs(smask) - 1;
@@ -505,12 +507,25 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                 selr[col & (SRING - 1)] = col_sel(code);
             }
         };
+        // special row that is this band's bottom row: written here, coalesced
+        int *io_sp = nullptr;
+        if (LOCAL && a.k > 0) {
+            const int bottom = (b + 1) * BH;
+            if (bottom <= a.m && bottom % a.k == 0) io_sp = S.sp + (long long)(bottom / a.k - 1) * S.sp_stride;
+        }
         auto io_drain = [&](int cd) {
             const int2 *ringN = rings + NW * RING;
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = cd * W - SKEW + x;
-                if (col >= 0) __stcg(S.rowb + col, ringN[col & (RING - 1)]);
+                if (col >= 0) {
+                    const int2 v = ringN[col & (RING - 1)];
+                    __stcg(S.rowb + col, v);
+                    if (io_sp != nullptr && col < S.w) {
+                        __stcg(io_sp + col, v.x + a.gf);  // H = t + G_first
+                        __stcg(io_sp + S.sp_ld + col, v.y);
+                    }
+                }
             }
             __threadfence();
             __syncwarp();

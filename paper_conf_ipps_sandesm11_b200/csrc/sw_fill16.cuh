@@ -338,7 +338,8 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_c
             if (a.k > 0) {
                 // special rows are strip-bottom rows (k a multiple of 16): row0 + 16
                 const int row = row0 + 16;
-                if (row <= a.m && row % a.k == 0) sp_ptr = S.sp + (long long)(row / a.k - 1) * S.sp_stride;
+                if (row <= a.m && row % a.k == 0 && row != (b + 1) * BH)  // band bottom: the I/O warp's drain
+                    sp_ptr = S.sp + (long long)(row / a.k - 1) * S.sp_stride;
             }
             warp_sp = __any_sync(0xffffffffu, sp_ptr != nullptr);
         }
@@ -367,12 +368,24 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_c
                 selr[F::sel_index(col)] = col_sel16(code);
             }
         };
+        int *io_sp = nullptr;
+        if (a.k > 0) {
+            const int bottom = (b + 1) * BH;
+            if (bottom <= a.m && bottom % a.k == 0) io_sp = S.sp + (long long)(bottom / a.k - 1) * S.sp_stride;
+        }
         auto io_drain = [&](int cd) {
             const int2 *ringN = rings + NW * RING;
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = cd * W - SKEW + x;
-                if (col >= 0) __stcg(S.rowb + col, ringN[col & (RING - 1)]);
+                if (col >= 0) {
+                    const int2 v = ringN[col & (RING - 1)];
+                    __stcg(S.rowb + col, v);
+                    if (io_sp != nullptr && col < S.w) {
+                        __stcg(io_sp + col, v.x + a.gf);  // H = t + G_first
+                        __stcg(io_sp + S.sp_ld + col, v.y);
+                    }
+                }
             }
             __threadfence();
             __syncwarp();
