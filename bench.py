@@ -216,7 +216,10 @@ def main():
     m, n = len(A), len(B)
     dA = torch.from_numpy(A).to(dev)
     dB = torch.from_numpy(B).to(dev)
-    stream = torch.cuda.current_stream(dev)
+    # a dedicated stream: the library launches every kernel of the step on it, so
+    # the CUDA events recorded on it bracket exactly the step's device work
+    stream = torch.cuda.Stream(dev)
+    torch.cuda.set_stream(stream)
     sptr = stream.cuda_stream
     ctx = Context(dev_index)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2

@@ -67,6 +67,7 @@ struct Fill16 {
         uint32_t f7;          // packed F of slot 7 after the last step (row 15 in the high half)
         uint32_t selhi;       // high-half selector part of the previous column
         int B;                // warp-uniform frame base
+        int adj;              // BIAS16 - B: int32 value -> frame
         uint32_t FL;          // packed frame image of the local floor 0
     };
 
@@ -91,12 +92,21 @@ struct Fill16 {
         uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[7], 1);
         uint32_t up_f = __shfl_up_sync(0xffffffffu, L.f7, 1);
         const int jl = k - 2 * lane;
-        if (lane == 0) {
-            int2 v;
-            asm volatile("ld.shared.v2.s32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(ring_in + (uint32_t)(jl & (RING - 1)) * 8u) : "memory");
-            // F_in only enters as max(F_in - G_ext, t_in): clamping it to >= t_in is exact
-            up_t = (uint32_t)tofr(L, v.x) << 16;
-            up_f = (uint32_t)tofr(L, max(v.y, v.x)) << 16;
+        {
+            // lane 0: the warp above's bottom row (int32) from the ring, into this
+            // warp's frame; F_in only enters as max(F_in - G_ext, t_in), so
+            // clamping it to >= t_in is exact.  Predicated, not branched.
+            int vx, vy;
+            asm volatile("{\n\t.reg .pred p;\n\t"
+                         "setp.eq.s32 p, %2, 0;\n\t"
+                         "@p ld.shared.v2.s32 {%0, %1}, [%3];\n\t}"
+                         : "=r"(vx), "=r"(vy)
+                         : "r"(lane), "r"(ring_in + (uint32_t)(jl & (RING - 1)) * 8u)
+                         : "memory");
+            if (lane == 0) {
+                up_t = (uint32_t)(vx + L.adj) << 16;
+                up_f = (uint32_t)(max(vy, vx) + L.adj) << 16;
+            }
         }
         Lane S;
         if (GUARD) S = L;
@@ -221,6 +231,7 @@ struct Fill16 {
         L.tprev = (uint32_t)imad((int)L.tprev, a.one, d2);
         L.f7 = (uint32_t)imad((int)L.f7, a.one, d2);
         L.B += d;
+        L.adj = BIAS16 - L.B;
         const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
         L.FL = (uint32_t)fl * 0x10001u;
     }
@@ -248,6 +259,7 @@ struct Fill16 {
         L.f7 = (uint32_t)sv[17 * 32 + lane];
         L.selhi = (uint32_t)sv[18 * 32 + lane];
         L.B = sv[19 * 32 + lane];
+        L.adj = BIAS16 - L.B;
         const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
         L.FL = (uint32_t)fl * 0x10001u;
     }
@@ -316,6 +328,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_c
             if (from_left && row0 > 0) tp = ld_sys_int2(S.lb + row0).x;
             else tp = -a.gf;
             L.B = __shfl_sync(0xffffffffu, tv[0], 0);
+            L.adj = BIAS16 - L.B;
 #pragma unroll
             for (int s = 0; s < 8; s++) {
                 L.e[s] = pk(F::tofr(L, ev[s]), F::tofr(L, ev[s + 8]));
