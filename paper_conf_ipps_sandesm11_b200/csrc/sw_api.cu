@@ -105,6 +105,7 @@ struct Variant {
     size_t smem;
     const void *packed_fn;  // packed 16x2 Stage-1 kernel with the same band geometry (alpha 16 only)
     size_t smem16;
+    int io_warps;           // 1, or 0 for the cooperative-I/O packed kernel (block = (nw + io) warps)
 };
 
 template <int ALPHA, int NW, int W>
@@ -119,15 +120,21 @@ static Variant make_variant()
     v.smem = Fill<ALPHA, NW, W, true>::smem_bytes();
     v.packed_fn = nullptr;
     v.smem16 = 0;
+    v.io_warps = 1;
     if constexpr (ALPHA == 16) {
-        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W>;
+        if constexpr (NW == 16) {
+            v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, true>;
+            v.io_warps = 0;
+        } else {
+            v.packed_fn = (const void *)&sw_fill16_kernel<NW, W>;
+        }
         v.smem16 = Fill16<NW, W>::smem_bytes();
     }
     return v;
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 6;
+static constexpr int NVARIANTS = 7;
 
 static const Variant &variant_for(int idx)
 {
@@ -138,6 +145,7 @@ static const Variant &variant_for(int idx)
         make_variant<16, 12, 64>(),
         make_variant<16, 14, 64>(),
         make_variant<16, 15, 64>(),
+        make_variant<16, 16, 64>(),
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -458,7 +466,8 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         {DEFAULT_VARIANT, false, 2572.0},  // int32, 8 warps
         {0, true, 2785.0},                 // packed, 4 warps, 3 CTAs/SM
         {3, true, 2851.0},                 // packed, 12 warps
-        {5, true, 3178.0},                 // packed, 15 warps
+        {5, true, 3243.0},                 // packed, 15 warps + I/O warp
+        {6, true, 3470.0},                 // packed, 16 warps, cooperative I/O
     };
     double best_t = 1e300;
     int best = 0;
@@ -470,7 +479,8 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         const void *fn = C.packed ? V.packed_fn : V.local_fn;
         if (!fn) continue;
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, V.nw * 32 + 32, C.packed ? V.smem16 : V.smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, V.nw * 32 + (C.packed ? V.io_warps : 1) * 32,
+                                                      C.packed ? V.smem16 : V.smem);
         const long long P = (long long)std::max(1, per_sm) * ctx->num_sms;
         const long long bh = (long long)V.alpha * 32 * V.nw;
         const long long nb = (J.m + bh - 1) / bh;
@@ -539,8 +549,9 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     }
     const void *fill_fn = use16 ? V.packed_fn : (J.local ? V.local_fn : V.global_fn);
     const size_t fill_smem = use16 ? V.smem16 : V.smem;
+    const int block = V.nw * 32 + (use16 ? V.io_warps : 1) * 32;
     int blocks_per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, fill_fn, V.nw * 32 + 32, fill_smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, fill_fn, block, fill_smem);
     if (blocks_per_sm < 1) blocks_per_sm = 1;
     // every CTA of every stripe must be co-resident (stripes wait on each other)
     int per_stripe = std::max(1, std::min(nb, blocks_per_sm * ctx->num_sms / NS));
@@ -677,7 +688,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     }
     {
         void *args[] = {&a};
-        CK(cudaLaunchKernel(fill_fn, dim3(grid), dim3(V.nw * 32 + 32), args, fill_smem, st));
+        CK(cudaLaunchKernel(fill_fn, dim3(grid), dim3(block), args, fill_smem, st));
     }
     CK(cudaEventRecord(ctx->ev[2], st));
     sw_reduce_kernel<<<1, 256, 0, st>>>((const int4 *)ctx->slots.p, grid, J.local ? 1 : 0, d_hit_key, J.goal, d_res);

@@ -265,8 +265,12 @@ struct Fill16 {
     }
 };
 
-template <int NW, int W>
-__global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
+// COOP = false: NW compute warps + one I/O warp.  COOP = true: NW compute
+// warps that also share the I/O (each loads and drains W / NW columns per
+// tile), so all four SMSPs carry the same number of compute warps (16 warps:
+// 4 each) -- the lockstep interval otherwise waits for the busier SMSPs.
+template <int NW, int W, bool COOP = false>
+__global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
 {
     using F = Fill16<NW, W>;
     constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
@@ -416,11 +420,70 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_c
             __syncwarp();
         };
 
-        if (warp == NW) io_load(0);
+        // cooperative I/O: this warp's share of each tile's columns
+        constexpr int CPW = COOP ? W / NW : W;
+        static_assert(!COOP || (W % NW == 0 && W / NW <= 32), "W must split over the warps");
+        auto coop_wait = [&](int c) {
+            const int need = min((c + 1) * W, NT * W - SKEW);
+            if (b > 0 && lane == 0) {
+                const unsigned long long t0 = gtimer();
+                while (ld_acquire(S.progress + b - 1) < need) {
+                    if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
+                    __nanosleep(64);
+                }
+            }
+            __syncwarp();
+        };
+        auto coop_fetch = [&](int c, int2 &v, uint32_t &code) {  // issue the loads (results used after compute)
+            const int col = c * W + warp * CPW + lane;
+            v = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
+            code = 0u;
+            if (col < S.w) {
+                const int gc = S.col0 + col;
+                code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
+            }
+        };
+        auto coop_put = [&](int c, int2 v, uint32_t code) {
+            const int col = c * W + warp * CPW + lane;
+            rings[col & (RING - 1)] = v;
+            selr[F::sel_index(col)] = col_sel16(code);
+        };
+        auto coop_drain = [&](int cd) {
+            const int col = cd * W - SKEW + warp * CPW + lane;
+            if (col >= 0) {
+                const int2 v = rings[NW * RING + (col & (RING - 1))];
+                __stcg(S.rowb + col, v);
+                if (io_sp != nullptr && col < S.w) {
+                    __stcg(io_sp + col, v.x + a.gf);
+                    __stcg(io_sp + S.sp_ld + col, v.y);
+                }
+                __threadfence();
+            }
+        };
+
+        if constexpr (COOP) {
+            coop_wait(0);
+            if (lane < CPW) {
+                int2 v;
+                uint32_t code;
+                coop_fetch(0, v, code);
+                coop_put(0, v, code);
+            }
+        } else {
+            if (warp == NW) io_load(0);
+        }
         __syncthreads();
         const int S_END = NT + 2 * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s < S_END + 1; ++s) {
+            int2 fv = make_int2(0, 0);
+            uint32_t fcode = 0u;
+            if constexpr (COOP) {
+                if (s + 1 < NT) {
+                    coop_wait(s + 1);
+                    if (lane < CPW) coop_fetch(s + 1, fv, fcode);
+                }
+            }
             if (warp < NW) {
                 const int c = s - 2 * warp;
                 if (c >= 0 && c < NT) {
@@ -466,10 +529,21 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill16_kernel(const __grid_c
                 const int cd = s - 1 - 2 * (NW - 1);
                 if (cd >= 0) io_drain(cd);
             }
+            const int cdc = s - 1 - 2 * (NW - 1);
+            if constexpr (COOP) {
+                if (lane < CPW) {
+                    if (s + 1 < NT) coop_put(s + 1, fv, fcode);
+                    if (cdc >= 0) coop_drain(cdc);
+                }
+            }
             __syncthreads();
+            if constexpr (COOP) {
+                // every warp's drain of tile cdc is stored and fenced: publish it
+                if (threadIdx.x == 0 && cdc >= 0 && !s_abort) st_release(S.progress + b, cdc * W + W - SKEW);
+            }
             if (s_abort) break;
         }
-        if (warp == NW && lane == 0 && !s_abort) st_release(S.progress + b, INT_MAX);
+        if (threadIdx.x == (COOP ? 0 : NW * 32) && !s_abort) st_release(S.progress + b, INT_MAX);
         if (a.k > 0) {
             __threadfence();
             __syncthreads();

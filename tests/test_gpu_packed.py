@@ -10,7 +10,7 @@ import synth
 
 pytestmark = pytest.mark.gpu
 PAPER = (1, -3, 3, 2)
-PACKED_VARIANTS = [0, 3, 5]  # (16, 4), (16, 12), (16, 15) warps
+PACKED_VARIANTS = [0, 3, 5, 6]  # (16, 4), (16, 12), (16, 15) warps + I/O warp; 16 warps with cooperative I/O
 
 
 @pytest.fixture(scope="module")
