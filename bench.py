@@ -354,9 +354,9 @@ def main():
     peak = nsm * roof * sm_max * 1e6 / 1e9
     traffic = None
     try:
-        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        if tr.get("workload") == cfg.name and world == 1:
-            traffic = tr.get("fill_dram_bytes_per_launch")
+        for tr in json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))):
+            if tr.get("workload") == cfg.name and tr.get("kernel_dtype") == kdtype and world == 1:
+                traffic = tr.get("fill_dram_bytes_per_launch")
     except Exception:
         pass
     roofline = {"bound": "alu", "achieved": round(achieved, 2), "peak": round(peak, 1), "unit": "GCUPS",

@@ -132,8 +132,8 @@ int64_t sw_row_granularity(const sw_ctx *ctx);
 int64_t sw_band_height(const sw_ctx *ctx);
 
 /* Kernel selection (testing / tuning).  variant = -1: automatic choice per
- * call; 0..5: a fixed geometry (alpha, warps, tile width) of
- * the int32 kernel, or of the packed 16x2 kernel when packed = 1 and the call
+ * call; 0..7: a fixed geometry (alpha, warps, tile width) of
+ * the int32 kernel (DESIGN.md 4.1 lists them), or of the packed 16x2 kernel when packed = 1 and the call
  * qualifies (local mode, k % 16 == 0, small value window).  packed = 0 never
  * uses the packed kernel.  Results are identical for every choice. */
 int sw_set_kernel(sw_ctx *ctx, int variant, int packed);

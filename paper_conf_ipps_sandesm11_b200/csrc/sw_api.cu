@@ -106,6 +106,7 @@ struct Variant {
     const void *packed_fn;  // packed 16x2 Stage-1 kernel with the same band geometry (alpha 16 only)
     size_t smem16;
     int io_warps;           // 1, or 0 for the cooperative-I/O packed kernel (block = (nw + io) warps)
+    int skew_tiles;         // int32 kernel: tiles past the last column lane 31 needs (ceil(62 / W))
 };
 
 template <int ALPHA, int NW, int W>
@@ -121,7 +122,8 @@ static Variant make_variant()
     v.packed_fn = nullptr;
     v.smem16 = 0;
     v.io_warps = 1;
-    if constexpr (ALPHA == 16) {
+    v.skew_tiles = (Fill<ALPHA, NW, W, true>::SKEW + W - 1) / W;
+    if constexpr (ALPHA == 16 && W % 64 == 0) {
         if constexpr (NW == 16) {
             v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, true>;
             v.io_warps = 0;
@@ -134,7 +136,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 7;
+static constexpr int NVARIANTS = 8;
 
 static const Variant &variant_for(int idx)
 {
@@ -146,6 +148,7 @@ static const Variant &variant_for(int idx)
         make_variant<16, 14, 64>(),
         make_variant<16, 15, 64>(),
         make_variant<16, 16, 64>(),
+        make_variant<16, 8, 32>(),
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -176,11 +179,12 @@ struct sw_ctx {
     int num_sms = 0;
     cudaStream_t stream = nullptr, side = nullptr;
     cudaEvent_t ev[6] = {};
-    cudaEvent_t ev_row[8] = {};  // staging-row copies (special rows)
+    std::vector<cudaEvent_t> ev_row;  // one per staging slot: the slot's final copy is done
     int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
     DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
     HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
+    HostBuf colp[MAX_STRIPES];   // mapped pinned per-band final-column counts per stripe
     HostBuf stage;               // pinned staging for one special row (H then F)
     RecvArea vrecv[MAX_STRIPES]; // receive areas of virtual stripes 1..S-1
     // multi-GPU stripe (one per process): own receive area (exported), right neighbour's (imported)
@@ -294,8 +298,6 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
         if ((e = cudaStreamCreateWithFlags(&ctx->side, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
         for (auto &ev : ctx->ev)
             if ((e = cudaEventCreate(&ev)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
-        for (auto &ev : ctx->ev_row)
-            if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
         if (rc) break;
         if ((e = cudaHostAlloc(&ctx->res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
         for (int i = 0; i < NVARIANTS; i++) {
@@ -327,6 +329,7 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
         for (DevBuf *b : {&ctx->rowb[s], &ctx->progress[s], &ctx->sp[s]})
             if (b->p) cudaFree(b->p);
         if (ctx->flags[s].p) cudaFreeHost(ctx->flags[s].p);
+        if (ctx->colp[s].p) cudaFreeHost(ctx->colp[s].p);
         if (ctx->vrecv[s].base) cudaFree(ctx->vrecv[s].base);
     }
     if (ctx->right_base) cudaIpcCloseMemHandle(ctx->right_base);
@@ -464,6 +467,7 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
     }
     static const Candidate cands[] = {
         {DEFAULT_VARIANT, false, 2572.0},  // int32, 8 warps
+        {1, true, 3130.0},                 // packed, 8 warps + I/O warp
         {0, true, 2785.0},                 // packed, 4 warps, 3 CTAs/SM
         {3, true, 2851.0},                 // packed, 12 warps
         {5, true, 3243.0},                 // packed, 15 warps + I/O warp
@@ -497,8 +501,12 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
 
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
 {
+    const auto h0 = std::chrono::steady_clock::now();
+    double hck[6] = {0, 0, 0, 0, 0, 0};
+    auto hnow = [&]() { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - h0).count(); };
     bool use16 = false;
     const Variant &V = choose_variant(ctx, J, &use16);
+    hck[0] = hnow();
     const int W = V.w;
     const int BH = V.alpha * 32 * V.nw;
     const int m = (int)J.m, n = (int)J.n;
@@ -531,7 +539,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     const size_t border_flags = (size_t)nb * V.nw + 1;
     for (int s = 0; s < NS; s++) {
         const int npad = (int)((wid[s] + W - 1) / W) * W;
-        const int NT = npad / W + 1;
+        const int NT = npad / W + (use16 ? 1 : V.skew_tiles);
         if ((rc = grow(ctx, ctx->rowb[s], (size_t)(NT * W + 2 * W) * sizeof(int2)))) return rc;
         if ((rc = grow(ctx, ctx->progress[s], (size_t)(nb + 1) * sizeof(int)))) return rc;
         if (!J.rank_mode && s > 0)
@@ -557,6 +565,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     int per_stripe = std::max(1, std::min(nb, blocks_per_sm * ctx->num_sms / NS));
     if (const char *g = getenv("SWB_GRID")) per_stripe = std::max(1, std::min(per_stripe, atoi(g) / NS));
     const int grid = per_stripe * NS;
+    hck[1] = hnow();
     if ((rc = grow(ctx, ctx->slots, (size_t)grid * sizeof(int4)))) return rc;
 
     // special rows: all of them stay resident on the device (180 GB HBM) and
@@ -571,24 +580,44 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         row_ints += (size_t)stride[s];
     }
     if (nsp > 0) {
-        size_t freeb = 0, totb = 0;
-        cudaMemGetInfo(&freeb, &totb);
         size_t have = 0;
-        for (int s = 0; s < NS; s++) have += ctx->sp[s].cap;
-        const size_t need = (size_t)nsp * row_ints * sizeof(int);
-        if (need > have && need > (size_t)(0.8 * (double)(freeb + have))) {
-            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special rows need %zu bytes on the device", need);
-            return SW_ENOMEM;
+        bool grows = false;
+        for (int s = 0; s < NS; s++) {
+            have += ctx->sp[s].cap;
+            grows |= ctx->sp[s].cap < (size_t)nsp * stride[s] * sizeof(int);
         }
+        const size_t need = (size_t)nsp * row_ints * sizeof(int);
+        if (grows) {
+            // only when the buffers must grow: cudaMemGetInfo can take
+            // milliseconds (it stalled repeated calls by up to 19 ms)
+            size_t freeb = 0, totb = 0;
+            cudaMemGetInfo(&freeb, &totb);
+            if (need > (size_t)(0.8 * (double)(freeb + have))) {
+                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special rows need %zu bytes on the device", need);
+                return SW_ENOMEM;
+            }
+        }
+        hck[2] = hnow();
         for (int s = 0; s < NS; s++) {
             if ((rc = grow(ctx, ctx->sp[s], (size_t)nsp * stride[s] * sizeof(int)))) return rc;
             if ((rc = grow_host(ctx, ctx->flags[s], nsp * sizeof(unsigned int), true))) return rc;
             memset(ctx->flags[s].p, 0, nsp * sizeof(unsigned int));
         }
-        // staging ring: up to 8 rows, at most ~1 GiB of pinned memory
+        for (int s = 0; s < NS; s++) {
+            if ((rc = grow_host(ctx, ctx->colp[s], (size_t)nb * sizeof(unsigned int), true))) return rc;
+            memset(ctx->colp[s].p, 0, (size_t)nb * sizeof(unsigned int));
+        }
+        // staging window: every special row when they fit in ~1 GiB of pinned
+        // memory (a one-wave matrix completes all its rows together), else as
+        // many as fit (at least 2)
         const size_t row_bytes = (size_t)2 * (n + 64) * sizeof(int32_t);
-        ctx->nstage = (int)std::max<size_t>(2, std::min<size_t>(8, ((size_t)1 << 30) / row_bytes));
+        ctx->nstage = (int)std::max<size_t>(2, std::min<size_t>((size_t)nsp, ((size_t)1 << 30) / row_bytes));
         if ((rc = grow_host(ctx, ctx->stage, row_bytes * ctx->nstage, false))) return rc;
+        while ((int)ctx->ev_row.size() < ctx->nstage) {
+            cudaEvent_t ev;
+            CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+            ctx->ev_row.push_back(ev);
+        }
     }
 
     // With a caller stream, every kernel of the call is launched on it (so the
@@ -603,6 +632,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     int4 *d_res = (int4 *)(misc + 32);
     int *d_tickets = (int *)(misc + 64);  // MAX_STRIPES
 
+    hck[3] = hnow();
     CK(cudaEventRecord(ctx->ev[0], st));
     CK(cudaMemsetAsync(misc, 0, 16, st));
     CK(cudaMemsetAsync(d_hit_band, 0x7f, 4, st));
@@ -618,6 +648,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         CK(cudaGetLastError());
     }
     CK(cudaEventRecord(ctx->ev[1], st));
+    hck[4] = hnow();
 
     FillArgs a{};
     a.m = m;
@@ -661,7 +692,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         S.col0 = (int)col0[s];
         S.w = (int)wid[s];
         S.ncols_pad = (int)((wid[s] + W - 1) / W) * W;
-        S.NT = S.ncols_pad / W + 1;
+        S.NT = S.ncols_pad / W + (use16 ? 1 : V.skew_tiles);
         S.rowb = (int2 *)ctx->rowb[s].p;
         S.progress = (int *)ctx->progress[s].p;
         S.ticket = d_tickets + s;
@@ -671,6 +702,9 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         unsigned int *fd = nullptr;
         if (nsp > 0) CK(cudaHostGetDevicePointer((void **)&fd, ctx->flags[s].p, 0));
         S.row_done = fd;
+        unsigned int *cp = nullptr;
+        if (nsp > 0) CK(cudaHostGetDevicePointer((void **)&cp, ctx->colp[s].p, 0));
+        S.colp = cp;
         if (J.rank_mode) {
             S.lb = J.c_lo > 0 ? ctx->recv.lb() : nullptr;
             S.lready = J.c_lo > 0 ? ctx->recv.lready() : nullptr;
@@ -699,50 +733,80 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     CK(cudaEventRecord(ctx->ev[3], st));
 
     // Stream special rows to the sink in ascending order while the fill runs.
-    // A row is complete when every stripe of this launch has published it.
-    // Up to NSTAGE pinned staging rows: copies are issued as soon as rows are
-    // ready (bands of a short matrix finish in a burst), sinks run in order.
+    // A staged row is copied in column chunks as its band publishes final
+    // columns (colp), and completed once every stripe has published the row
+    // (row_done); the sink then runs on it in row order.
     int sink_rc = 0;
     long long bytes = 0;
     const int64_t nrow_out = J.rank_mode ? wid[0] : n;
     const int64_t sld = (NS == 1) ? ld[0] : nrow_out + 32;  // H at [0, sld), F at [sld, 2 sld)
     const int nstage = nsp > 0 ? ctx->nstage : 0;
+    const int64_t CHUNK = 65536;  // columns per partial copy (512 KiB of H + F)
+    std::vector<int64_t> copied((size_t)nstage * NS, 0);
+    std::vector<char> sealed(nstage, 0);
+    // SWB_DEBUG_HOST: host-side timeline of the special-row loop (stderr)
+    const bool dbg_host = nsp > 0 && getenv("SWB_DEBUG_HOST") != nullptr;
+    auto hms = [&]() { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - h0).count(); };
+    const double h_launch = hms();
+    double h_fill = -1, h_sink_max = 0;
+    long long n_copies = 0;
     auto row_ready = [&](long long q) -> bool {
         for (int s = 0; s < NS; s++)
             if (((volatile unsigned int *)ctx->flags[s].p)[q] == 0) return false;
         return true;
     };
-    auto issue_copy = [&](long long q) -> int {
-        int32_t *dst = (int32_t *)ctx->stage.p + (q % nstage) * 2 * sld;
+    // copy what is final of staged row q; true when the row has been sealed
+    auto pump = [&](long long q, bool &moved) -> int {
+        const int slot = (int)(q % nstage);
+        if (sealed[slot]) return SW_OK;
+        const bool ready = row_ready(q);
+        const int band = (int)(((q + 1) * J.k - 1) / BH);
+        bool all = true;
+        int32_t *dst = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
         for (int s = 0; s < NS; s++) {
-            const int32_t *src = (const int32_t *)ctx->sp[s].p + q * stride[s];
-            if (NS == 1) {
-                CK(cudaMemcpyAsync(dst, src, (size_t)stride[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
-            } else {
-                const int64_t off = J.rank_mode ? 0 : col0[s];
-                CK(cudaMemcpyAsync(dst + off, src, (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
-                CK(cudaMemcpyAsync(dst + sld + off, src + ld[s], (size_t)wid[s] * 4, cudaMemcpyDeviceToHost, ctx->side));
+            int64_t &c = copied[(size_t)slot * NS + s];
+            int64_t avail = wid[s];
+            if (!ready) avail = std::min<int64_t>(avail, ((volatile unsigned int *)ctx->colp[s].p)[band]);
+            if (avail > c && (ready || avail - c >= CHUNK)) {
+                const int32_t *src = (const int32_t *)ctx->sp[s].p + q * stride[s] + c;
+                const int64_t off = (NS == 1 || J.rank_mode) ? 0 : col0[s];
+                CK(cudaMemcpy2DAsync(dst + off + c, (size_t)sld * 4, src, (size_t)ld[s] * 4, (size_t)(avail - c) * 4, 2,
+                                     cudaMemcpyDeviceToHost, ctx->side));
+                n_copies++;
+                c = avail;
+                moved = true;
             }
+            if (c < wid[s]) all = false;
         }
-        CK(cudaEventRecord(ctx->ev_row[q % nstage], ctx->side));
+        if (ready && all) {
+            CK(cudaEventRecord(ctx->ev_row[slot], ctx->side));
+            sealed[slot] = 1;
+            moved = true;
+        }
         return SW_OK;
     };
-    long long issued = 0, done = 0;
+    long long done = 0;
     while (done < nsp) {
         bool progress = false;
-        while (issued < nsp && issued - done < nstage && row_ready(issued)) {
-            if (!sink_rc && (rc = issue_copy(issued))) return rc;
-            issued++;
-            progress = true;
+        if (dbg_host && h_fill < 0 && cudaEventQuery(ctx->ev[2]) == cudaSuccess) h_fill = hms();
+        if (!sink_rc) {
+            const long long hi = std::min<long long>(nsp, done + nstage);
+            for (long long q = done; q < hi; q++)
+                if ((rc = pump(q, progress))) return rc;
         }
-        if (issued > done) {
-            const cudaError_t qe = sink_rc ? cudaSuccess : cudaEventQuery(ctx->ev_row[done % nstage]);
+        const int slot = (int)(done % nstage);
+        if (sink_rc || sealed[slot]) {
+            const cudaError_t qe = sink_rc ? cudaSuccess : cudaEventQuery(ctx->ev_row[slot]);
             if (qe == cudaSuccess) {
                 if (!sink_rc) {
                     bytes += 8ll * nrow_out;
-                    int32_t *row = (int32_t *)ctx->stage.p + (done % nstage) * 2 * sld;
+                    int32_t *row = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
+                    const double t0 = dbg_host ? hms() : 0;
                     if (J.sink && J.sink(J.user, (done + 1) * J.k, row, row + sld, nrow_out)) sink_rc = SW_EABORTED;
+                    if (dbg_host) h_sink_max = std::max(h_sink_max, hms() - t0);
                 }
+                sealed[slot] = 0;
+                for (int s = 0; s < NS; s++) copied[(size_t)slot * NS + s] = 0;
                 done++;
                 progress = true;
             } else if (qe != cudaErrorNotReady) {
@@ -752,10 +816,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         if (!progress) {
             // nothing ready: make sure the fill is still running
             const cudaError_t fe = cudaEventQuery(ctx->ev[2]);
-            if (fe == cudaSuccess && issued < nsp && !row_ready(issued)) {
+            if (fe == cudaSuccess && !sealed[slot] && !row_ready(done)) {
                 CK(cudaStreamSynchronize(st));
                 if (ctx->res_h[1].x == 1) return SW_EALPHABET;
-                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", issued,
+                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", done,
                          ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
                 return SW_ECUDA;
             } else if (fe != cudaSuccess && fe != cudaErrorNotReady) {
@@ -764,7 +828,14 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             std::this_thread::yield();
         }
     }
+    if (dbg_host)
+        fprintf(stderr, "[swb host] rows %lld copies %lld launched %.2f ms fill_seen %.2f ms loop_end %.2f ms max_sink %.3f ms nstage %d\n",
+                nsp, n_copies, h_launch, h_fill, hms(), h_sink_max, nstage);
+    if (sink_rc) CK(cudaStreamSynchronize(ctx->side));  // no copy may land in a reused staging slot later
     CK(cudaStreamSynchronize(st));
+    if (dbg_host)
+        fprintf(stderr, "[swb host] synced %.2f ms; pre-launch: variant %.2f grid %.2f meminfo %.2f staging %.2f encode %.2f\n", hms(),
+                hck[0], hck[1], hck[2], hck[3], hck[4]);
     if (ctx->res_h[1].x == 1) return SW_EALPHABET;
     if (ctx->res_h[1].x == 2) {
         snprintf(ctx->errbuf, sizeof(ctx->errbuf), "fill kernel: border wait timeout (a neighbour stripe did not progress)");

@@ -51,7 +51,7 @@ struct StripeArgs {
     int col0;            // first global 0-based column
     int w;               // real columns of the stripe
     int ncols_pad;       // w rounded up to a multiple of W
-    int NT;              // tiles each warp runs per band = ncols_pad / W + 1
+    int NT;              // tiles each warp runs per band = ncols_pad / W + ceil(lane skew / W)
     int2 *rowb;          // row border: (t, F) per local column, >= NT*W + W entries
     int *progress;       // per band: number of leading columns of its bottom row published
     int *ticket;         // band ticket of this stripe
@@ -59,6 +59,7 @@ struct StripeArgs {
     long long sp_stride;
     int sp_ld;
     unsigned int *row_done;  // mapped host flags, one per special row
+    unsigned int *colp;  // mapped host words, one per band: leading columns of the band's special rows that are final
     const int2 *lb;      // left border (t, E) per DP row 0..m at column col0 - 1 (null: column-0 boundary)
     const int *lready;   // per (band, warp) epoch flags guarding lb
     int2 *rb;            // right neighbour's lb (null: last stripe); a peer-GPU pointer across GPUs
@@ -183,6 +184,27 @@ __device__ __forceinline__ void st_release_sys(unsigned int *p, unsigned int v)
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
+// True when DP rows b*BH+1 .. min((b+1)*BH, m) hold a special row (k > 0).
+__device__ __forceinline__ bool band_has_special(int b, int BH, int m, int k)
+{
+    if (k <= 0) return false;
+    const long long lo = (long long)b * BH + 1, hi = min((long long)(b + 1) * BH, (long long)m);
+    return ((lo + k - 1) / k) * k <= hi;
+}
+
+// Every 16th drained tile of a band holding special rows: tell the host how
+// many leading columns of them are final, so it can copy them while the band
+// is still running (the rows of a one-wave matrix all complete at the end).
+// Called by the thread that published the band's progress, after the drained
+// stores of the whole warp/CTA are fenced.
+__device__ __forceinline__ void publish_cols(unsigned int *colp, int b, int cd, int cols)
+{
+    if (colp != nullptr && (cd & 15) == 15) {
+        __threadfence_system();
+        st_release_sys(colp + b, (unsigned int)cols);
+    }
+}
+
 // (score, i, j) total order: higher score, then smaller i, then smaller j (reading S4)
 __device__ __forceinline__ bool better(int s, int i, int j, int bs, int bi, int bj)
 {
@@ -191,8 +213,11 @@ __device__ __forceinline__ bool better(int s, int i, int j, int bs, int bi, int 
 
 template <int W, int NW>
 struct Smem {
-    static constexpr int RING = 4 * W;
-    static constexpr int SRING_MIN = 2 * NW * W + 2 * 32 * LANE_SKEW;
+    // warp lag in tiles: lane 31 of the warp above must be done with a tile's
+    // columns before lane 0 below starts them (1 + ceil(skew / W), skew <= 63)
+    static constexpr int LAG = 1 + (63 + W - 1) / W;
+    static constexpr int RING = W >= 64 ? 4 * W : 256;
+    static constexpr int SRING_MIN = (LAG * (NW - 1) + 2) * W + 64;
     static constexpr int SRING = SRING_MIN <= 256 ? 256 : SRING_MIN <= 512 ? 512 : SRING_MIN <= 1024 ? 1024 : SRING_MIN <= 2048 ? 2048 : 4096;
 };
 
@@ -204,7 +229,10 @@ struct Fill {
     static constexpr int NSAVE = 2 * ALPHA + 5;
     static constexpr int SKEW = 31 * LANE_SKEW;  // columns lane 31 lags lane 0
     static constexpr int STEPS = W / LANE_SKEW;  // lane steps per tile
-    static_assert(W % 64 == 0 && W > SKEW, "W multiple of 64, larger than the warp skew");
+    static constexpr int LAG = 1 + (SKEW + W - 1) / W;  // tiles warp w+1 trails warp w
+    static constexpr int GUARD_TILES = (31 + STEPS - 1) / STEPS;  // tiles where some lane is left of column 0
+    static_assert(W % 32 == 0 && LAG <= Smem<W, NW>::LAG, "W multiple of 32");
+    static_assert((LAG + 1) * W <= RING, "ring holds the producer/consumer span");
     static_assert(ALPHA % 2 == 0 && ALPHA <= 16, "ALPHA even, <= 16");
 
     static size_t smem_bytes()
@@ -407,7 +435,7 @@ template <int ALPHA, int NW, int W, bool LOCAL>
 __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_constant__ FillArgs a)
 {
     using F = Fill<ALPHA, NW, W, LOCAL>;
-    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
+    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS, LAG = F::LAG;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int2 *rings = reinterpret_cast<int2 *>(smem_raw);                        // (NW+1) x RING
     uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * RING);  // SRING
@@ -513,6 +541,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             const int bottom = (b + 1) * BH;
             if (bottom <= a.m && bottom % a.k == 0) io_sp = S.sp + (long long)(bottom / a.k - 1) * S.sp_stride;
         }
+        unsigned int *const colp = (LOCAL && band_has_special(b, BH, a.m, a.k)) ? S.colp : nullptr;
         auto io_drain = [&](int cd) {
             const int2 *ringN = rings + NW * RING;
 #pragma unroll
@@ -529,7 +558,10 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             }
             __threadfence();
             __syncwarp();
-            if (lane == 0) st_release(S.progress + b, cd * W + W - SKEW);
+            if (lane == 0) {
+                st_release(S.progress + b, cd * W + W - SKEW);
+                publish_cols(colp, b, cd, cd * W + W - SKEW);
+            }
         };
         // left border of this warp's rows (stripes after the first): wait for the
         // left neighbour's flags, then take (t, E) at column col0 - 1 as the state.
@@ -556,11 +588,11 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
         if (warp == NW) io_load(0);
         __syncthreads();
         if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 1] = gtimer();
-        const int S_END = NT + 2 * (NW - 1);
+        const int S_END = NT + LAG * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s <= S_END; ++s) {
             if (warp < NW) {
-                const int c = s - 2 * warp;
+                const int c = s - LAG * warp;
                 if (c >= 0 && c < NT) {
                     const uint32_t rin = pin((uint32_t)__cvta_generic_to_shared(rings + warp * RING));
                     const uint32_t rout = pin((uint32_t)__cvta_generic_to_shared(rings + (warp + 1) * RING));
@@ -580,7 +612,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                             __syncwarp();
                             if (lane == 0) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
                         }
-                    } else if (c == 0 || (warp_sp && spm == 2)) {
+                    } else if (c < F::GUARD_TILES || (warp_sp && spm == 2)) {
                         tmax = F::template tile<true, false, 2>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, smask);
                     } else if (warp_sp) {
                         tmax = F::template tile_fast<true>(a, X, L, c, lane, rin, rout, selr_s, sp_ptr);
@@ -603,7 +635,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                 }
             } else {
                 if (s + 1 < NT) io_load(s + 1);
-                const int cd = s - 1 - 2 * (NW - 1);
+                const int cd = s - 1 - LAG * (NW - 1);
                 if (cd >= 0) io_drain(cd);
                 if (!LOCAL && lane == 0 && ld_relaxed(a.hit_band) < b) s_abort = 1;
             }

@@ -390,6 +390,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             const int bottom = (b + 1) * BH;
             if (bottom <= a.m && bottom % a.k == 0) io_sp = S.sp + (long long)(bottom / a.k - 1) * S.sp_stride;
         }
+        unsigned int *const colp = band_has_special(b, BH, a.m, a.k) ? S.colp : nullptr;
         auto io_drain = [&](int cd) {
             const int2 *ringN = rings + NW * RING;
 #pragma unroll
@@ -406,7 +407,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             }
             __threadfence();
             __syncwarp();
-            if (lane == 0) st_release(S.progress + b, cd * W + W - SKEW);
+            if (lane == 0) {
+                st_release(S.progress + b, cd * W + W - SKEW);
+                publish_cols(colp, b, cd, cd * W + W - SKEW);
+            }
         };
         auto wait_left = [&]() {
             if (lane == 0) {
@@ -539,7 +543,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             __syncthreads();
             if constexpr (COOP) {
                 // every warp's drain of tile cdc is stored and fenced: publish it
-                if (threadIdx.x == 0 && cdc >= 0 && !s_abort) st_release(S.progress + b, cdc * W + W - SKEW);
+                if (threadIdx.x == 0 && cdc >= 0 && !s_abort) {
+                    st_release(S.progress + b, cdc * W + W - SKEW);
+                    publish_cols(colp, b, cdc, cdc * W + W - SKEW);
+                }
             }
             if (s_abort) break;
         }

@@ -130,6 +130,18 @@ def test_bad_parameters(ctx):
     assert rc == SW_ERANGE
 
 
+@pytest.mark.parametrize("packed", [True, False])
+def test_special_rows_streamed_in_chunks(ctx, packed):
+    # rows wider than the host's copy chunk (65536 columns): the host copies
+    # each row's final columns while its band still runs, then the rest
+    A, B = synth.random_pair(77, 8292, 200_003, plant_len=6000, s=0.05, g=0.01)
+    ctx.set_kernel(-1, packed)
+    try:
+        check_stage1(ctx, A, B, PAPER, 2048)
+    finally:
+        ctx.set_kernel(-1, True)
+
+
 def test_sink_abort(ctx):
     from paper_conf_ipps_sandesm11_b200 import SW_EABORTED, SwError
 
