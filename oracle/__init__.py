@@ -80,6 +80,8 @@ def _load():
             lib.or_global.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64]
             lib.or_global.restype = i64
             lib.or_reverse_goal.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, ctypes.POINTER(_Res)]
+            lib.or_stage2.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, i64, i64, i64, p64, i64]
+            lib.or_stage2.restype = i64
             lib.or_flush_rows.argtypes = [i64, i64, i64, i64]
             lib.or_flush_rows.restype = i64
             _lib = lib
@@ -163,6 +165,23 @@ def reverse_goal(A, i_end, B, j_end, ma, mi, go, ge, goal):
     res = _Res()
     found = lib.or_reverse_goal(a, i_end, b, j_end, ma, mi, go, ge, goal, ctypes.byref(res))
     return (res.score, res.i, res.j) if found else None
+
+
+def stage2(A, B, ma, mi, go, ge, k, best, i_end, j_end):
+    """Stage 2 crosspoint list L_2, ascending: [(i, j, score, type), ...]
+    from the start point to the end point (i_end, j_end, best, 0); type 2 = vertical gap."""
+    lib = _load()
+    a, b = _b(A), _b(B)
+    cap = 64
+    while True:
+        buf = (ctypes.c_int64 * (4 * cap))()
+        cnt = lib.or_stage2(a, len(a), b, len(b), ma, mi, go, ge, k, best, i_end, j_end,
+                            ctypes.cast(buf, ctypes.POINTER(ctypes.c_int64)), cap)
+        if cnt < 0:
+            raise RuntimeError(f"or_stage2 failed rc={cnt}")
+        if cnt <= cap:
+            return [tuple(int(buf[4 * q + x]) for x in range(4)) for q in range(cnt)]
+        cap = cnt
 
 
 def flush_rows(m, n, alphaT, sra_bytes) -> int:

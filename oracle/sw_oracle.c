@@ -26,6 +26,8 @@
  *   S7  characters are compared case-insensitively (codes A,C,G,T).
  *   S9/S10 reverse pass: anchored global recurrence on the reversed
  *       prefixes; first hit in row-major order of the reverse matrix.
+ *   S18-S22 Stage 2 (or_stage2): junction rules, anchor initialisation by
+ *       crosspoint type, event order of the orthogonal sweep, termination.
  *
  * Arithmetic: int64 everywhere (wider than any kernel; the paper uses
  * 4-byte cells, and all values here stay far inside int32).
@@ -286,4 +288,140 @@ int64_t or_flush_rows(int64_t m, int64_t n, int64_t alphaT, int64_t sra_bytes)
     while (q > 0 && (long double)(q - 1) * den >= num) q--;
     if (q < 1) q = 1;
     return alphaT * q;
+}
+
+/*
+ * Stage 2, partial traceback, plainly: from the end point
+ * C = (i_end, j_end, best, 0) back to the start point, one partition at a
+ * time, returning the crosspoint list L_2 in ascending order
+ * (start point first, end point last).  A crosspoint is (i, j, score, type),
+ * type 0 = match/mismatch, 2 = gap in S1 (a vertical gap, matrix F).
+ *
+ * One iteration, for the current crosspoint (i_c, j_c, g, type):
+ *  - the partition is rows r..i_c, r = the nearest special row strictly above
+ *    i_c (r = ((i_c - 1) / k) k; r = 0 means "none": row 0 then plays the
+ *    special row with H = 0, F = -infinity, the local boundary, reading S21);
+ *  - the reverse DP is the global recurrence anchored at (i_c, j_c)
+ *    over i' = i_c - i in [0, i_c - r], j' = j_c - j in [0, j_c]:
+ *    H'(0,0) = 0, column j' = 0: H' = F' = -(G_open + i' G_ext), E' = -inf;
+ *    row i' = 0: H' = E' = -(G_open + j' G_ext), F' = -inf.  When the anchor
+ *    is a gap crosspoint (type 2) the path must leave it by continuing that
+ *    vertical gap, so the row i' = 0 (j' >= 1) is -infinity and so is the
+ *    diagonal out of the anchor ("the initialization must be adjusted not to
+ *    consider a duplicated gap open penalty"; reading S20);
+ *  - events, in the order of the orthogonal sweep (Fig. 7: vertical
+ *    strips j' = 0, 1, 2, ...; reading S19), the first one wins:
+ *      start:   H'(i', j') == g for 1 <= i' < i_c - r  -> the start point
+ *               (i_c - i', j_c - j', 0, 0);
+ *      H-match: Hs(j) + H'(i_c - r, j') == g           -> (r, j, Hs(j), 0);
+ *      F-match: Fs(j) + F'(i_c - r, j') + G_open == g  -> (r, j, Fs(j), 2)
+ *               (a vertical gap crossing row r is charged G_open once, not
+ *               twice; reading S18), where j = j_c - j' and Hs, Fs are
+ *               the special row r of Stage 1 (Hs(0) = 0, Fs(0) = -inf);
+ *      within one strip: starts by increasing i', then H-match, then F-match.
+ *  - the new crosspoint's score is the special row's H, or its F for a gap
+ *    (P:233); the loop ends at a crosspoint with score 0 and type 0 (the
+ *    start point; a gap crosspoint may have a score <= 0, reading S22).
+ * The special rows are recomputed here with or_stage1 (rows k, 2k, ...).
+ * Returns the number of crosspoints (writes min(count, cap) of them), or
+ * -1 (allocation), -3 (no event: inconsistent inputs).
+ */
+typedef struct {
+    int64_t i;
+    int64_t j;
+    int64_t score;
+    int64_t type;
+} or_crosspoint;
+
+typedef struct {
+    int64_t n, k, count;
+    int64_t *H, *F; /* count rows of n + 1 values (column 0 included) */
+} or_rows;
+
+static int keep_row(void *user, int64_t row, const int64_t *H, const int64_t *F, int64_t n)
+{
+    or_rows *R = (or_rows *)user;
+    int64_t q = row / R->k - 1;
+    R->H[q * (n + 1)] = 0;   /* H(r, 0) = 0   (local boundary, reading S3) */
+    R->F[q * (n + 1)] = NEG; /* F(r, 0) = -inf */
+    memcpy(R->H + q * (n + 1) + 1, H, (size_t)n * sizeof(int64_t));
+    memcpy(R->F + q * (n + 1) + 1, F, (size_t)n * sizeof(int64_t));
+    R->count = q + 1;
+    return 0;
+}
+
+int64_t or_stage2(const char *S0, int64_t m, const char *S1, int64_t n, int64_t ma, int64_t mi,
+                  int64_t G_open, int64_t G_ext, int64_t k, int64_t best, int64_t i_end, int64_t j_end,
+                  or_crosspoint *out, int64_t cap)
+{
+    const int64_t G_first = G_open + G_ext;
+    or_rows R = {n, k, 0, NULL, NULL};
+    const int64_t nrows = k > 0 ? m / k : 0;
+    if (nrows > 0) {
+        R.H = malloc((size_t)(nrows * (n + 1)) * sizeof(int64_t));
+        R.F = malloc((size_t)(nrows * (n + 1)) * sizeof(int64_t));
+        if (!R.H || !R.F) { free(R.H); free(R.F); return -1; }
+        or_result b1;
+        or_stage1(S0, m, S1, n, ma, mi, G_open, G_ext, k, keep_row, &R, &b1);
+    }
+    /* the list is built from the end point backwards */
+    int64_t ncp = 0, capl = 16;
+    or_crosspoint *L = malloc((size_t)capl * sizeof(or_crosspoint));
+    or_crosspoint C = {i_end, j_end, best, 0};
+    L[ncp++] = C;
+    int64_t rc = 0;
+    while (!(C.score == 0 && C.type == 0)) {
+        const int64_t ic = C.i, jc = C.j, g = C.score;
+        const int64_t r = k > 0 ? ((ic - 1) / k) * k : 0;
+        const int64_t Lr = ic - r;
+        const int64_t w = jc + 1;
+        int64_t *RH = malloc((size_t)((Lr + 1) * w) * sizeof(int64_t));
+        int64_t *RE = malloc((size_t)((Lr + 1) * w) * sizeof(int64_t));
+        int64_t *RF = malloc((size_t)((Lr + 1) * w) * sizeof(int64_t));
+        if (!RH || !RE || !RF) { free(RH); free(RE); free(RF); rc = -1; break; }
+        for (int64_t a = 0; a <= Lr; a++)
+            for (int64_t b = 0; b <= jc; b++) {
+                int64_t *h = &RH[a * w + b], *e = &RE[a * w + b], *f = &RF[a * w + b];
+                if (a == 0 && b == 0) { *h = 0; *e = NEG; *f = NEG; continue; }
+                if (b == 0) { *h = -(G_open + a * G_ext); *f = *h; *e = NEG; continue; }
+                if (a == 0) {
+                    if (C.type == 2) { *h = NEG; *e = NEG; }
+                    else { *h = -(G_open + b * G_ext); *e = *h; }
+                    *f = NEG;
+                    continue;
+                }
+                *e = max2(RE[a * w + b - 1] - G_ext, RH[a * w + b - 1] - G_first); /* Eq. 2 */
+                *f = max2(RF[(a - 1) * w + b] - G_ext, RH[(a - 1) * w + b] - G_first); /* Eq. 3 */
+                int64_t diag = RH[(a - 1) * w + b - 1];
+                if (a == 1 && b == 1 && C.type == 2) diag = NEG;
+                /* reversed sequences: row i' pairs S0[ic - i' + 1] (1-based) */
+                *h = max2(max2(*e, *f), diag + p_score(S0[ic - a], S1[jc - b], ma, mi)); /* Eq. 1, no 0 */
+            }
+        const int64_t *Hs = r > 0 ? R.H + (r / k - 1) * (n + 1) : NULL;
+        const int64_t *Fs = r > 0 ? R.F + (r / k - 1) * (n + 1) : NULL;
+        int found = 0;
+        or_crosspoint X = {0, 0, 0, 0};
+        for (int64_t b = 0; b <= jc && !found; b++) {
+            for (int64_t a = 1; a < Lr && !found; a++)
+                if (RH[a * w + b] == g) { X.i = ic - a; X.j = jc - b; X.score = 0; X.type = 0; found = 1; }
+            if (found) break;
+            const int64_t j = jc - b;
+            const int64_t hs = Hs ? Hs[j] : 0, fs = Fs ? Fs[j] : NEG;
+            if (hs + RH[Lr * w + b] == g) { X.i = r; X.j = j; X.score = hs; X.type = 0; found = 1; break; }
+            if (fs > NEG / 2 && RF[Lr * w + b] > NEG / 2 && fs + RF[Lr * w + b] + G_open == g) {
+                X.i = r; X.j = j; X.score = fs; X.type = 2; found = 1; break;
+            }
+        }
+        free(RH); free(RE); free(RF);
+        if (!found) { rc = -3; break; }
+        if (ncp == capl) { capl *= 2; L = realloc(L, (size_t)capl * sizeof(or_crosspoint)); }
+        L[ncp++] = X;
+        C = X;
+    }
+    if (rc == 0) {
+        for (int64_t q = 0; q < ncp && q < cap; q++) out[q] = L[ncp - 1 - q];
+        rc = ncp;
+    }
+    free(L); free(R.H); free(R.F);
+    return rc;
 }

@@ -333,3 +333,113 @@ def test_flush_interval_reproduces_table_viii():
             assert abs(predicted - int(printed)) <= 1
     # SRA of 50 GiB gives R = 229,632 rows
     assert oracle.flush_rows(m, n, alphaT, 50 << 30) == 229_632
+
+
+# ---------------------------------------------------------------- Stage 2
+#
+# or_stage2 is pinned by (1) closed forms of a planted gap crossing special
+# rows, (2) the partition property S(C_s, C_e) = score_e - score_s
+# checked with an independent, test-local Gotoh that honours the crosspoint
+# types (a segment leaving a gap crosspoint continues its vertical gap at
+# G_ext per row; a segment entering one ends with a vertical gap), (3) the
+# start point rescored with the pinned global oracle, (4) one crosspoint per
+# special row between start and end, and (5) crosspoint scores equal to the
+# Stage-1 special rows (H, or F for a gap).
+
+NEGI = -(1 << 40)
+
+
+def _segment_score(a, b, ma, mi, go, ge, t_s, t_e):
+    """Best global score of a[0:] x b[0:] as a segment between two crosspoints:
+    t_s = 2 -> must start by continuing a vertical gap (G_ext per row, no
+    opening); t_e = 2 -> must end with a vertical gap into the end cell."""
+    gf = go + ge
+    m, n = len(a), len(b)
+    H = [[NEGI] * (n + 1) for _ in range(m + 1)]
+    E = [[NEGI] * (n + 1) for _ in range(m + 1)]
+    F = [[NEGI] * (n + 1) for _ in range(m + 1)]
+    if t_s == 0:
+        H[0][0] = 0
+        for j in range(1, n + 1):
+            H[0][j] = E[0][j] = -(go + j * ge)
+        for i in range(1, m + 1):
+            H[i][0] = F[i][0] = -(go + i * ge)
+    else:  # continuing the vertical gap of the start crosspoint
+        for i in range(1, m + 1):
+            H[i][0] = F[i][0] = -i * ge
+    for i in range(1, m + 1):
+        for j in range(1, n + 1):
+            E[i][j] = max(E[i][j - 1] - ge, H[i][j - 1] - gf)
+            F[i][j] = max(F[i - 1][j] - ge, H[i - 1][j] - gf)
+            p = ma if a[i - 1] == b[j - 1] else mi
+            H[i][j] = max(E[i][j], F[i][j], H[i - 1][j - 1] + p)
+    if t_e == 2:
+        return F[m][n]
+    return H[m][n]
+
+
+def _check_stage2_list(A, B, sc, k):
+    (best, ie, je), rows = oracle.stage1(A, B, *sc, k=k, keep_rows=True) if k > 0 else (oracle.stage1(A, B, *sc, k=0)[0], [])
+    L = oracle.stage2(A, B, *sc, k, best, ie, je)
+    assert L[-1] == (ie, je, best, 0)
+    i1, j1, s1, t1 = L[0]
+    assert (s1, t1) == (0, 0)
+    # (3) the start point: the alignment from it to the end scores best
+    assert oracle.global_score(A[i1:ie], B[j1:je], *sc) == best or best == 0
+    # (4) one crosspoint per special row strictly between start and end
+    if k > 0:
+        want_rows = [r for r in range(k, ie, k) if r > i1]
+        assert [c[0] for c in L[1:-1]] == want_rows
+    # (5) scores are the special rows' H (type 0) or F (type 2)
+    H = {r: h for r, h, f in rows}
+    Fm = {r: f for r, h, f in rows}
+    for (i, j, s, t) in L[1:-1]:
+        if j == 0:
+            assert (s, t) == (0, 0)
+        else:
+            assert s == (Fm[i][j - 1] if t == 2 else H[i][j - 1]), (i, j, s, t)
+    # (2) partition additivity with the type-aware segment score
+    for (cs, ce) in zip(L, L[1:]):
+        seg = _segment_score(A[cs[0]:ce[0]], B[cs[1]:ce[1]], *sc, cs[3], ce[3])
+        assert seg == ce[2] - cs[2], (cs, ce, seg)
+    return L
+
+
+def test_stage2_planted_gap_closed_forms():
+    # X + TTTT + Y against X + Y: a 4-row vertical gap (a gap in S1) after
+    # 20 matches.  Crossing row 20 + d (d = 1..3) inside the gap, the special
+    # row's F is 20 - G_first - (d - 1) G_ext (Eq. 3); at row 24 the gap has
+    # closed and the crosspoint is H-type with H = 20 - 3 - 4*2 = 9.
+    X = "ACGTTGCAACGGTACCTGAT"
+    Y = "GGCATTACGATCCAGTACGA"
+    A, B = X + "TTTT" + Y, X + Y
+    best = 40 - (3 + 4 * 2)
+    assert oracle.stage1(A, B, *PAPER, k=0)[0] == (best, 44, 40)
+    L = _check_stage2_list(A, B, PAPER, 22)
+    assert L == [(0, 0, 0, 0), (22, 20, 20 - 5 - 2, 2), (44, 40, best, 0)]
+    L1 = _check_stage2_list(A, B, PAPER, 1)
+    assert L1[21:25] == [(21, 20, 15, 2), (22, 20, 13, 2), (23, 20, 11, 2), (24, 20, 9, 0)]
+    assert all(c == (r, r, r, 0) for r, c in zip(range(21), L1[:21]))
+    # no special row between start and end: the list is {start, end}
+    assert _check_stage2_list(A, B, PAPER, 100) == [(0, 0, 0, 0), (44, 40, best, 0)]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_stage2_properties_random(seed):
+    rng = random.Random(seed)
+    sc = [PAPER, (2, -1, 4, 1), (1, -1, 0, 2), (5, -4, 10, 1), (3, -2, 0, 1), (1, -3, 3, 2)][seed]
+    A, B = synth.random_pair(300 + seed, 160 + 7 * seed, 150, plant_len=120, s=0.08, g=0.04, mu=3)
+    A, B = A.tobytes().decode(), B.tobytes().decode()
+    for k in (1, 3, 16, 40, 500):
+        _check_stage2_list(A, B, sc, k)
+    # an inserted/deleted block crossing several special rows
+    base = _rand_seq(rng, 60)
+    A2 = base[:30] + _rand_seq(rng, 9) + base[30:]
+    _check_stage2_list(A2, base, sc, 4)
+    _check_stage2_list(base, A2, sc, 4)
+
+
+def test_stage2_zero_score_and_no_rows():
+    assert oracle.stage2("AAAA", "CCCC", *PAPER, 2, 0, 0, 0) == [(0, 0, 0, 0)]
+    (b, i, j), _ = oracle.stage1("ACGT", "ACGT", *PAPER, k=0)
+    assert oracle.stage2("ACGT", "ACGT", *PAPER, 0, b, i, j) == [(0, 0, 0, 0), (4, 4, 4, 0)]
