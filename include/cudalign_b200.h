@@ -59,6 +59,16 @@ typedef struct {
     int64_t j;
 } sw_result;
 
+/* Crosspoint: a cell (i, j) where the optimal alignment crosses a
+ * special row, its score there and its type: 0 = match/mismatch (H), 2 = gap
+ * in S1 (a vertical gap, matrix F).  The start point has score 0, type 0. */
+typedef struct {
+    int64_t i;
+    int64_t j;
+    int32_t score;
+    int32_t type;
+} sw_crosspoint;
+
 /* Special-row sink: H and F are columns 1..n of DP row `row`, int32,
  * in library-owned pinned host memory valid only during the call.  Called
  * from the thread that called sw_align_stage1, rows strictly ascending.
@@ -122,6 +132,31 @@ int sw_reverse_goal(sw_ctx *ctx, const char *seqA, int64_t i_end, const char *se
 int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end, const char *dseqB, int64_t j_end,
                         int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
                         int32_t goal, void *stream, sw_result *start_out);
+
+/* Stage 2, partial traceback (readings S18-S22).
+ * From the end point `end` (the Stage-1 result) back to the start point, find
+ * where the optimal alignment crosses each special row by goal-based matching
+ * of a reverse global fill against the special rows, which must still
+ * be resident from the LAST sw_align_stage1 / sw_align_stage1_dev call on this
+ * context with the same sequences, m, n, scoring and special_row_interval, run
+ * on one GPU without virtual stripes (else SW_EINVAL; the sequences themselves
+ * are the caller's responsibility).  special_row_interval 0 is allowed (one
+ * partition: the start point only).
+ * Output: the crosspoint list L_2 in ascending order, start point
+ * first and `end` last, into out[0 .. cap) (caller-owned); *count = its
+ * length.  cap < *count: the first cap entries are written and SW_ERANGE is
+ * returned.  SW_ENOTFOUND when no junction exists (inputs inconsistent with
+ * the rows).  The sequences are host pointers; the device variant below takes
+ * HBM pointers and a stream. */
+int sw_stage2(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, int64_t n,
+              int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+              int64_t special_row_interval, const sw_result *end,
+              sw_crosspoint *out, int64_t cap, int64_t *count);
+
+int sw_stage2_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                  int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                  int64_t special_row_interval, const sw_result *end, void *stream,
+                  sw_crosspoint *out, int64_t cap, int64_t *count);
 
 /* Rows per thread strip (alpha): special_row_interval multiples of this take
  * the fast special-row path. */

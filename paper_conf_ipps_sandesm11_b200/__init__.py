@@ -37,6 +37,8 @@ EXPORTED = [
     "sw_align_stage1_dev",
     "sw_reverse_goal",
     "sw_reverse_goal_dev",
+    "sw_stage2",
+    "sw_stage2_dev",
     "sw_row_granularity",
     "sw_band_height",
     "sw_set_kernel",
@@ -60,6 +62,10 @@ class SwError(RuntimeError):
 
 class _Result(ctypes.Structure):
     _fields_ = [("score", ctypes.c_int32), ("i", ctypes.c_int64), ("j", ctypes.c_int64)]
+
+
+class _Crosspoint(ctypes.Structure):
+    _fields_ = [("i", ctypes.c_int64), ("j", ctypes.c_int64), ("score", ctypes.c_int32), ("type", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -115,6 +121,11 @@ def load_library(path: str = LIB_PATH):
     lib.sw_reverse_goal.restype = ctypes.c_int
     lib.sw_reverse_goal_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, vp, R]
     lib.sw_reverse_goal_dev.restype = ctypes.c_int
+    CP = ctypes.POINTER(_Crosspoint)
+    lib.sw_stage2.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i64, R, CP, i64, ctypes.POINTER(i64)]
+    lib.sw_stage2.restype = ctypes.c_int
+    lib.sw_stage2_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i64, R, vp, CP, i64, ctypes.POINTER(i64)]
+    lib.sw_stage2_dev.restype = ctypes.c_int
     lib.sw_row_granularity.argtypes = [vp]
     lib.sw_row_granularity.restype = i64
     lib.sw_band_height.argtypes = [vp]
@@ -246,6 +257,35 @@ class Context:
                                            goal, stream or None, ctypes.byref(out))
         self._check(rc, "sw_reverse_goal_dev")
         return Result(out.score, out.i, out.j)
+
+    def _stage2_call(self, fn, args, cap):
+        while True:
+            buf = (_Crosspoint * max(1, cap))()
+            cnt = ctypes.c_int64(0)
+            rc = fn(*args, buf, cap, ctypes.byref(cnt))
+            if rc == SW_ERANGE and cnt.value > cap:
+                cap = cnt.value
+                continue
+            self._check(rc, fn.__name__)
+            return [(c.i, c.j, c.score, c.type) for c in buf[: cnt.value]]
+
+    def stage2(self, A, B, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0, end=None):
+        """Stage 2 crosspoint list L_2 (ascending, start point first) from the end
+        point `end` (a Result / (score, i, j)) against the special rows kept from
+        the last align_stage1 call with the same inputs, k and scoring."""
+        pa, m, ka = _as_bytes_ptr(A)
+        pb, n, kb = _as_bytes_ptr(B)
+        e = end if isinstance(end, tuple) else end.astuple()
+        r = _Result(e[0], e[1], e[2])
+        return self._stage2_call(self._lib.sw_stage2, (self._h, pa, m, pb, n, match, mismatch, gap_open, gap_ext, k,
+                                                       ctypes.byref(r)), 64)
+
+    def stage2_dev(self, dA_ptr, m, dB_ptr, n, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0, end=None,
+                   stream: int = 0):
+        e = end if isinstance(end, tuple) else end.astuple()
+        r = _Result(e[0], e[1], e[2])
+        return self._stage2_call(self._lib.sw_stage2_dev, (self._h, dA_ptr, m, dB_ptr, n, match, mismatch, gap_open,
+                                                           gap_ext, k, ctypes.byref(r), stream or None), 64)
 
     def row_granularity(self) -> int:
         return int(self._lib.sw_row_granularity(self._h))

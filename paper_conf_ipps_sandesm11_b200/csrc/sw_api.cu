@@ -174,6 +174,14 @@ struct RecvArea {
     int *lready() const { return (int *)((char *)base + rows * sizeof(int2)); }
 };
 
+// Where the special rows of the last Stage-1 call live (for Stage 2).
+struct S1Rows {
+    bool valid = false;
+    int64_t m = 0, n = 0, k = 0;
+    int32_t ma = 0, mi = 0, go = 0, ge = 0;
+    int64_t ld = 0, stride = 0;  // row q at sp[0] + q * stride: H[0..n), F at + ld
+};
+
 struct sw_ctx {
     int device = 0;
     int num_sms = 0;
@@ -198,6 +206,7 @@ struct sw_ctx {
     char errbuf[512] = {0};
     int variant_override = -1;
     int vstripes = 1;           // virtual stripes for the single-process calls
+    S1Rows s1;                  // special rows resident from the last Stage-1 call
     int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
     long long timeout_ns = 120ll * 1000000000ll;
 };
@@ -434,6 +443,12 @@ struct Job {
     void *user;
     bool local;
     int32_t goal;
+    // Stage-2 partition: start-check width, anchor type, matching
+    int hit_w = 0x7fffffff;
+    bool anchor_gap = false;
+    bool match = false;
+    int64_t mjc = 0;
+    const int *mH = nullptr, *mF = nullptr;
     // stripes: either `nv` virtual stripes of [0, n) on this GPU, or (rank mode)
     // one stripe [c_lo, c_hi) whose borders come from / go to other GPUs.
     int nv = 1;
@@ -502,6 +517,7 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
 {
     const auto h0 = std::chrono::steady_clock::now();
+    if (J.local) ctx->s1.valid = false;
     double hck[6] = {0, 0, 0, 0, 0, 0};
     auto hnow = [&]() { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - h0).count(); };
     bool use16 = false;
@@ -673,6 +689,12 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     a.gbest = d_gbest;
     a.slots = (int4 *)ctx->slots.p;
     a.goal = J.goal;
+    a.hit_w = J.hit_w;
+    a.anchor_gap = J.anchor_gap ? 1 : 0;
+    a.match = J.match ? 1 : 0;
+    a.mjc = (int)J.mjc;
+    a.mH = J.mH;
+    a.mF = J.mF;
     a.hit_key = d_hit_key;
     a.hit_band = d_hit_band;
     a.replays = d_replays;
@@ -859,6 +881,14 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     ctx->stats.warps = V.nw;
     ctx->stats.width = W;
     ctx->stats.grid = grid;
+    if (J.local) {
+        // Stage 2 can match against these rows while they stay resident
+        S1Rows &R = ctx->s1;
+        R.valid = NS == 1 && !J.rank_mode;
+        R.m = J.m; R.n = J.n; R.k = J.k;
+        R.ma = J.ma; R.mi = J.mi; R.go = J.go; R.ge = J.ge;
+        R.ld = ld[0]; R.stride = stride[0];
+    }
     return SW_OK;
 }
 
@@ -1135,4 +1165,133 @@ extern "C" int sw_reverse_goal_dev(sw_ctx *ctx, const char *dseqA, int64_t i_end
     if (i_end == 0 || j_end == 0) return SW_ENOTFOUND;
     return reverse_common(ctx, (const unsigned char *)dseqA, i_end, (const unsigned char *)dseqB, j_end, match,
                           mismatch, gap_open, gap_ext, goal, (cudaStream_t)stream, start_out);
+}
+
+// ---------------------------------------------------------------- Stage 2 (N1)
+
+// Stage 2, partial traceback (readings S18-S22):
+// from the end point back to the start point, one partition per special row.
+// Each partition is a reverse GLOBAL fill of the TRANSPOSED problem -- DP
+// rows j' = reversed S1 prefix (original columns j_c - j'), DP columns
+// i' = reversed S0[r+1..i_c] -- so a band is a vertical strip of the original
+// matrix (orthogonal execution) and the special row r is the last DP
+// column, where the capture tiles run the goal-based matching; the band that
+// holds the first event stops the bands after it.
+static int stage2_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const unsigned char *dB, int64_t n,
+                         int32_t ma, int32_t mi, int32_t go, int32_t ge, int64_t k, const sw_result *end,
+                         cudaStream_t us, sw_crosspoint *out, int64_t cap, int64_t *count)
+{
+    const S1Rows &R = ctx->s1;
+    if (!R.valid || R.m != m || R.n != n || R.k != k || R.ma != ma || R.mi != mi || R.go != go || R.ge != ge) {
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf),
+                 "stage 2 needs the special rows of the last single-GPU sw_align_stage1 call with the same m, n, k and scoring");
+        return SW_EINVAL;
+    }
+    cudaStream_t st = us ? us : ctx->stream;
+    const int32_t *sp = (const int32_t *)ctx->sp[0].p;
+    // H, F of special row r at column j (row 0 and column 0: H = 0, F = -inf)
+    auto fetch = [&](int64_t r, int64_t j, long long *h, long long *f) -> int {
+        *h = 0;
+        *f = NEG;
+        if (r == 0 || j == 0) return SW_OK;
+        const int32_t *row = sp + (r / k - 1) * R.stride;
+        CK(cudaMemcpyAsync(ctx->res_h + 3, row + j - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync((int32_t *)(ctx->res_h + 3) + 1, row + R.ld + j - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        *h = ((const int32_t *)(ctx->res_h + 3))[0];
+        *f = ((const int32_t *)(ctx->res_h + 3))[1];
+        return SW_OK;
+    };
+    std::vector<sw_crosspoint> L;
+    sw_crosspoint C{end->i, end->j, end->score, 0};
+    L.push_back(C);
+    int rc;
+    while (!(C.score == 0 && C.type == 0)) {
+        if (C.i <= 0) return SW_ENOTFOUND;
+        const int64_t r = k > 0 ? ((C.i - 1) / k) * k : 0, Lr = C.i - r;
+        sw_crosspoint X{};
+        bool found = false;
+        {
+            // strip j' = 0 is the reverse DP's boundary column: H' = F' = -(G_open + Lr G_ext) at row r
+            long long hs, fs;
+            if ((rc = fetch(r, C.j, &hs, &fs))) return rc;
+            const long long rb = -((long long)go + Lr * (long long)ge);
+            if (hs + rb == C.score) { X = sw_crosspoint{r, C.j, (int32_t)hs, 0}; found = true; }
+            else if (fs > NEG / 2 && fs + rb + go == C.score) { X = sw_crosspoint{r, C.j, (int32_t)fs, 2}; found = true; }
+        }
+        if (!found) {
+            if (C.j == 0) return SW_ENOTFOUND;
+            Job J{};
+            J.dA = dB; J.m = C.j; J.revA = true;      // DP rows: S1[C.j - j'] (0-based)
+            J.dB = dA + r; J.n = Lr; J.revB = true;   // DP columns: S0[C.i - i'] (0-based)
+            J.ma = ma; J.mi = mi; J.go = go; J.ge = ge;
+            J.k = 0; J.sink = nullptr; J.user = nullptr;
+            J.local = false;
+            J.goal = C.score;
+            J.nv = 1;
+            J.epoch = ++ctx->epoch;
+            J.hit_w = (int)(Lr - 1);  // start check strictly below row r
+            J.anchor_gap = C.type == 2;
+            J.match = true;
+            J.mjc = C.j;
+            J.mH = r > 0 ? sp + (r / k - 1) * R.stride : nullptr;
+            J.mF = r > 0 ? J.mH + R.ld : nullptr;
+            int4 res;
+            if ((rc = run_job(ctx, J, us, &res))) return rc;
+            if (!res.w) return SW_ENOTFOUND;
+            const int64_t jp = res.y, col = res.z;
+            if (col <= Lr - 1) {
+                X = sw_crosspoint{C.i - col, C.j - jp, 0, 0};  // the start point
+            } else {
+                long long hs, fs;
+                if ((rc = fetch(r, C.j - jp, &hs, &fs))) return rc;
+                X = col == Lr ? sw_crosspoint{r, C.j - jp, (int32_t)hs, 0} : sw_crosspoint{r, C.j - jp, (int32_t)fs, 2};
+            }
+        }
+        L.push_back(X);
+        C = X;
+    }
+    *count = (int64_t)L.size();
+    for (int64_t q = 0; q < (int64_t)L.size() && q < cap; q++) out[q] = L[L.size() - 1 - q];
+    return cap < (int64_t)L.size() ? SW_ERANGE : SW_OK;
+}
+
+static bool valid_stage2(const sw_ctx *ctx, int64_t m, int64_t n, int64_t k, const sw_result *end,
+                         const sw_crosspoint *out, int64_t cap, const int64_t *count)
+{
+    if (!ctx || !end || !count || m < 0 || n < 0 || k < 0 || cap < 0 || (cap > 0 && !out)) return false;
+    if (end->score < 0 || end->i < 0 || end->j < 0 || end->i > m || end->j > n) return false;
+    return true;
+}
+
+extern "C" int sw_stage2(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, int64_t n, int32_t match,
+                         int32_t mismatch, int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
+                         const sw_result *end, sw_crosspoint *out, int64_t cap, int64_t *count)
+{
+    if (!valid_stage2(ctx, m, n, special_row_interval, end, out, cap, count)) return SW_EINVAL;
+    if ((m && !seqA) || (n && !seqB)) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    if ((rc = upload(ctx, seqA, m, seqB, n))) return rc;
+    rc = stage2_common(ctx, (const unsigned char *)ctx->seq.p, m, (const unsigned char *)ctx->seq.p + m, n, match,
+                       mismatch, gap_open, gap_ext, special_row_interval, end, nullptr, out, cap, count);
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return rc;
+}
+
+extern "C" int sw_stage2_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n, int32_t match,
+                             int32_t mismatch, int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
+                             const sw_result *end, void *stream, sw_crosspoint *out, int64_t cap, int64_t *count)
+{
+    if (!valid_stage2(ctx, m, n, special_row_interval, end, out, cap, count)) return SW_EINVAL;
+    if ((m && !dseqA) || (n && !dseqB)) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    begin_stats(ctx);
+    return stage2_common(ctx, (const unsigned char *)dseqA, m, (const unsigned char *)dseqB, n, match, mismatch,
+                         gap_open, gap_ext, special_row_interval, end, (cudaStream_t)stream, out, cap, count);
 }

@@ -80,6 +80,11 @@ struct FillArgs {
     int *gbest;          // running best-score hint
     int4 *slots;         // per-CTA (score, i, j, 0)
     int goal;            // GLOBAL mode
+    int hit_w;           // GLOBAL: DP columns 1..hit_w may hold a goal hit (start check)
+    int anchor_gap;      // GLOBAL: the anchor is a gap crosspoint: column 0 and the corner diagonal are -inf (S20)
+    int match;           // Stage-2 matching at the last column of a transposed partition
+    int mjc;             // anchor column j_c: DP row j' of the partition is original column j_c - j'
+    const int *mH, *mF;  // special row r's H and F at original columns 1..n (index j - 1); null: row 0 (H 0, F -inf)
     unsigned long long *hit_key;  // min over hits of (i' << 32 | j')
     int *hit_band;       // min band containing a hit
     unsigned long long *replays;
@@ -99,6 +104,7 @@ struct StepInfo {
     long long sp_stride;
     int jcap;            // local column whose (t, E) goes to the right neighbour
     int2 *rbrow;         // right-border destination for this lane's first row
+    int hw;              // columns eligible for tracking (w, or the Stage-2 start-check width)
 };
 
 __device__ __forceinline__ unsigned long long gtimer()
@@ -249,6 +255,29 @@ struct Fill {
         int out_t0, out_f0, out_t1, out_f1;  // (t, F) of the strip's bottom row at the two last columns
     };
 
+    // The stripe's last column: (t, E) to the right neighbour, or, in a
+    // Stage-2 partition (transposed), the goal-based matching
+    // against the special row: DP row `row` is original column
+    // j = j_c - row, t + G_first is the reverse H and E the reverse F at row r.
+    static __device__ __forceinline__ void cap_cell(const FillArgs &a, const StepInfo &X, int row, int r, int t, int e)
+    {
+        if (X.rbrow != nullptr) {
+            X.rbrow[r] = make_int2(t, e);
+        } else if (!LOCAL && a.match && row <= a.m) {
+            const int j = a.mjc - row;
+            const long long hs = (a.mH != nullptr && j > 0) ? (long long)a.mH[j - 1] : 0ll;
+            const long long fs = (a.mH != nullptr && j > 0) ? (long long)a.mF[j - 1] : (long long)NEG;
+            int kind = -1;
+            if (hs + t + a.gf == a.goal) kind = 0;                                            // H junction
+            else if (fs > NEG / 2 && e > NEG / 2 && fs + e + a.go == a.goal) kind = 1;  // gap junction (S18)
+            if (kind >= 0) {
+                // after every start hit of the same row (columns <= w - 1): the sweep order S19
+                atomicMin(a.hit_key, ((unsigned long long)(unsigned)row << 32) | (unsigned)(X.w + kind));
+                atomicMin(a.hit_band, (row - 1) / BH);
+            }
+        }
+    }
+
     // One lane step (warp-synchronous): the lane handles 0-based columns
     // j0 = 2 (k - lane) and j0 + 1.  TRACK: exact best / first-hit tracking.
     // SPM: 0 = no special rows, 1 = special rows are strip-bottom rows,
@@ -309,21 +338,21 @@ struct Fill {
                 }
             }
             if (CAP) {  // the stripe's last column: hand (t, E) to the right neighbour
-                if (j0 == X.jcap) X.rbrow[r] = make_int2(tA, eA);
-                if (j0 + 1 == X.jcap) X.rbrow[r] = make_int2(tB, eB);
+                if (j0 == X.jcap) cap_cell(a, X, row1 + r, r, tA, eA);
+                if (j0 + 1 == X.jcap) cap_cell(a, X, row1 + r, r, tB, eB);
             }
             if (TRACK) {
                 const int row = row1 + r;
                 if (row <= a.m) {
                     const int cA = X.col0 + j0 + 1, cB = cA + 1;  // global DP columns
-                    if (j0 + 1 <= X.w) {
+                    if (j0 + 1 <= X.hw) {
                         if (LOCAL) {
                             if (better(hA, row, cA, bs, bi, bj)) { bs = hA; bi = row; bj = cA; }
                         } else if (hA == a.goal && (row < bi || (row == bi && cA < bj))) {
                             bi = row; bj = cA;
                         }
                     }
-                    if (j0 + 2 <= X.w) {
+                    if (j0 + 2 <= X.hw) {
                         if (LOCAL) {
                             if (better(hB, row, cB, bs, bi, bj)) { bs = hB; bi = row; bj = cB; }
                         } else if (hB == a.goal && (row < bi || (row == bi && cB < bj))) {
@@ -446,7 +475,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
     const uint32_t selr_base = (uint32_t)__cvta_generic_to_shared(selr);
     const StripeArgs &S = a.st[blockIdx.x % a.nstripes];
     const int NT = S.NT;
-    const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr;
+    const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr || (!LOCAL && a.match);
     int bs = 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
     long long nrep = 0;
     if (*a.err) return;
@@ -457,6 +486,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
     X.sp_stride = S.sp_stride;
     X.jcap = S.w - 1;
     X.rbrow = nullptr;
+    X.hw = LOCAL ? S.w : min(S.w, a.hit_w);
     // tiles in which a lane meets the capture column jcap (lane l at step jcap/2 + l)
     const int cap_t0 = (X.jcap >> 1) / STEPS, cap_t1 = ((X.jcap >> 1) + 31) / STEPS;
 
@@ -478,7 +508,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
         int *sp_ptr = nullptr;
         uint32_t smask = 0;
         bool warp_sp = false;
-        X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
+        X.rbrow = S.rb != nullptr ? S.rb + row0 + 1 : nullptr;
         if (warp < NW) {
             const uint32_t w = row0 < a.m ? a.A2[row0 >> 4] : 0u;
             const int sh = (row0 & 15) * 2;
@@ -487,9 +517,10 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                 const uint32_t code = (w >> (sh + 2 * r)) & 3u;
                 L.P[r] = (row0 + r < a.m) ? a.prof[code] : PADPROF;
                 L.e[r] = NEG;
-                L.t[r] = LOCAL ? -a.gf : -(a.go + (row0 + r + 1) * a.ge) - a.gf;  // H(i,0) - G_first
+                // H(i,0) - G_first; -inf when the anchor is a gap crosspoint (S20)
+                L.t[r] = LOCAL ? -a.gf : a.anchor_gap ? NEG : -(a.go + (row0 + r + 1) * a.ge) - a.gf;
             }
-            L.tprev = LOCAL ? -a.gf : (row0 == 0 ? -a.gf : -(a.go + row0 * a.ge) - a.gf);
+            L.tprev = LOCAL ? -a.gf : a.anchor_gap ? NEG : (row0 == 0 ? -a.gf : -(a.go + row0 * a.ge) - a.gf);
             L.out_t0 = L.out_f0 = L.out_t1 = L.out_f1 = 0;
             if (LOCAL && a.k > 0) {
                 // special rows among DP rows row0+1 .. row0+ALPHA (<= m); the band's
@@ -610,7 +641,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                             // this warp's rows are complete at the stripe's last column
                             __threadfence_system();
                             __syncwarp();
-                            if (lane == 0) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
+                            if (lane == 0 && S.rready != nullptr) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
                         }
                     } else if (c < F::GUARD_TILES || (warp_sp && spm == 2)) {
                         tmax = F::template tile<true, false, 2>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, smask);

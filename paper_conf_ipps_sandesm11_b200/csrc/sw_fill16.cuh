@@ -290,6 +290,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
     if (*a.err) return;
     StepInfo X;
     X.w = S.w;
+    X.hw = S.w;
     X.col0 = S.col0;
     X.sp_ld = S.sp_ld;
     X.sp_stride = S.sp_stride;
