@@ -277,15 +277,17 @@ class Context:
         pb, n, kb = _as_bytes_ptr(B)
         e = end if isinstance(end, tuple) else end.astuple()
         r = _Result(e[0], e[1], e[2])
+        # at most one crosspoint per special row, plus the start and end points
         return self._stage2_call(self._lib.sw_stage2, (self._h, pa, m, pb, n, match, mismatch, gap_open, gap_ext, k,
-                                                       ctypes.byref(r)), 64)
+                                                       ctypes.byref(r)), (m // k if k > 0 else 0) + 2)
 
     def stage2_dev(self, dA_ptr, m, dB_ptr, n, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0, end=None,
                    stream: int = 0):
         e = end if isinstance(end, tuple) else end.astuple()
         r = _Result(e[0], e[1], e[2])
         return self._stage2_call(self._lib.sw_stage2_dev, (self._h, dA_ptr, m, dB_ptr, n, match, mismatch, gap_open,
-                                                           gap_ext, k, ctypes.byref(r), stream or None), 64)
+                                                           gap_ext, k, ctypes.byref(r), stream or None),
+                                 (m // k if k > 0 else 0) + 2)
 
     def row_granularity(self) -> int:
         return int(self._lib.sw_row_granularity(self._h))

@@ -190,6 +190,7 @@ struct sw_ctx {
     std::vector<cudaEvent_t> ev_row;  // one per staging slot: the slot's final copy is done
     int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
+    DevBuf capbuf;  // Stage 2: (t, E) of every DP row at the special row's column
     DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
     HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
     HostBuf colp[MAX_STRIPES];   // mapped pinned per-band final-column counts per stripe
@@ -332,7 +333,7 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->side) cudaStreamSynchronize(ctx->side);
-    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg})
+    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg, &ctx->capbuf})
         if (b->p) cudaFree(b->p);
     for (int s = 0; s < MAX_STRIPES; s++) {
         for (DevBuf *b : {&ctx->rowb[s], &ctx->progress[s], &ctx->sp[s]})
@@ -551,6 +552,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     if ((rc = grow(ctx, ctx->a2, wa * 4))) return rc;
     if ((rc = grow(ctx, ctx->b2, wb * 4))) return rc;
     if ((rc = grow(ctx, ctx->misc, 256))) return rc;
+    if (J.match && (rc = grow(ctx, ctx->capbuf, ((size_t)nb * BH + 2) * sizeof(int2)))) return rc;
     const size_t border_rows = (size_t)nb * BH + 2;
     const size_t border_flags = (size_t)nb * V.nw + 1;
     for (int s = 0; s < NS; s++) {
@@ -740,6 +742,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             S.lready = s > 0 ? ctx->vrecv[s].lready() : nullptr;
             S.rb = s + 1 < NS ? ctx->vrecv[s + 1].lb() : nullptr;
             S.rready = s + 1 < NS ? ctx->vrecv[s + 1].lready() : nullptr;
+            if (J.match) {  // Stage 2: capture the last column for the band-end matching
+                S.rb = (int2 *)ctx->capbuf.p;
+                S.rready = nullptr;
+            }
         }
     }
     {
@@ -1237,7 +1243,14 @@ static int stage2_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const 
             J.mH = r > 0 ? sp + (r / k - 1) * R.stride : nullptr;
             J.mF = r > 0 ? J.mH + R.ld : nullptr;
             int4 res;
+            const auto tj = std::chrono::steady_clock::now();
+            const double f0 = ctx->stats.fill_ms;
             if ((rc = run_job(ctx, J, us, &res))) return rc;
+            if (getenv("SWB_DEBUG_HOST"))
+                fprintf(stderr, "[swb stage2] partition rows %lld..%lld jc %lld: run_job %.2f ms (fill %.2f ms) event (%d, %d)\n",
+                        (long long)r, (long long)C.i, (long long)C.j,
+                        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tj).count(),
+                        ctx->stats.fill_ms - f0, res.y, res.z);
             if (!res.w) return SW_ENOTFOUND;
             const int64_t jp = res.y, col = res.z;
             if (col <= Lr - 1) {

@@ -255,29 +255,6 @@ struct Fill {
         int out_t0, out_f0, out_t1, out_f1;  // (t, F) of the strip's bottom row at the two last columns
     };
 
-    // The stripe's last column: (t, E) to the right neighbour, or, in a
-    // Stage-2 partition (transposed), the goal-based matching
-    // against the special row: DP row `row` is original column
-    // j = j_c - row, t + G_first is the reverse H and E the reverse F at row r.
-    static __device__ __forceinline__ void cap_cell(const FillArgs &a, const StepInfo &X, int row, int r, int t, int e)
-    {
-        if (X.rbrow != nullptr) {
-            X.rbrow[r] = make_int2(t, e);
-        } else if (!LOCAL && a.match && row <= a.m) {
-            const int j = a.mjc - row;
-            const long long hs = (a.mH != nullptr && j > 0) ? (long long)a.mH[j - 1] : 0ll;
-            const long long fs = (a.mH != nullptr && j > 0) ? (long long)a.mF[j - 1] : (long long)NEG;
-            int kind = -1;
-            if (hs + t + a.gf == a.goal) kind = 0;                                            // H junction
-            else if (fs > NEG / 2 && e > NEG / 2 && fs + e + a.go == a.goal) kind = 1;  // gap junction (S18)
-            if (kind >= 0) {
-                // after every start hit of the same row (columns <= w - 1): the sweep order S19
-                atomicMin(a.hit_key, ((unsigned long long)(unsigned)row << 32) | (unsigned)(X.w + kind));
-                atomicMin(a.hit_band, (row - 1) / BH);
-            }
-        }
-    }
-
     // One lane step (warp-synchronous): the lane handles 0-based columns
     // j0 = 2 (k - lane) and j0 + 1.  TRACK: exact best / first-hit tracking.
     // SPM: 0 = no special rows, 1 = special rows are strip-bottom rows,
@@ -338,8 +315,8 @@ struct Fill {
                 }
             }
             if (CAP) {  // the stripe's last column: hand (t, E) to the right neighbour
-                if (j0 == X.jcap) cap_cell(a, X, row1 + r, r, tA, eA);
-                if (j0 + 1 == X.jcap) cap_cell(a, X, row1 + r, r, tB, eB);
+                if (j0 == X.jcap) X.rbrow[r] = make_int2(tA, eA);
+                if (j0 + 1 == X.jcap) X.rbrow[r] = make_int2(tB, eB);
             }
             if (TRACK) {
                 const int row = row1 + r;
@@ -475,7 +452,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
     const uint32_t selr_base = (uint32_t)__cvta_generic_to_shared(selr);
     const StripeArgs &S = a.st[blockIdx.x % a.nstripes];
     const int NT = S.NT;
-    const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr || (!LOCAL && a.match);
+    const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr;
     int bs = 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
     long long nrep = 0;
     if (*a.err) return;
@@ -544,10 +521,17 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             if (b > 0) {
                 if (lane == 0) {
                     const unsigned long long t0 = gtimer();
+                    unsigned long long spins = 0;
                     while (ld_acquire(S.progress + b - 1) < need) {
                         if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
                         if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                         __nanosleep(64);
+                        spins++;
+                    }
+                    if (a.dbg && S.col0 == 0 && spins) {  // debug: total wait ns, spin loops, waits
+                        a.dbg[80 * b + 5] += gtimer() - t0;
+                        a.dbg[80 * b + 6] += spins;
+                        a.dbg[80 * b + 7] += 1;
                     }
                 }
                 __syncwarp();
@@ -622,6 +606,8 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
         const int S_END = NT + LAG * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s <= S_END; ++s) {
+            if (a.dbg && threadIdx.x == 0 && S.col0 == 0 && (s == NT / 4 || s == NT / 2 || s == 3 * NT / 4))
+                a.dbg[80 * b + 2 + (s == NT / 2) + 2 * (s == 3 * NT / 4)] = gtimer();
             if (warp < NW) {
                 const int c = s - LAG * warp;
                 if (c >= 0 && c < NT) {
@@ -674,6 +660,32 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             if (s_abort) break;
         }
         if (warp == NW && lane == 0 && !s_abort) st_release(S.progress + b, INT_MAX);
+        if (!LOCAL && a.match && !s_abort) {
+            // Stage-2 goal-based matching: the
+            // capture tiles left (t, E) of the special row's DP column for
+            // every row of the band in S.rb; row j' is original column
+            // j = j_c - j', t + G_first the reverse H there, E the reverse F.
+            // Coalesced, once per band (per-lane matching inside the capture
+            // tiles stalled each warp on dependent global loads).
+            __syncthreads();
+            unsigned long long key = ~0ull;
+            const int hi = min((b + 1) * BH, a.m);
+            for (int row = b * BH + 1 + (int)threadIdx.x; row <= hi; row += (int)blockDim.x) {
+                const int2 v = __ldcg(S.rb + row);
+                const int j = a.mjc - row;
+                const long long hs = (a.mH != nullptr && j > 0) ? (long long)__ldg(a.mH + j - 1) : 0ll;
+                const long long fs = (a.mH != nullptr && j > 0) ? (long long)__ldg(a.mF + j - 1) : (long long)NEG;
+                int kind = -1;
+                if (hs + v.x + a.gf == a.goal) kind = 0;                                          // H junction
+                else if (fs > NEG / 2 && v.y > NEG / 2 && fs + v.y + a.go == a.goal) kind = 1;  // gap junction (S18)
+                // after every start hit of the same row (DP columns <= w - 1): the sweep order S19
+                if (kind >= 0) key = min(key, ((unsigned long long)(unsigned)row << 32) | (unsigned)(S.w + kind));
+            }
+            if (key != ~0ull) {
+                atomicMin(a.hit_key, key);
+                atomicMin(a.hit_band, b);
+            }
+        }
         if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 15] = gtimer();
         if (LOCAL && a.k > 0) {
             // publish this band's special rows (this stripe's slice) to the host
