@@ -53,92 +53,109 @@ struct Fill16 {
     static constexpr int SKEW = 63;     // lane 31's output column lags lane 0's by 2*31 + 1
     static constexpr int STEPS = W;     // one column per lane step
     static constexpr int NSAVE = 20;
+    static constexpr int HALF = SRING / 2 + 32;  // selector ring: one parity half + a 32-entry mirror
+    // Warp-to-warp rings of (t, F): column col lives at ridx(col) in [1, RING]
+    // (stride RS = RING + 1), so the 64 columns k0 - 63 .. k0 a lane-31 tile
+    // writes (k0 a multiple of 64) sit at consecutive indices from
+    // ((k0 - 64) & (RING - 1)) + 1: immediate offsets, no wrap.
+    static constexpr int RS = RING + 1;
+    static __device__ __forceinline__ int ridx(int col) { return ((col - 1) & (RING - 1)) + 1; }
     static_assert(W % 64 == 0 && W > SKEW, "W multiple of 64, larger than the warp skew");
+    static_assert(W == 64, "the converted-ring and selector addressing assume 64-column tiles");
 
+    // rings (int2, (NW+1) x RS) | selectors (2 x HALF u32) | converted ring (NW x W u32) | saves
     static size_t smem_bytes()
     {
-        return sizeof(int2) * RING * (NW + 1) + sizeof(uint32_t) * SRING + sizeof(int) * NSAVE * 32 * NW;
+        return sizeof(int2) * RS * (NW + 1) + sizeof(uint32_t) * 2 * HALF + sizeof(uint32_t) * NW * W +
+               sizeof(int) * NSAVE * 32 * NW;
     }
 
     struct Lane {
         uint32_t P[8], Q[8];  // int8x4 profiles of rows s (low halves) and s+8 (high halves)
         uint32_t e[8], t[8];  // packed E and t = H - G_first of the previous column of each half
         uint32_t tprev;       // packed diagonal input of slot 0
-        uint32_t f7;          // packed F of slot 7 after the last step (row 15 in the high half)
-        uint32_t selhi;       // high-half selector part of the previous column
+        uint32_t fn;          // packed F of the rows after slot 7 (low: row 8 at j, high: row 16 at j-1)
         int B;                // warp-uniform frame base
         int adj;              // BIAS16 - B: int32 value -> frame
+        int Bm;               // B - BIAS16: frame -> int32 value
         uint32_t FL;          // packed frame image of the local floor 0
     };
 
     // Selector ring layout: even columns in the first half, odd in the second,
     // so the 32 lanes of a step (columns k - 2 lane, all of one parity) read
-    // 32 consecutive words: no bank conflicts.
-    static __device__ __forceinline__ uint32_t sel_index(int col)
+    // 32 consecutive words: no bank conflicts.  Each half has a 32-word mirror
+    // of its first 32 words, so a lane's 64 steps of a tile read
+    // base + (kk >> 1) + (kk & 1) * HALF without wrapping (immediate offsets).
+    // The word of column c is the complete PRMT selector of a lane step whose
+    // low half is at c and high half at c - 1.
+    static __device__ __forceinline__ void put_sel(uint32_t *selr, int col, uint32_t code, uint32_t code_left)
     {
-        const uint32_t c = (uint32_t)col & (SRING - 1);
-        return (c >> 1) + (c & 1u) * (SRING / 2);
+        const uint32_t c = (uint32_t)col & (SRING - 1), h = c >> 1, par = c & 1u;
+        const uint32_t v = (col_sel16(code) & 0xffu) | (col_sel16(code_left) & 0xff00u);
+        selr[par * HALF + h] = v;
+        if (h < 32) selr[par * HALF + h + SRING / 2] = v;
     }
 
-    static __device__ __forceinline__ int toabs(const Lane &L, int q) { return q - BIAS16 + L.B; }
+    static __device__ __forceinline__ int toabs(const Lane &L, int q) { return q + L.Bm; }
     static __device__ __forceinline__ int tofr(const Lane &L, int x) { return x - L.B + BIAS16; }
 
     // One lane step: low half at local column jl = k - 2 lane, high half at jl - 1.
+    //
+    // Cell update, with D = max(H_diag + p, E, 0) (so H = max(D, F), Eq. 1):
+    //   E*  = max(E*_left - G_ext, t_left, 0)     Eq. 2, floored at 0 (below)
+    //   D   = max(t_diag + (p + G_first), E*)
+    //   H   = max(D, F);  t = H - G_first
+    //   F'  = max(F - G_ext, D - G_first)         Eq. 3 for the next row
+    // F' = max(F - G_ext, t) = max(F - G_ext, D - G_first, F - G_first) and
+    // G_ext <= G_first, so the F chain down the lane's rows is one max per row
+    // and D (which only needs the previous column) is off that chain.
+    // Flooring E at 0 is exact for H and F: max(E, 0) satisfies the same
+    // recurrence (max(max(E,0) - G_ext, t, 0) = max(E - G_ext, t, 0)), and H
+    // takes max(.., E, .., 0) anyway.  E only leaves the lane as a stripe's
+    // right border, where the receiver's H and F are unchanged by the floor.
     template <bool GUARD, bool TRACK, bool SP1, bool CAP>
     static __device__ __forceinline__ uint32_t step(const FillArgs &a, const StepInfo &X, Lane &L, int k, int lane,
-                                                    uint32_t ring_in, uint32_t ring_out, uint32_t selr, uint32_t tmax,
-                                                    int row1, int &bs, int &bi, int &bj, int *sp_ptr)
+                                                    uint32_t cr_a, uint32_t ro_a, uint32_t sel_a, uint32_t pt_sel,
+                                                    int one, uint32_t tmax, int row1, int &bs, int &bi, int &bj,
+                                                    int *sp_ptr)
     {
-        uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[7], 1);
-        uint32_t up_f = __shfl_up_sync(0xffffffffu, L.f7, 1);
+        const uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[7], 1);
+        const uint32_t up_f = __shfl_up_sync(0xffffffffu, L.fn, 1);
         const int jl = k - 2 * lane;
-        {
-            // lane 0: the warp above's bottom row (int32) from the ring, into this
-            // warp's frame; F_in only enters as max(F_in - G_ext, t_in), so
-            // clamping it to >= t_in is exact.  Predicated, not branched.
-            int vx, vy;
-            asm volatile("{\n\t.reg .pred p;\n\t"
-                         "setp.eq.s32 p, %2, 0;\n\t"
-                         "@p ld.shared.v2.s32 {%0, %1}, [%3];\n\t}"
-                         : "=r"(vx), "=r"(vy)
-                         : "r"(lane), "r"(ring_in + (uint32_t)(jl & (RING - 1)) * 8u)
-                         : "memory");
-            if (lane == 0) {
-                up_t = (uint32_t)(vx + L.adj) << 16;
-                up_f = (uint32_t)(max(vy, vx) + L.adj) << 16;
-            }
-        }
+        // lane 0: the warp above's bottom row at column jl, already in this warp's
+        // frame (converted at tile start): low half t, high half F of row 0.
+        uint32_t cr, sel;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(cr) : "r"(cr_a) : "memory");
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(sel) : "r"(sel_a) : "memory");
         Lane S;
         if (GUARD) S = L;
         const uint32_t tmax_in = tmax;
-        // slot-0 inputs: low = upper lane's row 15 (its high half), high = own row 7 (low half of slot 7)
-        uint32_t tu = __byte_perm(up_t, L.t[7], 0x5432);
-        uint32_t fu = __byte_perm(up_f, L.f7, 0x5432);
+        // slot-0 inputs: low = upper lane's row 15 (its high half) or the ring, high = own row 7
+        uint32_t tu = __byte_perm(lane == 0 ? cr : up_t, L.t[7], pt_sel);
+        uint32_t fu = __byte_perm(lane == 0 ? cr : up_f, L.fn, 0x5432);  // F of slot 0's rows
         uint32_t td = L.tprev;
         L.tprev = tu;
-        uint32_t sw;
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(sw) : "r"(selr + sel_index(jl) * 4u) : "memory");
-        const uint32_t sel = (sw & 0xffu) | L.selhi;
-        L.selhi = sw & 0xff00u;  // nibbles 2,3 (bytes 2,3 of the result) for the next column
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
+        uint32_t f15 = 0;  // F entering slot 7 (row 15 in the high half)
 #pragma unroll
         for (int s = 0; s < 8; s += 2) {
-            const uint32_t e0 = __vmaxu2((uint32_t)imad((int)L.e[s], a.one, nge2), L.t[s]);
-            fu = __vmaxu2((uint32_t)imad((int)fu, a.one, nge2), tu);
+            const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
             const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
-            const uint32_t h0 = __viaddmax_u16x2(td, p0, __vimax3_u16x2(e0, fu, L.FL));
+            const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
+            const uint32_t h0 = __vmaxu2(d0, fu);
             td = L.t[s];
-            const uint32_t t0 = (uint32_t)imad((int)h0, a.one, ngf2);
-            tu = t0;
+            const uint32_t t0 = (uint32_t)imad((int)h0, one, ngf2);
+            fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d0, one, ngf2));
             L.e[s] = e0;
             L.t[s] = t0;
-            const uint32_t e1 = __vmaxu2((uint32_t)imad((int)L.e[s + 1], a.one, nge2), L.t[s + 1]);
-            fu = __vmaxu2((uint32_t)imad((int)fu, a.one, nge2), tu);
+            if (s == 6) f15 = fu;
+            const uint32_t e1 = __vimax3_u16x2((uint32_t)imad((int)L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
             const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
-            const uint32_t h1 = __viaddmax_u16x2(td, p1, __vimax3_u16x2(e1, fu, L.FL));
+            const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
+            const uint32_t h1 = __vmaxu2(d1, fu);
             td = L.t[s + 1];
-            const uint32_t t1 = (uint32_t)imad((int)h1, a.one, ngf2);
-            tu = t1;
+            const uint32_t t1 = (uint32_t)imad((int)h1, one, ngf2);
+            fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d1, one, ngf2));
             L.e[s + 1] = e1;
             L.t[s + 1] = t1;
             tmax = __vimax3_u16x2(tmax, h0, h1);
@@ -168,7 +185,7 @@ struct Fill16 {
                 }
             }
         }
-        L.f7 = fu;
+        L.fn = fu;
         if (GUARD) {
             // lanes left of column 0 keep their state; at jl == 0 only the high half waits
             const uint32_t keep = (jl >= 0 ? 0x0000ffffu : 0u) | (jl >= 1 ? 0xffff0000u : 0u);
@@ -179,41 +196,70 @@ struct Fill16 {
             }
             if (jl < 0) {
                 L.tprev = S.tprev;
-                L.f7 = S.f7;
-                L.selhi = S.selhi;
+                L.fn = S.fn;
             }
             tmax = (tmax & keep) | (tmax_in & ~keep);
         }
         const int jo = jl - 1;  // row 15's column (high half of slot 7)
         if (SP1 && sp_ptr != nullptr && jo >= 0 && jo < X.w) {
             sp_ptr[jo] = toabs(L, hi16(L.t[7])) + a.gf;  // H = t + G_first
-            sp_ptr[X.sp_ld + jo] = toabs(L, hi16(L.f7));
+            sp_ptr[X.sp_ld + jo] = toabs(L, hi16(f15));
         }
         if (!TRACK && lane == 31 && (!GUARD || jo >= 0)) {
             // (t, F) of row 15 at column jo for the next warp (int32, absolute)
-            asm volatile("st.shared.v2.s32 [%0], {%1, %2};" ::"r"(ring_out + (uint32_t)(jo & (RING - 1)) * 8u),
-                         "r"(toabs(L, hi16(L.t[7]))), "r"(toabs(L, hi16(L.f7))) : "memory");
+            asm volatile("st.shared.v2.s32 [%0], {%1, %2};" ::"r"(ro_a),
+                         "r"(toabs(L, hi16(L.t[7]))), "r"(toabs(L, hi16(f15))) : "memory");
         }
         return tmax;
     }
 
+    // Lane 0's ring input of this tile, converted once into the warp's frame:
+    // cring[x] = t | F' << 16 for column c*W + x, F' = max(F - G_ext, t) the F of
+    // the warp's first row.  Warp w-1 finished these columns LAG tiles ago.
+    static __device__ __forceinline__ void convert_ring(const FillArgs &a, const Lane &L, const int2 *ring_in,
+                                                        uint32_t *cring, int c, int lane)
+    {
+#pragma unroll
+        for (int x = lane; x < W; x += 32) {
+            const int2 v = ring_in[ridx(c * W + x)];
+            cring[x] = (uint32_t)((v.x + L.adj) & 0xffff) | ((uint32_t)(max(v.y - a.ge, v.x) + L.adj) << 16);
+        }
+        __syncwarp();
+    }
+
     template <bool GUARD, bool TRACK, bool SP1, bool CAP>
     static __device__ __forceinline__ uint32_t tile(const FillArgs &a, const StepInfo &X, Lane &L, int c, int lane,
-                                                    uint32_t ring_in, uint32_t ring_out, uint32_t selr, int row1,
+                                                    uint32_t cring, uint32_t ring_out, uint32_t selr, int row1,
                                                     int &bs, int &bi, int &bj, int *sp_ptr)
     {
         uint32_t tmax = 0;
         const int k0 = c * STEPS;
+        const uint32_t pt_sel = lane == 0 ? 0x5410u : 0x5432u;
+        const int one = (int)pin((uint32_t)a.one);
+        // this lane's selector words: column k0 + kk - 2 lane
+        const uint32_t sel0 = selr + 4u * ((((uint32_t)(k0 - 2 * lane)) & (SRING - 1)) >> 1);
+        // lane 31's ring output: column k0 + kk - 63 at ridx = base + kk
+        const uint32_t ro0 = ring_out + 8u * (uint32_t)(((k0 - 64) & (RING - 1)) + 1);
         if (GUARD || TRACK || CAP) {
 #pragma unroll 1
             for (int kk = 0; kk < STEPS; kk++)
-                tmax = step<GUARD, TRACK, SP1, CAP>(a, X, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1, bs,
-                                                   bi, bj, sp_ptr);
+                tmax = step<GUARD, TRACK, SP1, CAP>(a, X, L, k0 + kk, lane, cring + 4u * kk, ro0 + 8u * kk,
+                                                    sel0 + 4u * ((kk >> 1) + (kk & 1) * HALF), pt_sel, one, tmax,
+                                                    row1, bs, bi, bj, sp_ptr);
         } else {
-#pragma unroll 4
-            for (int kk = 0; kk < STEPS; kk++)
-                tmax = step<false, false, SP1, false>(a, X, L, k0 + kk, lane, ring_in, ring_out, selr, tmax, row1,
-                                                      bs, bi, bj, sp_ptr);
+#pragma unroll 1
+            for (int kq = 0; kq < STEPS; kq += 4) {
+                const uint32_t sq = sel0 + 2u * kq, cq = cring + 4u * kq, oq = ro0 + 8u * kq;
+                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq, lane, cq, oq, sq, pt_sel, one, tmax,
+                                                      row1, bs, bi, bj, sp_ptr);
+                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + 1, lane, cq + 4u, oq + 8u, sq + 4u * HALF,
+                                                      pt_sel, one, tmax, row1, bs, bi, bj, sp_ptr);
+                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + 2, lane, cq + 8u, oq + 16u, sq + 4u,
+                                                      pt_sel, one, tmax, row1, bs, bi, bj, sp_ptr);
+                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + 3, lane, cq + 12u, oq + 24u,
+                                                      sq + 4u + 4u * HALF, pt_sel, one, tmax, row1, bs, bi, bj,
+                                                      sp_ptr);
+            }
         }
         return tmax;
     }
@@ -229,9 +275,10 @@ struct Fill16 {
             L.t[s] = (uint32_t)imad((int)L.t[s], a.one, d2);
         }
         L.tprev = (uint32_t)imad((int)L.tprev, a.one, d2);
-        L.f7 = (uint32_t)imad((int)L.f7, a.one, d2);
+        L.fn = (uint32_t)imad((int)L.fn, a.one, d2);
         L.B += d;
         L.adj = BIAS16 - L.B;
+        L.Bm = L.B - BIAS16;
         const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
         L.FL = (uint32_t)fl * 0x10001u;
     }
@@ -244,8 +291,7 @@ struct Fill16 {
             sv[(8 + s) * 32 + lane] = (int)L.t[s];
         }
         sv[16 * 32 + lane] = (int)L.tprev;
-        sv[17 * 32 + lane] = (int)L.f7;
-        sv[18 * 32 + lane] = (int)L.selhi;
+        sv[17 * 32 + lane] = (int)L.fn;
         sv[19 * 32 + lane] = L.B;
     }
     static __device__ __forceinline__ void restore(Lane &L, const int *sv, int lane)
@@ -256,10 +302,10 @@ struct Fill16 {
             L.t[s] = (uint32_t)sv[(8 + s) * 32 + lane];
         }
         L.tprev = (uint32_t)sv[16 * 32 + lane];
-        L.f7 = (uint32_t)sv[17 * 32 + lane];
-        L.selhi = (uint32_t)sv[18 * 32 + lane];
+        L.fn = (uint32_t)sv[17 * 32 + lane];
         L.B = sv[19 * 32 + lane];
         L.adj = BIAS16 - L.B;
+        L.Bm = L.B - BIAS16;
         const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
         L.FL = (uint32_t)fl * 0x10001u;
     }
@@ -273,17 +319,23 @@ template <int NW, int W, bool COOP = false>
 __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
 {
     using F = Fill16<NW, W>;
-    constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
+    constexpr int BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int2 *rings = reinterpret_cast<int2 *>(smem_raw);
-    uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * RING);
-    int *saves = reinterpret_cast<int *>(selr + SRING);
+    uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * F::RS);
+    uint32_t *crings = selr + 2 * F::HALF;
+    int *saves = reinterpret_cast<int *>(crings + NW * W);
     __shared__ int s_band, s_abort;
 
     const int warp = threadIdx.x >> 5, lane = lane_id();
     const uint32_t selr_base = (uint32_t)__cvta_generic_to_shared(selr);
     const StripeArgs &S = a.st[blockIdx.x % a.nstripes];
     const int NT = S.NT;
+    auto code_at = [&](int col) -> uint32_t {  // 2-bit code of local column col; pad and col < 0: 0
+        if (col < 0 || col >= S.w) return 0u;
+        const int gc = S.col0 + col;
+        return (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
+    };
     const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr;
     int bs = 0, bi = 0, bj = 0;
     long long nrep = 0;
@@ -334,13 +386,14 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             else tp = -a.gf;
             L.B = __shfl_sync(0xffffffffu, tv[0], 0);
             L.adj = BIAS16 - L.B;
+            L.Bm = L.B - BIAS16;
 #pragma unroll
             for (int s = 0; s < 8; s++) {
                 L.e[s] = pk(F::tofr(L, ev[s]), F::tofr(L, ev[s + 8]));
                 L.t[s] = pk(F::tofr(L, tv[s]), F::tofr(L, tv[s + 8]));
             }
             L.tprev = pk(F::tofr(L, tp), F::tofr(L, tp));
-            L.f7 = L.t[7];
+            L.fn = L.t[7];  // only feeds the high half at column -1 (kept by GUARD)
             const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
             L.FL = (uint32_t)fl * 0x10001u;
         };
@@ -351,7 +404,6 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 L.P[s] = (row0 + s < a.m) ? a.prof[(w >> (2 * s)) & 3u] : PADPROF;
                 L.Q[s] = (row0 + s + 8 < a.m) ? a.prof[(w >> (2 * (s + 8))) & 3u] : PADPROF;
             }
-            L.selhi = 0;
             init_state(false);
             if (a.k > 0) {
                 // special rows are strip-bottom rows (k a multiple of 16): row0 + 16
@@ -377,13 +429,9 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = c * W + x;
-                rings[col & (RING - 1)] = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
-                uint32_t code = 0u;  // pad columns: code 0 (harmless, see header)
-                if (col < S.w) {
-                    const int gc = S.col0 + col;
-                    code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
-                }
-                selr[F::sel_index(col)] = col_sel16(code);
+                rings[F::ridx(col)] = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
+                // pad columns: code 0 (harmless, see header)
+                F::put_sel(selr, col, code_at(col), code_at(col - 1));
             }
         };
         int *io_sp = nullptr;
@@ -393,12 +441,12 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         }
         unsigned int *const colp = band_has_special(b, BH, a.m, a.k) ? S.colp : nullptr;
         auto io_drain = [&](int cd) {
-            const int2 *ringN = rings + NW * RING;
+            const int2 *ringN = rings + NW * F::RS;
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = cd * W - SKEW + x;
                 if (col >= 0) {
-                    const int2 v = ringN[col & (RING - 1)];
+                    const int2 v = ringN[F::ridx(col)];
                     __stcg(S.rowb + col, v);
                     if (io_sp != nullptr && col < S.w) {
                         __stcg(io_sp + col, v.x + a.gf);  // H = t + G_first
@@ -442,21 +490,17 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         auto coop_fetch = [&](int c, int2 &v, uint32_t &code) {  // issue the loads (results used after compute)
             const int col = c * W + warp * CPW + lane;
             v = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
-            code = 0u;
-            if (col < S.w) {
-                const int gc = S.col0 + col;
-                code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
-            }
+            code = code_at(col) | (code_at(col - 1) << 2);
         };
         auto coop_put = [&](int c, int2 v, uint32_t code) {
             const int col = c * W + warp * CPW + lane;
-            rings[col & (RING - 1)] = v;
-            selr[F::sel_index(col)] = col_sel16(code);
+            rings[F::ridx(col)] = v;
+            F::put_sel(selr, col, code & 3u, code >> 2);
         };
         auto coop_drain = [&](int cd) {
             const int col = cd * W - SKEW + warp * CPW + lane;
             if (col >= 0) {
-                const int2 v = rings[NW * RING + (col & (RING - 1))];
+                const int2 v = rings[NW * F::RS + F::ridx(col)];
                 __stcg(S.rowb + col, v);
                 if (io_sp != nullptr && col < S.w) {
                     __stcg(io_sp + col, v.x + a.gf);
@@ -492,14 +536,15 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             if (warp < NW) {
                 const int c = s - 2 * warp;
                 if (c >= 0 && c < NT) {
-                    const uint32_t rin = pin((uint32_t)__cvta_generic_to_shared(rings + warp * RING));
-                    const uint32_t rout = pin((uint32_t)__cvta_generic_to_shared(rings + (warp + 1) * RING));
+                    const uint32_t rin = pin((uint32_t)__cvta_generic_to_shared(crings + warp * W));
+                    const uint32_t rout = pin((uint32_t)__cvta_generic_to_shared(rings + (warp + 1) * F::RS));
                     const uint32_t selr_s = pin(selr_base);
                     if (c == 0 && has_left) {
                         wait_left();
                         init_state(true);
                     }
                     if (c > 0) F::rebase(a, L);
+                    F::convert_ring(a, L, rings + warp * F::RS, crings + warp * W, c, lane);
                     const int thr = max(max(bs, ld_relaxed(a.gbest)), 1);
                     F::save(L, sv, lane);
                     uint32_t tm;
