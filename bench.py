@@ -355,7 +355,8 @@ def main():
     traffic = None
     try:
         for tr in json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))):
-            if tr.get("workload") == cfg.name and tr.get("kernel_dtype") == kdtype and world == 1:
+            if (tr.get("workload") == cfg.name and tr.get("kernel_dtype") == kdtype and world == 1
+                    and tr.get("alpha", abs(s1["alpha"])) == abs(s1["alpha"]) and tr.get("warps", s1["warps"]) == s1["warps"]):
                 traffic = tr.get("fill_dram_bytes_per_launch")
     except Exception:
         pass

@@ -109,20 +109,31 @@ struct Variant {
     int skew_tiles;         // int32 kernel: tiles past the last column lane 31 needs (ceil(62 / W))
 };
 
-template <int ALPHA, int NW, int W>
+template <int ALPHA, int NW, int W, bool COOP = false>
 static Variant make_variant()
 {
     Variant v;
     v.alpha = ALPHA;
     v.nw = NW;
     v.w = W;
-    v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
-    v.global_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, false>;
-    v.smem = Fill<ALPHA, NW, W, true>::smem_bytes();
+    v.local_fn = v.global_fn = nullptr;
+    v.smem = 0;
     v.packed_fn = nullptr;
     v.smem16 = 0;
     v.io_warps = 1;
-    v.skew_tiles = (Fill<ALPHA, NW, W, true>::SKEW + W - 1) / W;
+    v.skew_tiles = 1;
+    if constexpr (ALPHA == 32) {
+        // packed kernel only (16 slots per lane); int32 work falls back to the default geometry
+        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, 16>;
+        v.io_warps = COOP ? 0 : 1;
+        v.smem16 = Fill16<NW, W, 16>::smem_bytes();
+        return v;
+    } else {
+        v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
+        v.global_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, false>;
+        v.smem = Fill<ALPHA, NW, W, true>::smem_bytes();
+        v.skew_tiles = (Fill<ALPHA, NW, W, true>::SKEW + W - 1) / W;
+    }
     if constexpr (ALPHA == 16 && W % 64 == 0) {
         if constexpr (NW == 16) {
             v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, true>;
@@ -136,7 +147,8 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 8;
+static constexpr int NVARIANTS = 12;
+static constexpr int NINT32_VARIANTS = 8;  // variants 0..7 have int32 kernels; 8.. are packed-only (alpha 32)
 
 static const Variant &variant_for(int idx)
 {
@@ -149,6 +161,10 @@ static const Variant &variant_for(int idx)
         make_variant<16, 15, 64>(),
         make_variant<16, 16, 64>(),
         make_variant<16, 8, 32>(),
+        make_variant<32, 4, 64>(),
+        make_variant<32, 4, 64, true>(),
+        make_variant<32, 8, 64>(),
+        make_variant<32, 16, 64, true>(),
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -312,8 +328,8 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
         if ((e = cudaHostAlloc(&ctx->res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
         for (int i = 0; i < NVARIANTS; i++) {
             const Variant &v = variant_for(i);
-            cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
-            cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+            if (v.local_fn) cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+            if (v.global_fn) cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
             if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaFuncSetAttribute"); break; }
@@ -355,15 +371,18 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     delete ctx;
 }
 
+// The geometry int32 work (reverse pass, Stage 2) runs with: the override when
+// it has an int32 kernel, else the default.
 static const Variant &ctx_variant(const sw_ctx *ctx)
 {
-    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT);
+    const int v = ctx->variant_override;
+    return variant_for(v >= 0 && v < NINT32_VARIANTS ? v : DEFAULT_VARIANT);
 }
 
 extern "C" int64_t sw_row_granularity(const sw_ctx *ctx)
 {
     if (!ctx) return 0;
-    return ctx_variant(ctx).alpha;
+    return variant_for(ctx->variant_override >= 0 ? ctx->variant_override : DEFAULT_VARIANT).alpha;
 }
 
 extern "C" int64_t sw_band_height(const sw_ctx *ctx)
@@ -460,42 +479,65 @@ struct Job {
 }  // namespace
 
 // Kernel choice per call: a small cost model over candidate
-// (kernel, geometry) pairs.  A band takes a CTA one sweep; with P resident
-// CTAs the fill takes ceil(nb / P) sweeps of time ~ BH * P / rate, where
-// `rate` is the measured steady-state GCUPS of the candidate (R10Mx1M, one
-// B200, profiles/r01_variants.txt).  Deterministic in (m, n, k, scoring), so
-// all ranks of a stripe group agree.
+// (kernel, geometry) pairs -- the band pipeline recurrence below with each
+// candidate's measured column speed per CTA (one B200,
+// profiles/r01_variants.txt).  Deterministic in (m, n, k, scoring), so all
+// ranks of a stripe group agree.
 struct Candidate {
     int variant;
     bool packed;
-    double rate;
+    double cps_full;  // columns/s one CTA sweeps with every resident CTA busy (R10M x 1M, one B200)
+    double cps_solo;  // columns/s of a CTA alone on its SM (C2: 133 bands on 148 SMs)
 };
+
+// Modelled fill time of a candidate: band b starts when its CTA is free and
+// band b-1 is `lag` columns ahead,
+//   start(b) = max(start(b - P) + n / cps, start(b - 1) + lag / cps),
+//   T = start(nb - 1) + n / cps,
+// with P resident CTAs and lag = (2 NW + 2) W columns (NW warps skewed by two
+// tiles, plus the border load one tile ahead and drain one tile behind).
+static double model_fill_time(long long nb, long long P, long long n, long long lag, double cps)
+{
+    // closed form of the recurrence: the max is at the last full CTA sweep when n >= P lag
+    const long long b = nb - 1;
+    const double chain = (double)b * (double)lag;
+    const double waves = (double)(b / P) * (double)n + (double)(b % P) * (double)lag;
+    return (std::max(chain, waves) + (double)n) / cps;
+}
 
 static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
 {
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
-    const bool packed_ok = ctx->packed && J.local && (J.k == 0 || J.k % 16 == 0) &&
-                           650ll * (pmax_abs + J.go + J.ge) + 1024 < 30000;
+    // packed preconditions: local mode, special rows at strip
+    // bottoms, and a warp's live values (32 alpha rows x ~130 columns of
+    // Manhattan distance, each step <= p_max + G_first apart) inside the 16-bit frame
+    auto packed_ok = [&](const Variant &V) {
+        const long long span = 32ll * V.alpha + 140;
+        return ctx->packed && J.local && V.packed_fn && (J.k == 0 || J.k % V.alpha == 0) &&
+               span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
+    };
     if (ctx->variant_override >= 0) {
         const Variant &V = variant_for(ctx->variant_override);
-        *use16 = packed_ok && V.packed_fn;
+        *use16 = packed_ok(V);
+        if (!*use16 && !V.local_fn) return variant_for(DEFAULT_VARIANT);  // packed-only geometry
         return V;
     }
+    // profiles/r01_variants.txt; earlier entries win near-ties (3 %)
     static const Candidate cands[] = {
-        {DEFAULT_VARIANT, false, 2572.0},  // int32, 8 warps
-        {1, true, 3130.0},                 // packed, 8 warps + I/O warp
-        {0, true, 2785.0},                 // packed, 4 warps, 3 CTAs/SM
-        {3, true, 2851.0},                 // packed, 12 warps
-        {5, true, 3243.0},                 // packed, 15 warps + I/O warp
-        {6, true, 3470.0},                 // packed, 16 warps, cooperative I/O
+        {DEFAULT_VARIANT, false, 4.24e6, 4.24e6},  // int32, 8 warps + I/O warp
+        {1, true, 5.967e6, 6.04e6},                // packed alpha 16, 8 warps + I/O warp
+        {8, true, 3.180e6, 6.05e6},                // packed alpha 32, 4 warps + I/O warp (2 CTAs/SM)
+        {10, true, 3.349e6, 3.349e6},              // packed alpha 32, 8 warps + I/O warp
+        {5, true, 3.363e6, 3.363e6},               // packed alpha 16, 15 warps + I/O warp
+        {6, true, 3.084e6, 3.084e6},               // packed alpha 16, 16 warps, cooperative I/O
     };
     double best_t = 1e300;
     int best = 0;
     for (int c = 0; c < (int)(sizeof(cands) / sizeof(cands[0])); c++) {
         const Candidate &C = cands[c];
-        if (C.packed && !packed_ok) continue;
-        if (!C.packed && !J.local) { best = c; break; }  // reverse pass: int32 only
         const Variant &V = variant_for(C.variant);
+        if (C.packed && !packed_ok(V)) continue;
+        if (!C.packed && !J.local) { best = c; break; }  // reverse pass: int32 only
         const void *fn = C.packed ? V.packed_fn : V.local_fn;
         if (!fn) continue;
         int per_sm = 0;
@@ -503,10 +545,10 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
                                                       C.packed ? V.smem16 : V.smem);
         const long long P = (long long)std::max(1, per_sm) * ctx->num_sms;
         const long long bh = (long long)V.alpha * 32 * V.nw;
-        const long long nb = (J.m + bh - 1) / bh;
-        // one sweep of one band takes bh * P / rate whether or not all P CTAs are busy
-        const double t = (double)((nb + P - 1) / P) * (double)bh * (double)P / C.rate;
-        if (t < best_t * 0.97) {  // prefer earlier (simpler) candidates on near-ties
+        const long long nb = std::max<long long>(1, (J.m + bh - 1) / bh);
+        const double cps = nb <= ctx->num_sms ? C.cps_solo : C.cps_full;
+        const double t = model_fill_time(nb, P, std::max<long long>(J.n, 1), (2ll * V.nw + 2) * V.w, cps);
+        if (t < best_t * 0.97) {
             best_t = t;
             best = c;
         }

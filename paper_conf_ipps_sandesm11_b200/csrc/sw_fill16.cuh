@@ -45,14 +45,14 @@ __device__ __forceinline__ uint32_t col_sel16(uint32_t code)
     return lo | (hi << 8);
 }
 
-template <int NW, int W>
+template <int NW, int W, int NS = 8>
 struct Fill16 {
-    static constexpr int ALPHA = 16, BH = ALPHA * 32 * NW;
+    static constexpr int ALPHA = 2 * NS, BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
     static constexpr int SRING = Smem<W, NW>::SRING;
     static constexpr int SKEW = 63;     // lane 31's output column lags lane 0's by 2*31 + 1
     static constexpr int STEPS = W;     // one column per lane step
-    static constexpr int NSAVE = 20;
+    static constexpr int NSAVE = 2 * NS + 3;
     static constexpr int HALF = SRING / 2 + 32;  // selector ring: one parity half + a 32-entry mirror
     // Warp-to-warp rings of (t, F): column col lives at ridx(col) in [1, RING]
     // (stride RS = RING + 1), so the 64 columns k0 - 63 .. k0 a lane-31 tile
@@ -71,10 +71,10 @@ struct Fill16 {
     }
 
     struct Lane {
-        uint32_t P[8], Q[8];  // int8x4 profiles of rows s (low halves) and s+8 (high halves)
-        uint32_t e[8], t[8];  // packed E and t = H - G_first of the previous column of each half
+        uint32_t P[NS], Q[NS];  // int8x4 profiles of rows s (low halves) and s+NS (high halves)
+        uint32_t e[NS], t[NS];  // packed E and t = H - G_first of the previous column of each half
         uint32_t tprev;       // packed diagonal input of slot 0
-        uint32_t fn;          // packed F of the rows after slot 7 (low: row 8 at j, high: row 16 at j-1)
+        uint32_t fn;          // packed F of the rows after the last slot (low: row NS at j, high: row 2NS at j-1)
         int B;                // warp-uniform frame base
         int adj;              // BIAS16 - B: int32 value -> frame
         int Bm;               // B - BIAS16: frame -> int32 value
@@ -119,7 +119,7 @@ struct Fill16 {
                                                     int one, uint32_t tmax, int row1, int &bs, int &bi, int &bj,
                                                     int *sp_ptr)
     {
-        const uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[7], 1);
+        const uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[NS - 1], 1);
         const uint32_t up_f = __shfl_up_sync(0xffffffffu, L.fn, 1);
         const int jl = k - 2 * lane;
         // lane 0: the warp above's bottom row at column jl, already in this warp's
@@ -129,16 +129,17 @@ struct Fill16 {
         asm volatile("ld.shared.u32 %0, [%1];" : "=r"(sel) : "r"(sel_a) : "memory");
         Lane S;
         if (GUARD) S = L;
+        if (TRACK) tmax = 0;
         const uint32_t tmax_in = tmax;
         // slot-0 inputs: low = upper lane's row 15 (its high half) or the ring, high = own row 7
-        uint32_t tu = __byte_perm(lane == 0 ? cr : up_t, L.t[7], pt_sel);
+        uint32_t tu = __byte_perm(lane == 0 ? cr : up_t, L.t[NS - 1], pt_sel);
         uint32_t fu = __byte_perm(lane == 0 ? cr : up_f, L.fn, 0x5432);  // F of slot 0's rows
         uint32_t td = L.tprev;
         L.tprev = tu;
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
         uint32_t f15 = 0;  // F entering slot 7 (row 15 in the high half)
 #pragma unroll
-        for (int s = 0; s < 8; s += 2) {
+        for (int s = 0; s < NS; s += 2) {
             const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
             const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
             const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
@@ -148,7 +149,7 @@ struct Fill16 {
             fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d0, one, ngf2));
             L.e[s] = e0;
             L.t[s] = t0;
-            if (s == 6) f15 = fu;
+            if (s == NS - 2) f15 = fu;
             const uint32_t e1 = __vimax3_u16x2((uint32_t)imad((int)L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
             const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
             const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
@@ -158,30 +159,15 @@ struct Fill16 {
             fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d1, one, ngf2));
             L.e[s + 1] = e1;
             L.t[s + 1] = t1;
-            tmax = __vimax3_u16x2(tmax, h0, h1);
-            if (TRACK) {
-                const uint32_t hs[2] = {h0, h1};
-#pragma unroll
-                for (int q = 0; q < 2; q++) {
-                    const int rlo = row1 + s + q, rhi = rlo + 8;
-                    if (jl >= 0 && jl < X.w && rlo <= a.m) {
-                        const int v = toabs(L, lo16(hs[q])), c = X.col0 + jl + 1;
-                        if (better(v, rlo, c, bs, bi, bj)) { bs = v; bi = rlo; bj = c; }
-                    }
-                    if (jl >= 1 && jl - 1 < X.w && rhi <= a.m) {
-                        const int v = toabs(L, hi16(hs[q])), c = X.col0 + jl;
-                        if (better(v, rhi, c, bs, bi, bj)) { bs = v; bi = rhi; bj = c; }
-                    }
-                }
-            }
+            tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
             if (CAP) {
                 if (jl == X.jcap) {
                     X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
                     X.rbrow[s + 1] = make_int2(toabs(L, lo16(t1)), toabs(L, lo16(e1)));
                 }
                 if (jl - 1 == X.jcap) {
-                    X.rbrow[s + 8] = make_int2(toabs(L, hi16(t0)), toabs(L, hi16(e0)));
-                    X.rbrow[s + 9] = make_int2(toabs(L, hi16(t1)), toabs(L, hi16(e1)));
+                    X.rbrow[s + NS] = make_int2(toabs(L, hi16(t0)), toabs(L, hi16(e0)));
+                    X.rbrow[s + NS + 1] = make_int2(toabs(L, hi16(t1)), toabs(L, hi16(e1)));
                 }
             }
         }
@@ -190,7 +176,7 @@ struct Fill16 {
             // lanes left of column 0 keep their state; at jl == 0 only the high half waits
             const uint32_t keep = (jl >= 0 ? 0x0000ffffu : 0u) | (jl >= 1 ? 0xffff0000u : 0u);
 #pragma unroll
-            for (int s = 0; s < 8; s++) {
+            for (int s = 0; s < NS; s++) {
                 L.e[s] = (L.e[s] & keep) | (S.e[s] & ~keep);
                 L.t[s] = (L.t[s] & keep) | (S.t[s] & ~keep);
             }
@@ -200,15 +186,46 @@ struct Fill16 {
             }
             tmax = (tmax & keep) | (tmax_in & ~keep);
         }
-        const int jo = jl - 1;  // row 15's column (high half of slot 7)
+        if (TRACK) {
+            // Replay: the step's cells are t[s] + G_first now.  The best cell
+            // of the step (max, then min row; a row occurs once per step) is
+            // the only one that can beat the running best.  Halves outside
+            // the stripe's columns are masked; a pad row (> m) never holds a
+            // step maximum that beats the best (its F is below an H of a real
+            // row of the same column, examined at this or the previous step,
+            // and rows are scanned in increasing order).
+            const bool lo_ok = jl >= 0 && jl < X.w, hi_ok = jl >= 1 && jl - 1 < X.w;
+            const uint32_t vm = (lo_ok ? 0x0000ffffu : 0u) | (hi_ok ? 0xffff0000u : 0u);
+            const uint32_t tm = tmax & vm;
+            const int M = max(lo16(tm), hi16(tm));
+            if (vm != 0u && toabs(L, M) >= max(bs, 1)) {
+                const uint32_t Mt = (uint32_t)(M - a.gf) * 0x10001u;
+                uint32_t lob = 0u, hib = 0u;
+#pragma unroll
+                for (int s = 0; s < NS; s++) {
+                    const uint32_t eq = __vcmpeq2(L.t[s], Mt);
+                    lob |= (eq & 1u) << s;
+                    hib |= (eq >> 31) << s;
+                }
+                lob = lo_ok ? lob : 0u;
+                hib = hi_ok ? hib : 0u;
+                int row, col;
+                if (lob) { row = row1 + __ffs(lob) - 1; col = X.col0 + jl + 1; }
+                else { row = row1 + NS + __ffs(hib) - 1; col = X.col0 + jl; }
+                const int v = toabs(L, M);
+                if ((lob | hib) && row <= a.m && better(v, row, col, bs, bi, bj)) { bs = v; bi = row; bj = col; }
+            }
+            return 0;
+        }
+        const int jo = jl - 1;  // row 2NS-1's column (high half of the last slot)
         if (SP1 && sp_ptr != nullptr && jo >= 0 && jo < X.w) {
-            sp_ptr[jo] = toabs(L, hi16(L.t[7])) + a.gf;  // H = t + G_first
+            sp_ptr[jo] = toabs(L, hi16(L.t[NS - 1])) + a.gf;  // H = t + G_first
             sp_ptr[X.sp_ld + jo] = toabs(L, hi16(f15));
         }
         if (!TRACK && lane == 31 && (!GUARD || jo >= 0)) {
             // (t, F) of row 15 at column jo for the next warp (int32, absolute)
             asm volatile("st.shared.v2.s32 [%0], {%1, %2};" ::"r"(ro_a),
-                         "r"(toabs(L, hi16(L.t[7]))), "r"(toabs(L, hi16(f15))) : "memory");
+                         "r"(toabs(L, hi16(L.t[NS - 1]))), "r"(toabs(L, hi16(f15))) : "memory");
         }
         return tmax;
     }
@@ -270,7 +287,7 @@ struct Fill16 {
         const int d = __shfl_sync(0xffffffffu, lo16(L.t[0]), 0) - BIAS16;
         const int d2 = -(d * 0x10001);
 #pragma unroll
-        for (int s = 0; s < 8; s++) {
+        for (int s = 0; s < NS; s++) {
             L.e[s] = (uint32_t)imad((int)L.e[s], a.one, d2);
             L.t[s] = (uint32_t)imad((int)L.t[s], a.one, d2);
         }
@@ -286,24 +303,24 @@ struct Fill16 {
     static __device__ __forceinline__ void save(const Lane &L, int *sv, int lane)
     {
 #pragma unroll
-        for (int s = 0; s < 8; s++) {
+        for (int s = 0; s < NS; s++) {
             sv[s * 32 + lane] = (int)L.e[s];
-            sv[(8 + s) * 32 + lane] = (int)L.t[s];
+            sv[(NS + s) * 32 + lane] = (int)L.t[s];
         }
-        sv[16 * 32 + lane] = (int)L.tprev;
-        sv[17 * 32 + lane] = (int)L.fn;
-        sv[19 * 32 + lane] = L.B;
+        sv[(2 * NS) * 32 + lane] = (int)L.tprev;
+        sv[(2 * NS + 1) * 32 + lane] = (int)L.fn;
+        sv[(2 * NS + 2) * 32 + lane] = L.B;
     }
     static __device__ __forceinline__ void restore(Lane &L, const int *sv, int lane)
     {
 #pragma unroll
-        for (int s = 0; s < 8; s++) {
+        for (int s = 0; s < NS; s++) {
             L.e[s] = (uint32_t)sv[s * 32 + lane];
-            L.t[s] = (uint32_t)sv[(8 + s) * 32 + lane];
+            L.t[s] = (uint32_t)sv[(NS + s) * 32 + lane];
         }
-        L.tprev = (uint32_t)sv[16 * 32 + lane];
-        L.fn = (uint32_t)sv[17 * 32 + lane];
-        L.B = sv[19 * 32 + lane];
+        L.tprev = (uint32_t)sv[(2 * NS) * 32 + lane];
+        L.fn = (uint32_t)sv[(2 * NS + 1) * 32 + lane];
+        L.B = sv[(2 * NS + 2) * 32 + lane];
         L.adj = BIAS16 - L.B;
         L.Bm = L.B - BIAS16;
         const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
@@ -315,10 +332,11 @@ struct Fill16 {
 // warps that also share the I/O (each loads and drains W / NW columns per
 // tile), so all four SMSPs carry the same number of compute warps (16 warps:
 // 4 each) -- the lockstep interval otherwise waits for the busier SMSPs.
-template <int NW, int W, bool COOP = false>
+template <int NW, int W, bool COOP = false, int NS = 8>
 __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
 {
-    using F = Fill16<NW, W>;
+    using F = Fill16<NW, W, NS>;
+    constexpr int ALPHA = F::ALPHA;
     constexpr int BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int2 *rings = reinterpret_cast<int2 *>(smem_raw);
@@ -363,23 +381,23 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         if (b >= a.nb) break;
 
         typename F::Lane L;
-        const int row0 = b * BH + (warp * 32 + lane) * 16;
+        const int row0 = b * BH + (warp * 32 + lane) * ALPHA;
         int *sp_ptr = nullptr;
         bool warp_sp = false;
         X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
         auto init_state = [&](bool from_left) {
             // state at the column left of the stripe: the column-0 boundary or the left border
-            int tv[16], ev[16];
+            int tv[ALPHA], ev[ALPHA];
             if (from_left) {
 #pragma unroll
-                for (int r = 0; r < 16; r++) {
+                for (int r = 0; r < ALPHA; r++) {
                     const int2 v = ld_sys_int2(S.lb + row0 + 1 + r);
                     tv[r] = v.x;
                     ev[r] = v.y;
                 }
             } else {
 #pragma unroll
-                for (int r = 0; r < 16; r++) { tv[r] = -a.gf; ev[r] = -a.gf; }  // E(i,0) := t(i,0), exact
+                for (int r = 0; r < ALPHA; r++) { tv[r] = -a.gf; ev[r] = -a.gf; }  // E(i,0) := t(i,0), exact
             }
             int tp;
             if (from_left && row0 > 0) tp = ld_sys_int2(S.lb + row0).x;
@@ -388,26 +406,30 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             L.adj = BIAS16 - L.B;
             L.Bm = L.B - BIAS16;
 #pragma unroll
-            for (int s = 0; s < 8; s++) {
-                L.e[s] = pk(F::tofr(L, ev[s]), F::tofr(L, ev[s + 8]));
-                L.t[s] = pk(F::tofr(L, tv[s]), F::tofr(L, tv[s + 8]));
+            for (int s = 0; s < NS; s++) {
+                L.e[s] = pk(F::tofr(L, ev[s]), F::tofr(L, ev[s + NS]));
+                L.t[s] = pk(F::tofr(L, tv[s]), F::tofr(L, tv[s + NS]));
             }
             L.tprev = pk(F::tofr(L, tp), F::tofr(L, tp));
-            L.fn = L.t[7];  // only feeds the high half at column -1 (kept by GUARD)
+            L.fn = L.t[NS - 1];  // only feeds the high half at column -1 (kept by GUARD)
             const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
             L.FL = (uint32_t)fl * 0x10001u;
         };
         if (warp < NW) {
-            const uint32_t w = row0 < a.m ? a.A2[row0 >> 4] : 0u;
+            // row r's code: bits 2 (r & 15) of word r >> 4 (row0 is a multiple of 16)
+            uint32_t wv[ALPHA / 16];
 #pragma unroll
-            for (int s = 0; s < 8; s++) {
-                L.P[s] = (row0 + s < a.m) ? a.prof[(w >> (2 * s)) & 3u] : PADPROF;
-                L.Q[s] = (row0 + s + 8 < a.m) ? a.prof[(w >> (2 * (s + 8))) & 3u] : PADPROF;
+            for (int q = 0; q < ALPHA / 16; q++) wv[q] = row0 + 16 * q < a.m ? a.A2[(row0 >> 4) + q] : 0u;
+#pragma unroll
+            for (int s = 0; s < NS; s++) {
+                const int rp = s, rq = s + NS;
+                L.P[s] = (row0 + rp < a.m) ? a.prof[(wv[rp >> 4] >> (2 * (rp & 15))) & 3u] : PADPROF;
+                L.Q[s] = (row0 + rq < a.m) ? a.prof[(wv[rq >> 4] >> (2 * (rq & 15))) & 3u] : PADPROF;
             }
             init_state(false);
             if (a.k > 0) {
-                // special rows are strip-bottom rows (k a multiple of 16): row0 + 16
-                const int row = row0 + 16;
+                // special rows are strip-bottom rows (k a multiple of ALPHA): row0 + ALPHA
+                const int row = row0 + ALPHA;
                 if (row <= a.m && row % a.k == 0 && row != (b + 1) * BH)  // band bottom: the I/O warp's drain
                     sp_ptr = S.sp + (long long)(row / a.k - 1) * S.sp_stride;
             }

@@ -10,7 +10,9 @@ import synth
 
 pytestmark = pytest.mark.gpu
 PAPER = (1, -3, 3, 2)
-PACKED_VARIANTS = [0, 3, 5, 6]  # (16, 4), (16, 12), (16, 15) warps + I/O warp; 16 warps with cooperative I/O
+PACKED_VARIANTS = [0, 3, 5, 6, 8, 9, 10, 11]
+# alpha 16: 4, 12, 15 warps + I/O warp, 16 warps with cooperative I/O;
+# alpha 32 (16 slots per lane): 4 warps + I/O warp, 4 cooperative, 8 + I/O warp, 16 cooperative
 
 
 @pytest.fixture(scope="module")
@@ -51,7 +53,7 @@ def check(ctx, A, B, scoring, k, variant, stripes=1, expect_packed=True):
 @pytest.mark.parametrize("m,n", [(1, 1), (17, 1), (16, 300), (1000, 999), (3000, 64), (5000, 2049)])
 def test_packed_shapes(ctx, variant, m, n):
     A, B = synth.random_pair(m + 3 * n + variant, m, n, plant_len=min(m, n) // 2, s=0.05, g=0.01)
-    check(ctx, A, B, PAPER, 16, variant)
+    check(ctx, A, B, PAPER, 32, variant)
 
 
 @pytest.mark.parametrize("variant", PACKED_VARIANTS)
@@ -82,6 +84,19 @@ def test_packed_virtual_stripes(ctx, stripes):
     A, B = synth.random_pair(60 + stripes, 6000, 1500, plant_len=1200, s=0.04, g=0.01)
     check(ctx, A, B, PAPER, 16, 0, stripes=stripes)
     check(ctx, A, B, PAPER, 0, 5, stripes=stripes)
+
+
+@pytest.mark.parametrize("variant", [8, 9, 10, 11])
+def test_packed_alpha32(ctx, variant):
+    """16 slots per lane: special rows at strip bottoms (k % 32 == 0), ties,
+    stripes, and the int32 fallback when k is only a multiple of 16."""
+    A, B = synth.random_pair(70 + variant, 7000, 2100, plant_len=1500, s=0.04, g=0.01)
+    check(ctx, A, B, PAPER, 96, variant)
+    check(ctx, A, B, (5, -4, 10, 1), 64, variant)
+    check(ctx, A, B, PAPER, 16, variant, expect_packed=False)
+    X = synth.random_pair(4, 500, 1)[0]
+    check(ctx, np.concatenate([X, X, X, X]), X, PAPER, 32, variant)
+    check(ctx, A, B, PAPER, 32, variant, stripes=3)
 
 
 def test_packed_config_c1(ctx):
