@@ -109,7 +109,7 @@ struct Variant {
     int skew_tiles;         // int32 kernel: tiles past the last column lane 31 needs (ceil(62 / W))
 };
 
-template <int ALPHA, int NW, int W, bool COOP = false>
+template <int ALPHA, int NW, int W, bool COOP = false, bool SPLIT = false>
 static Variant make_variant()
 {
     Variant v;
@@ -124,9 +124,9 @@ static Variant make_variant()
     v.skew_tiles = 1;
     if constexpr (ALPHA == 32) {
         // packed kernel only (16 slots per lane); int32 work falls back to the default geometry
-        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, 16>;
+        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, 16, SPLIT>;
         v.io_warps = COOP ? 0 : 1;
-        v.smem16 = Fill16<NW, W, 16>::smem_bytes();
+        v.smem16 = Fill16<NW, W, 16, SPLIT>::smem_bytes();
         return v;
     } else {
         v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
@@ -147,7 +147,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 12;
+static constexpr int NVARIANTS = 13;
 static constexpr int NINT32_VARIANTS = 8;  // variants 0..7 have int32 kernels; 8.. are packed-only (alpha 32)
 
 static const Variant &variant_for(int idx)
@@ -165,6 +165,7 @@ static const Variant &variant_for(int idx)
         make_variant<32, 4, 64, true>(),
         make_variant<32, 8, 64>(),
         make_variant<32, 16, 64, true>(),
+        make_variant<32, 4, 64, false, true>(),  // split F chain (latency-bound one-wave fills)
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }

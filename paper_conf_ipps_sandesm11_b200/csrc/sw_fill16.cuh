@@ -45,7 +45,7 @@ __device__ __forceinline__ uint32_t col_sel16(uint32_t code)
     return lo | (hi << 8);
 }
 
-template <int NW, int W, int NS = 8>
+template <int NW, int W, int NS = 8, bool SPLIT = false>
 struct Fill16 {
     static constexpr int ALPHA = 2 * NS, BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
@@ -137,37 +137,93 @@ struct Fill16 {
         uint32_t td = L.tprev;
         L.tprev = tu;
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
-        uint32_t f15 = 0;  // F entering slot 7 (row 15 in the high half)
+        uint32_t f15 = 0;  // F entering the last slot (row 2NS-1 in the high half)
+        if constexpr (SPLIT) {
+            // Same cells, shorter F chain for latency-bound warps: D of every slot
+            // first (it only needs the previous column), then F down the rows as two
+            // half chains.  The second starts from D - G_first of the slot before
+            // it, a lower bound of the true F there, and is corrected by
+            // F_s = max(partial_s, F_h - (s - h) G_ext), h = NS/2 (the F recurrence
+            // is a max-plus scan: F_s = max over s' < s of (D_s' - G_first - (s-s'-1) G_ext)
+            // together with F_0 - s G_ext).
+            uint32_t d[NS];
 #pragma unroll
-        for (int s = 0; s < NS; s += 2) {
-            const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
-            const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
-            const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
-            const uint32_t h0 = __vmaxu2(d0, fu);
-            td = L.t[s];
-            const uint32_t t0 = (uint32_t)imad((int)h0, one, ngf2);
-            fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d0, one, ngf2));
-            L.e[s] = e0;
-            L.t[s] = t0;
-            if (s == NS - 2) f15 = fu;
-            const uint32_t e1 = __vimax3_u16x2((uint32_t)imad((int)L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
-            const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
-            const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
-            const uint32_t h1 = __vmaxu2(d1, fu);
-            td = L.t[s + 1];
-            const uint32_t t1 = (uint32_t)imad((int)h1, one, ngf2);
-            fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d1, one, ngf2));
-            L.e[s + 1] = e1;
-            L.t[s + 1] = t1;
-            tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
-            if (CAP) {
-                if (jl == X.jcap) {
-                    X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
-                    X.rbrow[s + 1] = make_int2(toabs(L, lo16(t1)), toabs(L, lo16(e1)));
+            for (int s = 0; s < NS; s++) {
+                const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
+                const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
+                d[s] = __viaddmax_u16x2(td, p0, e0);
+                td = L.t[s];
+                L.e[s] = e0;
+                if (CAP) {
+                    if (jl == X.jcap) X.rbrow[s].y = toabs(L, lo16(e0));
+                    if (jl - 1 == X.jcap) X.rbrow[s + NS].y = toabs(L, hi16(e0));
                 }
-                if (jl - 1 == X.jcap) {
-                    X.rbrow[s + NS] = make_int2(toabs(L, hi16(t0)), toabs(L, hi16(e0)));
-                    X.rbrow[s + NS + 1] = make_int2(toabs(L, hi16(t1)), toabs(L, hi16(e1)));
+            }
+            constexpr int HS = NS / 2;
+            uint32_t fa = fu, fb = (uint32_t)imad((int)d[HS - 1], one, ngf2);
+            uint32_t F[NS];
+#pragma unroll
+            for (int s = 0; s < HS; s++) {
+                F[s] = fa;
+                fa = __vmaxu2((uint32_t)imad((int)fa, one, nge2), (uint32_t)imad((int)d[s], one, ngf2));
+                F[HS + s] = fb;
+                fb = __vmaxu2((uint32_t)imad((int)fb, one, nge2), (uint32_t)imad((int)d[HS + s], one, ngf2));
+            }
+            // fa = F_HS; correct the second half and the outgoing F
+#pragma unroll
+            for (int s = 1; s < HS; s++) F[HS + s] = __vmaxu2(F[HS + s], (uint32_t)imad((int)fa, one, -(s * a.ge * 0x10001)));
+            F[HS] = fa;
+            fu = __vmaxu2(fb, (uint32_t)imad((int)fa, one, -(HS * a.ge * 0x10001)));
+            f15 = F[NS - 1];
+#pragma unroll
+            for (int s = 0; s < NS; s += 2) {
+                const uint32_t h0 = __vmaxu2(d[s], F[s]), h1 = __vmaxu2(d[s + 1], F[s + 1]);
+                L.t[s] = (uint32_t)imad((int)h0, one, ngf2);
+                L.t[s + 1] = (uint32_t)imad((int)h1, one, ngf2);
+                tmax = __vimax3_u16x2(tmax, h0, h1);
+                if (CAP) {
+                    if (jl == X.jcap) {
+                        X.rbrow[s].x = toabs(L, lo16(L.t[s]));
+                        X.rbrow[s + 1].x = toabs(L, lo16(L.t[s + 1]));
+                    }
+                    if (jl - 1 == X.jcap) {
+                        X.rbrow[s + NS].x = toabs(L, hi16(L.t[s]));
+                        X.rbrow[s + NS + 1].x = toabs(L, hi16(L.t[s + 1]));
+                    }
+                }
+            }
+        } else {
+#pragma unroll
+            for (int s = 0; s < NS; s += 2) {
+                const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
+                const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
+                const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
+                const uint32_t h0 = __vmaxu2(d0, fu);
+                td = L.t[s];
+                const uint32_t t0 = (uint32_t)imad((int)h0, one, ngf2);
+                fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d0, one, ngf2));
+                L.e[s] = e0;
+                L.t[s] = t0;
+                if (s == NS - 2) f15 = fu;
+                const uint32_t e1 = __vimax3_u16x2((uint32_t)imad((int)L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
+                const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
+                const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
+                const uint32_t h1 = __vmaxu2(d1, fu);
+                td = L.t[s + 1];
+                const uint32_t t1 = (uint32_t)imad((int)h1, one, ngf2);
+                fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d1, one, ngf2));
+                L.e[s + 1] = e1;
+                L.t[s + 1] = t1;
+                tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
+                if (CAP) {
+                    if (jl == X.jcap) {
+                        X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
+                        X.rbrow[s + 1] = make_int2(toabs(L, lo16(t1)), toabs(L, lo16(e1)));
+                    }
+                    if (jl - 1 == X.jcap) {
+                        X.rbrow[s + NS] = make_int2(toabs(L, hi16(t0)), toabs(L, hi16(e0)));
+                        X.rbrow[s + NS + 1] = make_int2(toabs(L, hi16(t1)), toabs(L, hi16(e1)));
+                    }
                 }
             }
         }
@@ -332,10 +388,10 @@ struct Fill16 {
 // warps that also share the I/O (each loads and drains W / NW columns per
 // tile), so all four SMSPs carry the same number of compute warps (16 warps:
 // 4 each) -- the lockstep interval otherwise waits for the busier SMSPs.
-template <int NW, int W, bool COOP = false, int NS = 8>
+template <int NW, int W, bool COOP = false, int NS = 8, bool SPLIT = false>
 __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
 {
-    using F = Fill16<NW, W, NS>;
+    using F = Fill16<NW, W, NS, SPLIT>;
     constexpr int ALPHA = F::ALPHA;
     constexpr int BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
     extern __shared__ __align__(16) unsigned char smem_raw[];

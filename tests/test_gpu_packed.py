@@ -10,9 +10,9 @@ import synth
 
 pytestmark = pytest.mark.gpu
 PAPER = (1, -3, 3, 2)
-PACKED_VARIANTS = [0, 3, 5, 6, 8, 9, 10, 11]
+PACKED_VARIANTS = [0, 3, 5, 6, 8, 9, 10, 11, 12]
 # alpha 16: 4, 12, 15 warps + I/O warp, 16 warps with cooperative I/O;
-# alpha 32 (16 slots per lane): 4 warps + I/O warp, 4 cooperative, 8 + I/O warp, 16 cooperative
+# alpha 32 (16 slots per lane): 4 warps + I/O warp, 4 cooperative, 8 + I/O warp, 16 cooperative, 4 + I/O split F chain
 
 
 @pytest.fixture(scope="module")
@@ -86,7 +86,7 @@ def test_packed_virtual_stripes(ctx, stripes):
     check(ctx, A, B, PAPER, 0, 5, stripes=stripes)
 
 
-@pytest.mark.parametrize("variant", [8, 9, 10, 11])
+@pytest.mark.parametrize("variant", [8, 9, 10, 11, 12])
 def test_packed_alpha32(ctx, variant):
     """16 slots per lane: special rows at strip bottoms (k % 32 == 0), ties,
     stripes, and the int32 fallback when k is only a multiple of 16."""
