@@ -22,6 +22,10 @@ G_first = gap_open + gap_ext, reading S2 in DESIGN.md):
 - ``global_score(A, B, ...)`` -> NW/Gotoh global score
 - ``reverse_goal(A, i_end, B, j_end, ..., goal)`` -> ``(goal, i_s, j_s)`` or None
 - ``flush_rows(m, n, alphaT, sra_bytes)`` -> special-row spacing
+- ``stage2(A, B, ..., k, best, i_end, j_end)`` -> crosspoint list L_2
+- ``align_partition(A, B, ..., Cs, Ce)`` -> (score, moves) of one partition
+- ``align(A, B, ..., k)`` -> the full optimal local alignment (Stages 1, 2, then
+  one partition at a time) with its GAP_1 / GAP_2 lists
 
 Parity pins live in ``tests/test_oracle_pins.py``; every function above is
 pinned (none is "parity unpinned").
@@ -82,6 +86,9 @@ def _load():
             lib.or_reverse_goal.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, ctypes.POINTER(_Res)]
             lib.or_stage2.argtypes = [cp, i64, cp, i64, i64, i64, i64, i64, i64, i64, i64, i64, p64, i64]
             lib.or_stage2.restype = i64
+            lib.or_align_partition.argtypes = [cp, cp, i64, i64, i64, i64, i64, i64, i64, i64, i64, i64,
+                                               ctypes.c_char_p, i64, p64]
+            lib.or_align_partition.restype = i64
             lib.or_flush_rows.argtypes = [i64, i64, i64, i64]
             lib.or_flush_rows.restype = i64
             _lib = lib
@@ -186,3 +193,70 @@ def stage2(A, B, ma, mi, go, ge, k, best, i_end, j_end):
 
 def flush_rows(m, n, alphaT, sra_bytes) -> int:
     return int(_load().or_flush_rows(m, n, alphaT, sra_bytes))
+
+
+def align_partition(A, B, ma, mi, go, ge, Cs, Ce):
+    """Optimal alignment of partition (Cs, Ce), Cs = (i_s, j_s, type_s),
+    Ce = (i_e, j_e, type_e); types 0 any / 1 horizontal gap (E) / 2 vertical gap (F).
+    Returns (score, moves) with moves a str over 'M' (pair), 'I' (gap in S0),
+    'D' (gap in S1), or (None, None) if no alignment has these end states."""
+    lib = _load()
+    a, b = _b(A), _b(B)
+    (i_s, j_s, t_s), (i_e, j_e, t_e) = Cs, Ce
+    cap = max(0, (i_e - i_s) + (j_e - j_s))
+    buf = ctypes.create_string_buffer(cap + 1)
+    nops = ctypes.c_int64(0)
+    sc = lib.or_align_partition(a, b, i_s, j_s, i_e, j_e, ma, mi, go, ge, t_s, t_e, buf, cap, ctypes.byref(nops))
+    if sc <= NEG // 2:
+        return None, None
+    if nops.value < 0:
+        raise RuntimeError("or_align_partition failed")
+    return int(sc), buf.raw[: nops.value].decode()
+
+
+def gap_lists(moves, i0, j0):
+    """GAP_1 / GAP_2 of P:281 from a move string starting at DP cell (i0, j0):
+    (i, j, length) per maximal gap run, (i, j) the cell the run leaves from
+    (reading S24).  GAP_1 = gaps in S0 (horizontal, 'I'), GAP_2 = gaps in S1
+    (vertical, 'D')."""
+    g1, g2 = [], []
+    i, j, q = i0, j0, 0
+    while q < len(moves):
+        c = moves[q]
+        r = q
+        while r < len(moves) and moves[r] == c:
+            r += 1
+        L = r - q
+        if c == "M":
+            i += L
+            j += L
+        elif c == "I":
+            g1.append((i, j, L))
+            j += L
+        else:
+            g2.append((i, j, L))
+            i += L
+        q = r
+    return g1, g2
+
+
+def align(A, B, ma, mi, go, ge, k):
+    """The full optimal local alignment: Stage 1 (best, end point, special rows
+    every k rows), Stage 2 (crosspoints L_2), then every partition between
+    consecutive crosspoints aligned on its own (Stages 3-5 reach the same
+    partition alignments in linear space).  Returns a dict with
+    score, start (i0, j0), end (i1, j1), moves, gap1, gap2, crosspoints."""
+    (best, ie, je), _ = stage1(A, B, ma, mi, go, ge, k=0, keep_rows=False)
+    if best == 0:
+        return {"score": 0, "start": (0, 0), "end": (0, 0), "moves": "", "gap1": [], "gap2": [], "crosspoints": []}
+    L = stage2(A, B, ma, mi, go, ge, k, best, ie, je)
+    moves = []
+    for (i_s, j_s, sc_s, t_s), (i_e, j_e, sc_e, t_e) in zip(L, L[1:]):
+        sc, mv = align_partition(A, B, ma, mi, go, ge, (i_s, j_s, t_s), (i_e, j_e, t_e))
+        if sc != sc_e - sc_s:
+            raise RuntimeError(f"partition {(i_s, j_s, t_s)} -> {(i_e, j_e, t_e)}: {sc} != {sc_e - sc_s}")
+        moves.append(mv)
+    mv = "".join(moves)
+    g1, g2 = gap_lists(mv, L[0][0], L[0][1])
+    return {"score": best, "start": (L[0][0], L[0][1]), "end": (ie, je), "moves": mv, "gap1": g1, "gap2": g2,
+            "crosspoints": L}

@@ -156,3 +156,33 @@ def all_local_starts(S0: str, S1: str, ma: int, mi: int, G_open: int, G_ext: int
             if found[0]:
                 starts.add((s, t))
     return starts
+
+
+def partition_best(S0: str, S1: str, ma: int, mi: int, G_open: int, G_ext: int, type_s: int, type_e: int):
+    """Max score over all alignments of the whole of S0 with the whole of S1
+    that start in crosspoint state type_s and end in state type_e:
+    type 1 = the path is inside a horizontal gap (a gap in S0), type 2 = inside
+    a vertical gap (a gap in S1), 0 = no constraint.  A gap run that continues
+    the start state costs G_ext per column (its opening was charged before the
+    partition); every other maximal run costs G_first + (L-1) G_ext.
+    Each alignment is listed explicitly (tiny inputs only).  None if no
+    alignment has the required end state."""
+    m, n = len(S0), len(S1)
+    G_first = G_open + G_ext
+    best = [None]
+    start_last = {0: None, 1: "H", 2: "V"}[type_s]
+    want_last = {0: None, 1: "H", 2: "V"}[type_e]
+
+    def walk(i, j, score, last):
+        if i == m and j == n and (want_last is None or last == want_last):
+            best[0] = _mx(best[0], score)
+        if i < m and j < n:
+            p = ma if S0[i].upper() == S1[j].upper() else mi
+            walk(i + 1, j + 1, score + p, "D")
+        if j < n:
+            walk(i, j + 1, score - (G_ext if last == "H" else G_first), "H")
+        if i < m:
+            walk(i + 1, j, score - (G_ext if last == "V" else G_first), "V")
+
+    walk(0, 0, 0, start_last)
+    return best[0]

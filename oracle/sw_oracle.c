@@ -425,3 +425,93 @@ int64_t or_stage2(const char *S0, int64_t m, const char *S1, int64_t n, int64_t 
     free(L); free(R.H); free(R.F);
     return rc;
 }
+
+/*
+ * Stages 3-5 for one partition P = (C_s, C_e) of L_k:
+ * the optimal alignment of S0[i_s+1..i_e] with S1[j_s+1..j_e] that starts in
+ * the state of C_s and ends in the state of C_e, by a full (h+1) x (w+1)
+ * Gotoh matrix and its traceback (the definition the paper's Myers-Miller
+ * stages reach in linear space; reading S23 in DESIGN.md):
+ *
+ *   types: 0 = match/mismatch (any state), 1 = gap in S0 (horizontal,
+ *   matrix E), 2 = gap in S1 (vertical, matrix F);
+ *   start: H(0,0) = 0, E(0,0) = 0 if type_s = 1 else -inf, F(0,0) = 0 if
+ *   type_s = 2 else -inf -- a gap that crosses C_s continues at G_ext without
+ *   a second opening;
+ *   cells: Eq. 1-3 without the 0 term (global recurrence);
+ *   end: the value of H, E or F at (h, w) by type_e.
+ *
+ * Writes the moves in forward order to ops ('M' diagonal pair, 'I' gap in S0
+ * = horizontal, 'D' gap in S1 = vertical); returns the partition score, or
+ * NEG if no alignment with these end states exists (-2 capacity / -1 memory
+ * errors are reported through *nops = -1).  Traceback preference at equal
+ * values: H state -> diagonal, then F, then E; E/F states -> extension, then
+ * opening.
+ */
+int64_t or_align_partition(const char *S0, const char *S1, int64_t i_s, int64_t j_s, int64_t i_e, int64_t j_e,
+                           int64_t ma, int64_t mi, int64_t G_open, int64_t G_ext, int64_t type_s,
+                           int64_t type_e, char *ops, int64_t cap, int64_t *nops)
+{
+    const int64_t G_first = G_open + G_ext;
+    const int64_t h = i_e - i_s, w = j_e - j_s, W = w + 1;
+    *nops = -1;
+    if (h < 0 || w < 0) return NEG;
+    int64_t *H = malloc((size_t)((h + 1) * W) * sizeof(int64_t));
+    int64_t *E = malloc((size_t)((h + 1) * W) * sizeof(int64_t));
+    int64_t *F = malloc((size_t)((h + 1) * W) * sizeof(int64_t));
+    if (!H || !E || !F) { free(H); free(E); free(F); return NEG; }
+#define AT(M, a, b) M[(a) * W + (b)]
+    for (int64_t a = 0; a <= h; a++)
+        for (int64_t b = 0; b <= w; b++) {
+            if (a == 0 && b == 0) {
+                AT(H, 0, 0) = 0;
+                AT(E, 0, 0) = type_s == 1 ? 0 : NEG;
+                AT(F, 0, 0) = type_s == 2 ? 0 : NEG;
+                continue;
+            }
+            const int64_t e = b > 0 ? max2(AT(E, a, b - 1) - G_ext, AT(H, a, b - 1) - G_first) : NEG; /* Eq. 2 */
+            const int64_t f = a > 0 ? max2(AT(F, a - 1, b) - G_ext, AT(H, a - 1, b) - G_first) : NEG; /* Eq. 3 */
+            const int64_t d = (a > 0 && b > 0) ? AT(H, a - 1, b - 1) + p_score(S0[i_s + a - 1], S1[j_s + b - 1], ma, mi)
+                                               : NEG;                                                   /* Eq. 1 */
+            AT(E, a, b) = e < NEG / 2 ? NEG : e;
+            AT(F, a, b) = f < NEG / 2 ? NEG : f;
+            const int64_t hv = max2(max2(e, f), d);
+            AT(H, a, b) = hv < NEG / 2 ? NEG : hv;
+        }
+    const int64_t score = type_e == 1 ? AT(E, h, w) : type_e == 2 ? AT(F, h, w) : AT(H, h, w);
+    if (score <= NEG / 2) { free(H); free(E); free(F); return NEG; }
+    /* traceback from (h, w) in the end state */
+    int64_t a = h, b = w, n = 0;
+    int st = type_e == 1 ? 1 : type_e == 2 ? 2 : 0;
+    char *rev = malloc((size_t)(h + w + 1));
+    if (!rev) { free(H); free(E); free(F); return NEG; }
+    while (a > 0 || b > 0) {
+        if (st == 0) {
+            if (a > 0 && b > 0 &&
+                AT(H, a, b) == AT(H, a - 1, b - 1) + p_score(S0[i_s + a - 1], S1[j_s + b - 1], ma, mi)) {
+                rev[n++] = 'M'; a--; b--;
+            } else if (a > 0 && AT(H, a, b) == AT(F, a, b)) {
+                st = 2;
+            } else {
+                st = 1;
+            }
+        } else if (st == 2) {
+            rev[n++] = 'D';
+            if (AT(F, a, b) == AT(F, a - 1, b) - G_ext && AT(F, a - 1, b) > NEG / 2) st = 2;
+            else st = 0;
+            a--;
+        } else {
+            rev[n++] = 'I';
+            if (AT(E, a, b) == AT(E, a, b - 1) - G_ext && AT(E, a, b - 1) > NEG / 2) st = 1;
+            else st = 0;
+            b--;
+        }
+    }
+#undef AT
+    free(H); free(E); free(F);
+    if (n > cap) { free(rev); return score; }
+    for (int64_t q = 0; q < n; q++) ops[q] = rev[n - 1 - q];
+    free(rev);
+    *nops = n;
+    return score;
+}

@@ -1,2 +1,4 @@
-timeout 600 python tools/fill_bench.py C2 0 1 3 5 6 8 9 10 11 --reps=2
-timeout 600 python tools/fill_bench.py R2000000x536165 0 1 3 5 6 8 9 10 11 --reps=2
+set -x
+timeout 900 python -m pytest tests/test_gpu_packed.py -x -q 2>&1 | tail -3
+timeout 300 python tools/fill_bench.py C2 8 12 --reps=3
+timeout 300 python tools/fill_bench.py R10000000x1000000 12 --reps=1
