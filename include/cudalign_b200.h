@@ -158,6 +158,43 @@ int sw_stage2_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, 
                   int64_t special_row_interval, const sw_result *end, void *stream,
                   sw_crosspoint *out, int64_t cap, int64_t *count);
 
+/* One maximal gap run of the final alignment: (i, j) is the DP cell
+ * the run leaves from (reading S24), len the number of gap columns.  GAP_1
+ * holds gaps in S0 (horizontal: S1 characters against '-'), GAP_2 gaps in S1
+ * (vertical). */
+typedef struct {
+    int64_t i;
+    int64_t j;
+    int64_t len;
+} sw_gap;
+
+/* The optimal local alignment: score, start cell (i0, j0) (the cell
+ * before the first aligned pair, reading S8), end cell (i1, j1) (Stage 1's best
+ * cell), the lengths of the GAP_1 / GAP_2 lists, and how the Myers-Miller stage
+ * ran (partitions aligned in Stage 5, splitting levels). */
+typedef struct {
+    int32_t score;
+    int64_t i0, j0, i1, j1;
+    int64_t n_gap1, n_gap2;
+    int64_t partitions, mm_levels;
+} sw_alignment;
+
+/* Stages 1-5: the full optimal local alignment of S0 and S1.
+ * Stage 1 with special rows every special_row_interval rows (0: none, one
+ * Stage-2 partition), Stage 2 (crosspoints on the special rows, sw_stage2),
+ * then Myers-Miller with balanced splitting on the GPU until every partition
+ * has at most 65,536 cells, a full traceback of each, and the concatenation.
+ * Sequences and scoring as sw_align_stage1; gap1[0 .. cap1) / gap2[0 .. cap2)
+ * are caller-owned output arrays.  Returns SW_OK, or SW_ERANGE when a list did
+ * not fit (out->n_gap1 / n_gap2 hold the lengths needed; the first cap
+ * entries are written), or the errors of sw_align_stage1 / sw_stage2.
+ * Alignments tie-break among optimal ones by the traceback preference
+ * (diagonal, then vertical, then horizontal) inside each final partition. */
+int sw_align(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, int64_t n,
+             int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+             int64_t special_row_interval, sw_alignment *out,
+             sw_gap *gap1, int64_t cap1, sw_gap *gap2, int64_t cap2);
+
 /* Rows per thread strip (alpha): special_row_interval multiples of this take
  * the fast special-row path. */
 int64_t sw_row_granularity(const sw_ctx *ctx);

@@ -39,6 +39,7 @@ EXPORTED = [
     "sw_reverse_goal_dev",
     "sw_stage2",
     "sw_stage2_dev",
+    "sw_align",
     "sw_row_granularity",
     "sw_band_height",
     "sw_set_kernel",
@@ -66,6 +67,16 @@ class _Result(ctypes.Structure):
 
 class _Crosspoint(ctypes.Structure):
     _fields_ = [("i", ctypes.c_int64), ("j", ctypes.c_int64), ("score", ctypes.c_int32), ("type", ctypes.c_int32)]
+
+
+class _Gap(ctypes.Structure):
+    _fields_ = [("i", ctypes.c_int64), ("j", ctypes.c_int64), ("len", ctypes.c_int64)]
+
+
+class _Alignment(ctypes.Structure):
+    _fields_ = [("score", ctypes.c_int32), ("i0", ctypes.c_int64), ("j0", ctypes.c_int64), ("i1", ctypes.c_int64),
+                ("j1", ctypes.c_int64), ("n_gap1", ctypes.c_int64), ("n_gap2", ctypes.c_int64),
+                ("partitions", ctypes.c_int64), ("mm_levels", ctypes.c_int64)]
 
 
 class Stats(ctypes.Structure):
@@ -126,6 +137,9 @@ def load_library(path: str = LIB_PATH):
     lib.sw_stage2.restype = ctypes.c_int
     lib.sw_stage2_dev.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i64, R, vp, CP, i64, ctypes.POINTER(i64)]
     lib.sw_stage2_dev.restype = ctypes.c_int
+    lib.sw_align.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i64, ctypes.POINTER(_Alignment),
+                             ctypes.POINTER(_Gap), i64, ctypes.POINTER(_Gap), i64]
+    lib.sw_align.restype = ctypes.c_int
     lib.sw_row_granularity.argtypes = [vp]
     lib.sw_row_granularity.restype = i64
     lib.sw_band_height.argtypes = [vp]
@@ -288,6 +302,29 @@ class Context:
         return self._stage2_call(self._lib.sw_stage2_dev, (self._h, dA_ptr, m, dB_ptr, n, match, mismatch, gap_open,
                                                            gap_ext, k, ctypes.byref(r), stream or None),
                                  (m // k if k > 0 else 0) + 2)
+
+    def align(self, A, B, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0):
+        """Stages 1-5: the full optimal local alignment (sw_align).  Returns a dict:
+        score, start (i0, j0), end (i1, j1), gap1 / gap2 lists of (i, j, len)
+        (P:281), partitions, mm_levels."""
+        pa, m, ka = _as_bytes_ptr(A)
+        pb, n, kb = _as_bytes_ptr(B)
+        cap1 = cap2 = 1024
+        while True:
+            g1 = (_Gap * cap1)()
+            g2 = (_Gap * cap2)()
+            out = _Alignment()
+            rc = self._lib.sw_align(self._h, pa, m, pb, n, match, mismatch, gap_open, gap_ext, k, ctypes.byref(out),
+                                    g1, cap1, g2, cap2)
+            if rc == -3 and (out.n_gap1 > cap1 or out.n_gap2 > cap2):
+                cap1, cap2 = max(cap1, out.n_gap1), max(cap2, out.n_gap2)
+                continue
+            self._check(rc, "sw_align")
+            break
+        return {"score": out.score, "start": (out.i0, out.j0), "end": (out.i1, out.j1),
+                "gap1": [(g.i, g.j, g.len) for g in g1[: out.n_gap1]],
+                "gap2": [(g.i, g.j, g.len) for g in g2[: out.n_gap2]],
+                "partitions": out.partitions, "mm_levels": out.mm_levels}
 
     def row_granularity(self) -> int:
         return int(self._lib.sw_row_granularity(self._h))

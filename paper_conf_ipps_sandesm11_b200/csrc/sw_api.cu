@@ -207,6 +207,7 @@ struct sw_ctx {
     std::vector<cudaEvent_t> ev_row;  // one per staging slot: the slot's final copy is done
     int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
+    DevBuf mm_parts, mm_scratch, mm_res, mm_codes, mm_moves;  // Stages 3-5
     DevBuf capbuf;  // Stage 2: (t, E) of every DP row at the special row's column
     DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
     HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
@@ -350,7 +351,8 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->side) cudaStreamSynchronize(ctx->side);
-    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg, &ctx->capbuf})
+    for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg, &ctx->capbuf, &ctx->mm_parts,
+                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves})
         if (b->p) cudaFree(b->p);
     for (int s = 0; s < MAX_STRIPES; s++) {
         for (DevBuf *b : {&ctx->rowb[s], &ctx->progress[s], &ctx->sp[s]})
@@ -1350,4 +1352,191 @@ extern "C" int sw_stage2_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const ch
     begin_stats(ctx);
     return stage2_common(ctx, (const unsigned char *)dseqA, m, (const unsigned char *)dseqB, n, match, mismatch,
                          gap_open, gap_ext, special_row_interval, end, (cudaStream_t)stream, out, cap, count);
+}
+
+// ---------------------------------------------------------------- Stages 3-5 (N2/N3)
+
+#include "sw_mm.cuh"
+
+static int noop_sink(void *, int64_t, const int32_t *, const int32_t *, int64_t) { return 0; }
+
+// Stages 3-5: from the crosspoints L_2 of Stage 2,
+// split every partition larger than MM_TB_CELLS by Myers-Miller with balanced
+// splitting on the GPU (one warp per partition, one launch per level), then
+// align every small partition with a full traceback (one warp each, one
+// launch) and concatenate.  The GAP_1 / GAP_2 lists are the maximal
+// runs of the concatenated moves.
+static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const unsigned char *dB, int64_t n,
+                        int32_t ma, int32_t mi, int32_t go, int32_t ge, int64_t k, cudaStream_t us,
+                        sw_alignment *out, sw_gap *gap1, int64_t cap1, sw_gap *gap2, int64_t cap2)
+{
+    cudaStream_t st = us ? us : ctx->stream;
+    sw_result best{};
+    int rc = stage1_common(ctx, dA, m, dB, n, ma, mi, go, ge, k, k > 0 ? noop_sink : nullptr, nullptr, us, &best);
+    if (rc) return rc;
+    *out = sw_alignment{};
+    out->score = best.score;
+    if (best.score == 0) return SW_OK;
+    // Stage 2: crosspoints on the special rows
+    std::vector<sw_crosspoint> L(64);
+    int64_t cnt = 0;
+    for (;;) {
+        rc = stage2_common(ctx, dA, m, dB, n, ma, mi, go, ge, k, &best, us, L.data(), (int64_t)L.size(), &cnt);
+        if (rc == SW_ERANGE && cnt > (int64_t)L.size()) { L.resize((size_t)cnt); continue; }
+        if (rc) return rc;
+        break;
+    }
+    L.resize((size_t)cnt);
+    std::vector<MMPart> parts;
+    for (size_t q = 0; q + 1 < L.size(); q++) {
+        MMPart p{};
+        p.i_s = (int)L[q].i; p.j_s = (int)L[q].j; p.i_e = (int)L[q + 1].i; p.j_e = (int)L[q + 1].j;
+        p.t_s = L[q].type; p.t_e = L[q + 1].type;
+        p.score = L[q + 1].score - L[q].score;
+        parts.push_back(p);
+    }
+    MMArgs g{};
+    g.A = dA; g.B = dB;
+    g.ma = ma; g.mi = mi; g.go = go; g.ge = ge; g.gf = go + ge;
+    auto cells = [](const MMPart &p) { return (long long)(p.i_e - p.i_s) * (long long)(p.j_e - p.j_s); };
+    const int WPB = 8;  // warps per block
+    // Stage 3/4: balanced Myers-Miller splitting until every partition is small
+    int levels = 0;
+    for (;; levels++) {
+        std::vector<size_t> big;
+        long long scr = 0;
+        for (size_t q = 0; q < parts.size(); q++)
+            if (cells(parts[q]) > MM_TB_CELLS) {
+                big.push_back(q);
+                const long long wd = std::min(parts[q].i_e - parts[q].i_s, parts[q].j_e - parts[q].j_s);
+                parts[q].off = scr;
+                scr += 3 * (wd + 1);
+            }
+        if (big.empty()) break;
+        std::vector<MMPart> bp(big.size());
+        for (size_t q = 0; q < big.size(); q++) bp[q] = parts[big[q]];
+        if ((rc = grow(ctx, ctx->mm_parts, bp.size() * sizeof(MMPart)))) return rc;
+        if ((rc = grow(ctx, ctx->mm_scratch, (size_t)scr * sizeof(int2)))) return rc;
+        if ((rc = grow(ctx, ctx->mm_res, bp.size() * sizeof(MMRes)))) return rc;
+        CK(cudaMemcpyAsync(ctx->mm_parts.p, bp.data(), bp.size() * sizeof(MMPart), cudaMemcpyHostToDevice, st));
+        g.nparts = (int)bp.size();
+        g.parts = (const MMPart *)ctx->mm_parts.p;
+        g.scratch = (int2 *)ctx->mm_scratch.p;
+        g.res = (MMRes *)ctx->mm_res.p;
+        sw_mm_split_kernel<<<(g.nparts + WPB - 1) / WPB, 32 * WPB, 0, st>>>(g);
+        CK(cudaGetLastError());
+        ctx->stats.kernel_launches++;
+        std::vector<MMRes> res(bp.size());
+        CK(cudaMemcpyAsync(res.data(), ctx->mm_res.p, res.size() * sizeof(MMRes), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        std::vector<MMPart> next;
+        size_t bi = 0;
+        for (size_t q = 0; q < parts.size(); q++) {
+            if (bi < big.size() && big[bi] == q) {
+                const MMRes &r = res[bi++];
+                if (r.type < 0) {
+                    snprintf(ctx->errbuf, sizeof(ctx->errbuf), "Myers-Miller split found no junction (partition %zu)", q);
+                    return SW_ENOTFOUND;
+                }
+                MMPart a = parts[q], b = parts[q];
+                a.i_e = r.i; a.j_e = r.j; a.t_e = r.type; a.score = r.sub;
+                b.i_s = r.i; b.j_s = r.j; b.t_s = r.type; b.score = parts[q].score - r.sub;
+                next.push_back(a);
+                next.push_back(b);
+            } else {
+                next.push_back(parts[q]);
+            }
+        }
+        parts.swap(next);
+        if (levels > 128) return SW_ECUDA;
+    }
+    // Stage 5: full traceback of every (small) partition
+    long long oc = 0, om = 0, os = 0;
+    for (MMPart &p : parts) {
+        const long long h = p.i_e - p.i_s, w = p.j_e - p.j_s;
+        p.off_c = oc;
+        p.off_m = om;
+        p.off = os;
+        oc += (w + 1) * ((h + 7) / 8);
+        om += h + w;
+        os += w + 1;
+    }
+    if ((rc = grow(ctx, ctx->mm_parts, parts.size() * sizeof(MMPart)))) return rc;
+    if ((rc = grow(ctx, ctx->mm_scratch, (size_t)std::max(1ll, os) * sizeof(int2)))) return rc;
+    if ((rc = grow(ctx, ctx->mm_codes, (size_t)std::max(1ll, oc) * sizeof(unsigned int)))) return rc;
+    if ((rc = grow(ctx, ctx->mm_moves, (size_t)std::max(1ll, om)))) return rc;
+    if ((rc = grow(ctx, ctx->mm_res, parts.size() * sizeof(int)))) return rc;
+    CK(cudaMemcpyAsync(ctx->mm_parts.p, parts.data(), parts.size() * sizeof(MMPart), cudaMemcpyHostToDevice, st));
+    g.nparts = (int)parts.size();
+    g.parts = (const MMPart *)ctx->mm_parts.p;
+    g.scratch = (int2 *)ctx->mm_scratch.p;
+    g.codes = (unsigned int *)ctx->mm_codes.p;
+    g.moves = (char *)ctx->mm_moves.p;
+    g.nmoves = (int *)ctx->mm_res.p;
+    sw_mm_tb_kernel<<<(g.nparts + WPB - 1) / WPB, 32 * WPB, 0, st>>>(g);
+    CK(cudaGetLastError());
+    ctx->stats.kernel_launches++;
+    std::vector<char> mv((size_t)std::max(1ll, om));
+    std::vector<int> nm(parts.size());
+    CK(cudaMemcpyAsync(mv.data(), ctx->mm_moves.p, (size_t)om, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(nm.data(), ctx->mm_res.p, nm.size() * sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    // concatenate and run-length encode into GAP_1 (gaps in S0) / GAP_2 (gaps in S1)
+    out->i0 = L.front().i; out->j0 = L.front().j;
+    out->i1 = best.i; out->j1 = best.j;
+    out->partitions = (int64_t)parts.size();
+    out->mm_levels = levels;
+    int64_t i = out->i0, j = out->j0, n1 = 0, n2 = 0;
+    char prev = 0;
+    for (size_t q = 0; q < parts.size(); q++) {
+        const MMPart &p = parts[q];
+        const long long len = (long long)(p.i_e - p.i_s) + (p.j_e - p.j_s);
+        const char *s = mv.data() + p.off_m + (len - nm[q]);
+        for (int x = 0; x < nm[q]; x++) {
+            const char c = s[x];
+            if (c == 'I') {
+                if (prev == 'I') { if (n1 <= cap1 && n1 > 0) gap1[n1 - 1].len++; }
+                else { if (n1 < cap1) gap1[n1] = sw_gap{i, j, 1}; n1++; }
+                j++;
+            } else if (c == 'D') {
+                if (prev == 'D') { if (n2 <= cap2 && n2 > 0) gap2[n2 - 1].len++; }
+                else { if (n2 < cap2) gap2[n2] = sw_gap{i, j, 1}; n2++; }
+                i++;
+            } else {
+                i++;
+                j++;
+            }
+            prev = c;
+        }
+    }
+    out->n_gap1 = n1;
+    out->n_gap2 = n2;
+    if (i != out->i1 || j != out->j1) {
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "alignment ends at (%lld, %lld), expected (%lld, %lld)",
+                 (long long)i, (long long)j, (long long)out->i1, (long long)out->j1);
+        return SW_ECUDA;
+    }
+    return (n1 > cap1 || n2 > cap2) ? SW_ERANGE : SW_OK;
+}
+
+extern "C" int sw_align(sw_ctx *ctx, const char *seqA, int64_t m, const char *seqB, int64_t n, int32_t match,
+                        int32_t mismatch, int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
+                        sw_alignment *out, sw_gap *gap1, int64_t cap1, sw_gap *gap2, int64_t cap2)
+{
+    if (!ctx || !out || m < 0 || n < 0 || special_row_interval < 0 || cap1 < 0 || cap2 < 0) return SW_EINVAL;
+    if ((cap1 > 0 && !gap1) || (cap2 > 0 && !gap2)) return SW_EINVAL;
+    if (m >= (1ll << 31) - (1 << 16) || n >= (1ll << 31) - (1 << 16)) return SW_EINVAL;
+    if ((m && !seqA) || (n && !seqB)) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    *out = sw_alignment{};
+    if (m == 0 || n == 0) return SW_OK;
+    if ((rc = upload(ctx, seqA, m, seqB, n))) return rc;
+    rc = align_common(ctx, (const unsigned char *)ctx->seq.p, m, (const unsigned char *)ctx->seq.p + m, n, match,
+                      mismatch, gap_open, gap_ext, special_row_interval, nullptr, out, gap1, cap1, gap2, cap2);
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return rc;
 }
