@@ -177,6 +177,7 @@ typedef struct {
     int64_t i0, j0, i1, j1;
     int64_t n_gap1, n_gap2;
     int64_t partitions, mm_levels;
+    double ms_stage1, ms_stage2, ms_mm, ms_stage5;  /* host wall time per stage (Stages 3-4 = ms_mm) */
 } sw_alignment;
 
 /* Stages 1-5: the full optimal local alignment of S0 and S1.

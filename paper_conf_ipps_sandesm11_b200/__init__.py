@@ -76,7 +76,8 @@ class _Gap(ctypes.Structure):
 class _Alignment(ctypes.Structure):
     _fields_ = [("score", ctypes.c_int32), ("i0", ctypes.c_int64), ("j0", ctypes.c_int64), ("i1", ctypes.c_int64),
                 ("j1", ctypes.c_int64), ("n_gap1", ctypes.c_int64), ("n_gap2", ctypes.c_int64),
-                ("partitions", ctypes.c_int64), ("mm_levels", ctypes.c_int64)]
+                ("partitions", ctypes.c_int64), ("mm_levels", ctypes.c_int64), ("ms_stage1", ctypes.c_double),
+                ("ms_stage2", ctypes.c_double), ("ms_mm", ctypes.c_double), ("ms_stage5", ctypes.c_double)]
 
 
 class Stats(ctypes.Structure):
@@ -324,7 +325,9 @@ class Context:
         return {"score": out.score, "start": (out.i0, out.j0), "end": (out.i1, out.j1),
                 "gap1": [(g.i, g.j, g.len) for g in g1[: out.n_gap1]],
                 "gap2": [(g.i, g.j, g.len) for g in g2[: out.n_gap2]],
-                "partitions": out.partitions, "mm_levels": out.mm_levels}
+                "partitions": out.partitions, "mm_levels": out.mm_levels,
+                "ms": {"stage1": out.ms_stage1, "stage2": out.ms_stage2, "stages3_4": out.ms_mm,
+                       "stage5": out.ms_stage5}}
 
     def row_granularity(self) -> int:
         return int(self._lib.sw_row_granularity(self._h))

@@ -858,7 +858,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         }
         return SW_OK;
     };
-    long long done = 0;
+    long long done = J.sink ? 0 : nsp;  // no sink (sw_align): the rows stay in HBM only
     while (done < nsp) {
         bool progress = false;
         if (dbg_host && h_fill < 0 && cudaEventQuery(ctx->ev[2]) == cudaSuccess) h_fill = hms();
@@ -1358,8 +1358,6 @@ extern "C" int sw_stage2_dev(sw_ctx *ctx, const char *dseqA, int64_t m, const ch
 
 #include "sw_mm.cuh"
 
-static int noop_sink(void *, int64_t, const int32_t *, const int32_t *, int64_t) { return 0; }
-
 // Stages 3-5: from the crosspoints L_2 of Stage 2,
 // split every partition larger than MM_TB_CELLS by Myers-Miller with balanced
 // splitting on the GPU (one warp per partition, one launch per level), then
@@ -1372,10 +1370,17 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
 {
     cudaStream_t st = us ? us : ctx->stream;
     sw_result best{};
-    int rc = stage1_common(ctx, dA, m, dB, n, ma, mi, go, ge, k, k > 0 ? noop_sink : nullptr, nullptr, us, &best);
+    auto tnow = std::chrono::steady_clock::now;
+    auto ms = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+        return std::chrono::duration<double, std::milli>(b - a).count();
+    };
+    const auto t0 = tnow();
+    // Stage 1; the special rows stay resident in HBM for Stage 2 (no host sink)
+    int rc = stage1_common(ctx, dA, m, dB, n, ma, mi, go, ge, k, nullptr, nullptr, us, &best);
     if (rc) return rc;
     *out = sw_alignment{};
     out->score = best.score;
+    out->ms_stage1 = ms(t0, tnow());
     if (best.score == 0) return SW_OK;
     // Stage 2: crosspoints on the special rows
     std::vector<sw_crosspoint> L(64);
@@ -1387,6 +1392,8 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
         break;
     }
     L.resize((size_t)cnt);
+    const auto t2 = tnow();
+    out->ms_stage2 = ms(t0, t2) - out->ms_stage1;
     std::vector<MMPart> parts;
     for (size_t q = 0; q + 1 < L.size(); q++) {
         MMPart p{};
@@ -1450,6 +1457,8 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
         parts.swap(next);
         if (levels > 128) return SW_ECUDA;
     }
+    const auto t3 = tnow();
+    out->ms_mm = ms(t2, t3);
     // Stage 5: full traceback of every (small) partition
     long long oc = 0, om = 0, os = 0;
     for (MMPart &p : parts) {
@@ -1511,6 +1520,7 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
     }
     out->n_gap1 = n1;
     out->n_gap2 = n2;
+    out->ms_stage5 = ms(t3, tnow());
     if (i != out->i1 || j != out->j1) {
         snprintf(ctx->errbuf, sizeof(ctx->errbuf), "alignment ends at (%lld, %lld), expected (%lld, %lld)",
                  (long long)i, (long long)j, (long long)out->i1, (long long)out->j1);
