@@ -207,7 +207,7 @@ struct sw_ctx {
     std::vector<cudaEvent_t> ev_row;  // one per staging slot: the slot's final copy is done
     int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
-    DevBuf mm_parts, mm_scratch, mm_res, mm_codes, mm_moves;  // Stages 3-5
+    DevBuf mm_parts, mm_scratch, mm_res, mm_codes, mm_moves, mm_err;  // Stages 3-5
     DevBuf capbuf;  // Stage 2: (t, E) of every DP row at the special row's column
     DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
     HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
@@ -352,7 +352,7 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->side) cudaStreamSynchronize(ctx->side);
     for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg, &ctx->capbuf, &ctx->mm_parts,
-                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves})
+                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves, &ctx->mm_err})
         if (b->p) cudaFree(b->p);
     for (int s = 0; s < MAX_STRIPES; s++) {
         for (DevBuf *b : {&ctx->rowb[s], &ctx->progress[s], &ctx->sp[s]})
@@ -1407,40 +1407,81 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
     g.ma = ma; g.mi = mi; g.go = go; g.ge = ge; g.gf = go + ge;
     auto cells = [](const MMPart &p) { return (long long)(p.i_e - p.i_s) * (long long)(p.j_e - p.j_s); };
     const int WPB = 8;  // warps per block
-    // Stage 3/4: balanced Myers-Miller splitting until every partition is small
+    if ((rc = grow(ctx, ctx->mm_err, sizeof(int)))) return rc;
+    CK(cudaMemsetAsync(ctx->mm_err.p, 0, sizeof(int), st));
+    g.err = (int *)ctx->mm_err.p;
+    g.timeout_ns = ctx->timeout_ns;
+    // Stage 3/4: balanced Myers-Miller splitting until every partition is small.
+    // Partitions whose split line is at least MM_CTA_ROWS away from C_s go to the
+    // CTA kernel (MM_NWP warps on the chunks), the rest one warp each.
+    long long MM_CTA_ROWS = 4ll * MM_CHUNK;
+    if (const char *e = getenv("SWB_MM_CTA_ROWS")) MM_CTA_ROWS = atoll(e);  // tuning
     int levels = 0;
     for (;; levels++) {
         std::vector<size_t> big;
-        long long scr = 0;
         for (size_t q = 0; q < parts.size(); q++)
-            if (cells(parts[q]) > MM_TB_CELLS) {
-                big.push_back(q);
-                const long long wd = std::min(parts[q].i_e - parts[q].i_s, parts[q].j_e - parts[q].j_s);
-                parts[q].off = scr;
-                scr += 3 * (wd + 1);
-            }
+            if (cells(parts[q]) > MM_TB_CELLS) big.push_back(q);
         if (big.empty()) break;
-        std::vector<MMPart> bp(big.size());
-        for (size_t q = 0; q < big.size(); q++) bp[q] = parts[big[q]];
+        // CTA partitions first (blocks 0..ncta-1), then warp partitions
+        std::vector<MMPart> bp;
+        std::vector<size_t> order;
+        long long scr = 0;
+        int ncta = 0;
+        for (int pass = 0; pass < 2; pass++)
+            for (size_t q : big) {
+                const MMPart &P = parts[q];
+                const long long hh = P.i_e - P.i_s, ww = P.j_e - P.j_s;
+                const long long H = std::max(hh, ww), Wd = std::min(hh, ww);
+                const bool cta = H / 2 >= MM_CTA_ROWS;
+                if (cta != (pass == 0)) continue;
+                MMPart c = P;
+                c.off = scr;
+                scr += (cta ? (MM_NWP + 3) : 3) * (Wd + 1);
+                bp.push_back(c);
+                order.push_back(q);
+                ncta += cta;
+            }
         if ((rc = grow(ctx, ctx->mm_parts, bp.size() * sizeof(MMPart)))) return rc;
         if ((rc = grow(ctx, ctx->mm_scratch, (size_t)scr * sizeof(int2)))) return rc;
         if ((rc = grow(ctx, ctx->mm_res, bp.size() * sizeof(MMRes)))) return rc;
         CK(cudaMemcpyAsync(ctx->mm_parts.p, bp.data(), bp.size() * sizeof(MMPart), cudaMemcpyHostToDevice, st));
-        g.nparts = (int)bp.size();
-        g.parts = (const MMPart *)ctx->mm_parts.p;
         g.scratch = (int2 *)ctx->mm_scratch.p;
-        g.res = (MMRes *)ctx->mm_res.p;
-        sw_mm_split_kernel<<<(g.nparts + WPB - 1) / WPB, 32 * WPB, 0, st>>>(g);
-        CK(cudaGetLastError());
-        ctx->stats.kernel_launches++;
-        std::vector<MMRes> res(bp.size());
-        CK(cudaMemcpyAsync(res.data(), ctx->mm_res.p, res.size() * sizeof(MMRes), cudaMemcpyDeviceToHost, st));
+        if (ncta > 0) {
+            g.nparts = ncta;
+            g.parts = (const MMPart *)ctx->mm_parts.p;
+            g.res = (MMRes *)ctx->mm_res.p;
+            sw_mm_split_cta_kernel<<<ncta, 32 * MM_NWP, 0, st>>>(g);
+            CK(cudaGetLastError());
+            ctx->stats.kernel_launches++;
+        }
+        if ((int)bp.size() > ncta) {
+            g.nparts = (int)bp.size() - ncta;
+            g.parts = (const MMPart *)ctx->mm_parts.p + ncta;
+            g.res = (MMRes *)ctx->mm_res.p + ncta;
+            sw_mm_split_kernel<<<(g.nparts + WPB - 1) / WPB, 32 * WPB, 0, st>>>(g);
+            CK(cudaGetLastError());
+            ctx->stats.kernel_launches++;
+        }
+        std::vector<MMRes> resv(bp.size());
+        int merr = 0;
+        CK(cudaMemcpyAsync(resv.data(), ctx->mm_res.p, resv.size() * sizeof(MMRes), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(&merr, ctx->mm_err.p, sizeof(int), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
+        if (merr) {
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "Myers-Miller split: spin-wait timeout");
+            return SW_ECUDA;
+        }
+        if (getenv("SWB_DEBUG_HOST"))
+            fprintf(stderr, "[swb mm] level %d: %zu partitions split (%d on CTAs), t=%.1f ms\n", levels, bp.size(),
+                    ncta, ms(t2, tnow()));
+        std::vector<MMRes> res(parts.size());
+        for (size_t q = 0; q < order.size(); q++) res[order[q]] = resv[q];
         std::vector<MMPart> next;
         size_t bi = 0;
         for (size_t q = 0; q < parts.size(); q++) {
             if (bi < big.size() && big[bi] == q) {
-                const MMRes &r = res[bi++];
+                bi++;
+                const MMRes &r = res[q];
                 if (r.type < 0) {
                     snprintf(ctx->errbuf, sizeof(ctx->errbuf), "Myers-Miller split found no junction (partition %zu)", q);
                     return SW_ENOTFOUND;

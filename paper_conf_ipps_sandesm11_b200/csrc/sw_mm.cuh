@@ -59,6 +59,8 @@ struct MMArgs {
     unsigned int *codes;
     char *moves;
     int *nmoves;
+    int *err;            // set to 2 when a spin-wait times out (watchdog)
+    long long timeout_ns;
 };
 
 // A global DP problem of h x w cells: row a (1..h) pairs rs[a * rstep],
@@ -167,6 +169,173 @@ __device__ void mm_warp_dp(const MMArgs &g, const DpProb &P, int2 *rowbuf, int c
         }
         __threadfence_block();
         __syncwarp();
+    }
+}
+
+// CTA version of the MODE-0 pass for large partitions: the NWP warps take the
+// 256-row chunks round robin (chunk c on warp c % NWP).  Chunk c reads its top
+// row from ring slot c % (NWP+1), written by chunk c-1, and writes its bottom
+// row to slot (c+1) % (NWP+1); the writer publishes (generation, columns) in
+// shared memory every 32 columns (after __threadfence_block), the reader's
+// lane 0 waits for it before each 32-column prefetch and loads through L2
+// (__ldcg).  A slot is reused by the same warp NWP chunks later, after its
+// reader (the next warp) is done with it.  Same arithmetic as mm_warp_dp.
+template <int NWP>
+__device__ void mm_cta_pass(const MMArgs &g, const DpProb &P, int2 *ring, long long rs, int capR, int2 *cap,
+                            volatile int *s_gen, volatile int *s_cols, int warp, int lane)
+{
+    constexpr int R = NWP + 1;
+    const int h = P.h, w = P.w, kind = P.kind;
+    for (int b = threadIdx.x; b <= w; b += blockDim.x) {
+        const int2 v = make_int2(b == 0 ? 0 : mm_row0(g, kind, b), (b == 0 && kind == 2) ? 0 : NEG);
+        ring[b] = v;
+        if (capR == 0) cap[b] = v;
+    }
+    if (threadIdx.x < R) {
+        s_gen[threadIdx.x] = threadIdx.x == 0 ? -1 : -2;
+        s_cols[threadIdx.x] = threadIdx.x == 0 ? w : 0;
+    }
+    if (capR > 0 && threadIdx.x == 0) cap[0] = make_int2(mm_col0(g, kind, capR), mm_col0(g, kind, capR));
+    __syncthreads();
+    const int diag00 = (kind == 3 || kind == 4) ? NEG : 0;
+    const int nchunks = (capR + MM_CHUNK - 1) / MM_CHUNK;
+    for (int c = warp; c < nchunks; c += NWP) {
+        const int a0 = c * MM_CHUNK;
+        const int in = c % R, out = (c + 1) % R;
+        const int2 *rin = ring + in * rs;
+        int2 *rout = ring + out * rs;
+        if (lane == 0) {
+            s_cols[out] = 0;
+            __threadfence_block();
+            s_gen[out] = c;
+        }
+        __syncwarp();
+        auto wait_cols = [&](int need) {
+            need = min(need, w);
+            if (lane == 0 && (s_gen[in] != c - 1 || s_cols[in] < need)) {
+                const unsigned long long t0 = gtimer();
+                while (s_gen[in] != c - 1 || s_cols[in] < need) {
+                    __nanosleep(32);
+                    if (gtimer() - t0 > (unsigned long long)g.timeout_ns) { atomicExch(g.err, 2); break; }
+                }
+            }
+            __syncwarp();
+            __threadfence_block();
+        };
+        const int r0 = a0 + lane * MM_ALPHA;
+        int rc[MM_ALPHA], Hp[MM_ALPHA], Ep[MM_ALPHA];
+#pragma unroll
+        for (int r = 0; r < MM_ALPHA; r++) {
+            const int a = r0 + r + 1;
+            rc[r] = a <= h ? mm_up(P.rs[(long long)a * P.rstep]) : 0x100;
+            Hp[r] = mm_col0(g, kind, a);
+            Ep[r] = NEG;
+        }
+        int hdiag = r0 == 0 ? diag00 : mm_col0(g, kind, r0);
+        int hu = 0, fu = 0;
+        wait_cols(64);
+        int2 cur = (1 + lane <= w) ? __ldcg(rin + 1 + lane) : make_int2(NEG, NEG);
+        int2 nxt = (33 + lane <= w) ? __ldcg(rin + 33 + lane) : make_int2(NEG, NEG);
+        int capH = 0, capF = 0;
+        const int nsteps = w + 31;
+        for (int k = 0; k < nsteps; k++) {
+            if (k > 0 && (k & 31) == 0) {
+                cur = nxt;
+                wait_cols(k + 64);
+                const int cc2 = k + 33 + lane;
+                nxt = cc2 <= w ? __ldcg(rin + cc2) : make_int2(NEG, NEG);
+            }
+            int upH = __shfl_up_sync(0xffffffffu, hu, 1);
+            int upF = __shfl_up_sync(0xffffffffu, fu, 1);
+            const int rH = __shfl_sync(0xffffffffu, cur.x, k & 31);
+            const int rF = __shfl_sync(0xffffffffu, cur.y, k & 31);
+            if (lane == 0) { upH = rH; upF = rF; }
+            const int b = k - lane + 1;
+            if (b >= 1 && b <= w) {
+                const int cc = mm_up(P.cs[(long long)b * P.cstep]);
+                int hd = hdiag;
+                hdiag = upH;
+#pragma unroll
+                for (int r = 0; r < MM_ALPHA; r++) {
+                    const int e = max(Ep[r] - g.ge, Hp[r] - g.gf);   // Eq. 2
+                    const int f = max(upF - g.ge, upH - g.gf);       // Eq. 3
+                    const int d = hd + (rc[r] == cc ? g.ma : g.mi);  // Eq. 1 (no 0 term)
+                    const int hv = max(max(e, f), d);
+                    if (r0 + r + 1 == capR) { capH = hv; capF = f; }
+                    hd = Hp[r];
+                    Hp[r] = max(hv, NEG);
+                    Ep[r] = max(e, NEG);
+                    upH = Hp[r];
+                    upF = max(f, NEG);
+                }
+                hu = upH;
+                fu = upF;
+                if (capR > r0 && capR <= r0 + MM_ALPHA) cap[b] = make_int2(capH, capF);
+                if (lane == 31) rout[b] = make_int2(hu, fu);
+            }
+            if ((k & 31) == 31 || k == nsteps - 1) {
+                __threadfence_block();
+                __syncwarp();
+                if (lane == 31) s_cols[out] = min(w, k - 30);
+            }
+        }
+    }
+    __syncthreads();
+}
+
+constexpr int MM_NWP = 8;  // warps per partition in the CTA split kernel
+
+// One CTA of MM_NWP warps per (large) partition: split it at the middle of
+// its larger dimension.  Same orientation, passes and junction rule as
+// sw_mm_split_kernel.
+__global__ void __launch_bounds__(32 * MM_NWP) sw_mm_split_cta_kernel(const __grid_constant__ MMArgs g)
+{
+    __shared__ int s_gen[MM_NWP + 1], s_cols[MM_NWP + 1];
+    __shared__ unsigned long long s_key;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int p = blockIdx.x;
+    if (p >= g.nparts) return;
+    const MMPart Pt = g.parts[p];
+    const bool tr = (Pt.j_e - Pt.j_s) > (Pt.i_e - Pt.i_s);
+    const unsigned char *X = tr ? g.B : g.A, *Y = tr ? g.A : g.B;
+    const int xs = tr ? Pt.j_s : Pt.i_s, xe = tr ? Pt.j_e : Pt.i_e;
+    const int ys = tr ? Pt.i_s : Pt.j_s, ye = tr ? Pt.i_e : Pt.j_e;
+    auto sw12 = [&](int t) { return tr ? (t == 1 ? 2 : t == 2 ? 1 : 0) : t; };
+    const int ts = sw12(Pt.t_s), te = sw12(Pt.t_e);
+    const int H = xe - xs, Wd = ye - ys, mid = H / 2;
+    const long long rsz = Wd + 1;
+    int2 *ring = g.scratch + Pt.off;
+    int2 *capf = ring + (MM_NWP + 1) * rsz;
+    int2 *capr = capf + rsz;
+    DpProb F{X + xs - 1, Y + ys - 1, 1, 1, mid, Wd, ts};
+    mm_cta_pass<MM_NWP>(g, F, ring, rsz, mid, capf, s_gen, s_cols, warp, lane);
+    DpProb R{X + xe, Y + ye, -1, -1, H - mid, Wd, te == 2 ? 3 : te == 1 ? 4 : 0};
+    mm_cta_pass<MM_NWP>(g, R, ring, rsz, H - mid, capr, s_gen, s_cols, warp, lane);
+    if (threadIdx.x == 0) s_key = 0ull;
+    __syncthreads();
+    long long key = -1;
+    for (int b = threadIdx.x; b <= Wd; b += blockDim.x) {
+        const int2 f = __ldcg(capf + b), r = __ldcg(capr + Wd - b);
+        if (f.x > NEG / 2 && r.x > NEG / 2 && f.x + r.x == Pt.score) key = max(key, 2ll * b + 1);
+        else if (f.y > NEG / 2 && r.y > NEG / 2 && f.y + r.y + g.go == Pt.score) key = max(key, 2ll * b);
+    }
+    for (int o = 16; o > 0; o >>= 1) key = max(key, __shfl_xor_sync(0xffffffffu, key, o));
+    if (lane == 0 && key >= 0) atomicMax(&s_key, (unsigned long long)(key + 1));
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        MMRes out{0, 0, -1, 0};
+        const long long k2 = (long long)s_key - 1;
+        if (k2 >= 0) {
+            const int b = (int)(k2 >> 1);
+            const bool hj = k2 & 1;
+            const int2 f = __ldcg(capf + b);
+            const int x = xs + mid, y = ys + b;
+            out.i = tr ? y : x;
+            out.j = tr ? x : y;
+            out.type = hj ? 0 : (tr ? 1 : 2);
+            out.sub = hj ? f.x : f.y;
+        }
+        g.res[p] = out;
     }
 }
 

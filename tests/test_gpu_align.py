@@ -105,6 +105,15 @@ def test_align_forces_myers_miller_splits(ctx, sc):
     check(ctx, B, A, sc, 256, want_levels=1)
 
 
+def test_align_cta_split_many_chunks(ctx):
+    # 12000-row partitions: the CTA split kernel runs 6000-row passes as 24 chunks on 8 warps
+    # (ring slots reused), in rows and -- for the transposed pair -- in columns
+    A, B = synth.random_pair(91, 12000, 3000, plant_len=3000, s=0.02, g=0.01)
+    A = A[:]
+    check(ctx, A, B, PAPER, 0, want_levels=3)
+    check(ctx, B, A, (2, -1, 4, 1), 0, want_levels=3)
+
+
 def test_align_long_gaps(ctx):
     rng = np.random.default_rng(5)
     X = "".join(rng.choice(list("ACGT"), 2500))

@@ -1,3 +1,3 @@
-set -x
-timeout 900 python -m pytest tests/test_gpu_align.py tests/test_gpu_stage2.py -x -q 2>&1 | tail -3
-timeout 900 python tools/align_bench.py C1 C2 C4 C3
+python tools/mm_bench.py 20000
+SWB_MM_CTA_ROWS=100000000 python tools/mm_bench.py 20000
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:sw_mm_split_cta -c 1 -o gpurun_out/mm_cta -f python tools/mm_bench.py 20000 > gpurun_out/ncu_mm.log 2>&1
