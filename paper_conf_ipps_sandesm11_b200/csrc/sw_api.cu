@@ -1405,6 +1405,11 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
     MMArgs g{};
     g.A = dA; g.B = dB;
     g.ma = ma; g.mi = mi; g.go = go; g.ge = ge; g.gf = go + ge;
+    for (int x = 0; x < 4; x++) {
+        uint32_t wv = 0;
+        for (int y = 0; y < 4; y++) wv |= (uint32_t)(uint8_t)(int8_t)((x == y ? ma : mi) + g.gf) << (8 * y);
+        g.prof[x] = wv;
+    }
     auto cells = [](const MMPart &p) { return (long long)(p.i_e - p.i_s) * (long long)(p.j_e - p.j_s); };
     const int WPB = 8;  // warps per block
     if ((rc = grow(ctx, ctx->mm_err, sizeof(int)))) return rc;

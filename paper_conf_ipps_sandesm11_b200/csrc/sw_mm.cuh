@@ -52,6 +52,7 @@ struct MMRes {
 struct MMArgs {
     const unsigned char *A, *B;  // ASCII S0, S1 (0-based; DP row i pairs A[i - 1])
     int ma, mi, go, ge, gf;
+    uint32_t prof[4];    // row code a -> int8x4 word, byte x = (a == x ? ma : mi) + G_first
     int nparts;
     const MMPart *parts;
     int2 *scratch;
@@ -87,18 +88,113 @@ __device__ __forceinline__ int mm_col0(const MMArgs &g, int kind, int a)  // H(a
 }
 __device__ __forceinline__ int mm_up(unsigned char c) { return c & 0xDF; }  // ASCII upper case (ACGT only)
 
-// MODE 0: run rows 1..capR and store H, F of row capR (columns 0..w) in cap.
-// MODE 1: run all rows and store the 4-bit traceback code of every cell:
-//   bits 0-1 H source (0 diagonal, 1 F, 2 E; ties prefer that order),
-//   bit 2 E extends (E(a,b-1) - G_ext >= H(a,b-1) - G_first), bit 3 F extends.
-//   Layout: codes[b * HW + (a - 1) / 8], nibble (a - 1) % 8, HW = ceil(h / 8).
+// 2-bit code of an ASCII base, case-insensitive: A/a 0, C/c 1, T/t 2, G/g 3.
+__device__ __forceinline__ uint32_t mm_code(unsigned char c) { return (c >> 1) & 3u; }
+
+// One chunk of MM_CHUNK rows starting at row a0 + 1, swept over columns 1..w.
+// The row above comes from rin (H, F per column; lane 0 reads it through a
+// 32-column prefetch), the chunk's bottom row goes to rout (lane 31).  Lane
+// state: rows r0+1 .. r0+MM_ALPHA as t = H - G_first and E, the substitution
+// score p + G_first from an int8x4 profile word and one PRMT per cell (as the
+// band kernel): per cell E = max(E - G_ext, t_left), F = max(F_up - G_ext, t_up),
+// H = max(E, F, t_diag + (p + G_first)) (Eq. 1-3, no 0 term), t = H - G_first.
+//   MODE 0: H, F of row capR into cap[b].
+//   MODE 1: 4-bit traceback codes: bits 0-1 H source (0 diagonal, 1 F, 2 E;
+//     ties prefer that order), bit 2 E extends (E(a,b-1) - G_ext >= t(a,b-1)),
+//     bit 3 F extends; codes[b * HW + (a - 1) / 8], nibble (a - 1) % 8.
+// wait(need): block until rin holds columns 1..need (CTA pipeline; no-op for
+// one warp); publish(cols): rout holds columns 1..cols.
+template <int MODE, bool CAPC, class Wait, class Publish>
+__device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a0, const int2 *rin, int2 *rout,
+                                         int capR, int2 *cap, unsigned int *codes, int lane, Wait wait,
+                                         Publish publish)
+{
+    const int h = P.h, w = P.w, kind = P.kind;
+    const int HW = (h + 7) / 8;
+    const int gf = g.gf, nge = -g.ge;
+    const int r0 = a0 + lane * MM_ALPHA;  // this lane: rows r0 + 1 .. r0 + MM_ALPHA
+    uint32_t Pw[MM_ALPHA];
+    int T[MM_ALPHA], E[MM_ALPHA];
+#pragma unroll
+    for (int r = 0; r < MM_ALPHA; r++) {
+        const int a = r0 + r + 1;
+        Pw[r] = a <= h ? g.prof[mm_code(P.rs[(long long)a * P.rstep])] : PADPROF;
+        T[r] = mm_col0(g, kind, a) - gf;
+        E[r] = NEG;
+    }
+    const int diag00 = (kind == 3 || kind == 4) ? NEG : 0;
+    int tdiag = (r0 == 0 ? diag00 : mm_col0(g, kind, r0)) - gf;  // t(r0, b - 1)
+    int tu_out = 0, fu_out = 0;
+    const bool cap_lane = CAPC && capR > r0 && capR <= r0 + MM_ALPHA;  // CAPC: this chunk holds row capR
+    wait(64);
+    int2 cur = (1 + lane <= w) ? __ldcg(rin + 1 + lane) : make_int2(NEG, NEG);
+    int2 nxt = (33 + lane <= w) ? __ldcg(rin + 33 + lane) : make_int2(NEG, NEG);
+    const int nsteps = w + 31;
+    auto step = [&](int k, bool guard) {
+        int tu = __shfl_up_sync(0xffffffffu, tu_out, 1);
+        int fu = __shfl_up_sync(0xffffffffu, fu_out, 1);
+        const int rH = __shfl_sync(0xffffffffu, cur.x, k & 31);
+        const int rF = __shfl_sync(0xffffffffu, cur.y, k & 31);
+        if (lane == 0) { tu = rH - gf; fu = rF; }
+        const int b = k - lane + 1;
+        if (guard && (b < 1 || b > w)) return;
+        const uint32_t sel = col_sel(mm_code(P.cs[(long long)b * P.cstep]));
+        int td = tdiag;
+        tdiag = tu;
+        unsigned int code = 0;
+        int capH = 0, capF = 0;
+#pragma unroll
+        for (int r = 0; r < MM_ALPHA; r++) {
+            const int e = __viaddmax_s32(E[r], nge, T[r]);   // Eq. 2
+            const int f = __viaddmax_s32(fu, nge, tu);       // Eq. 3
+            const int x = td + prmt(Pw[r], PADPROF, sel);    // H_diag + p
+            const int hv = __vimax3_s32(e, f, x);            // Eq. 1 (global: no 0 term)
+            if (MODE == 1) {
+                const unsigned int src = (x >= e && x >= f) ? 0u : (f >= e ? 1u : 2u);
+                const unsigned int ext = (E[r] + nge >= T[r] ? 4u : 0u) | (fu + nge >= tu ? 8u : 0u);
+                code |= (src | ext) << (4 * r);
+            }
+            if (CAPC && cap_lane && r0 + r + 1 == capR) { capH = hv; capF = f; }
+            td = T[r];
+            T[r] = hv - gf;
+            E[r] = e;
+            tu = T[r];
+            fu = f;
+        }
+        tu_out = tu;
+        fu_out = fu;
+        if (MODE == 1 && r0 < h) codes[(long long)b * HW + r0 / 8] = code;
+        if (CAPC && cap_lane) cap[b] = make_int2(capH, capF);
+        if (lane == 31) rout[b] = make_int2(tu + gf, fu);
+    };
+    for (int kb = 0; kb < nsteps; kb += 32) {
+        if (kb > 0) {
+            cur = nxt;
+            wait(kb + 64);
+            const int c = kb + 33 + lane;
+            nxt = c <= w ? __ldcg(rin + c) : make_int2(NEG, NEG);
+        }
+        if (kb >= 32 && kb + 32 <= w) {
+#pragma unroll 4
+            for (int u = 0; u < 32; u++) step(kb + u, false);
+        } else {
+            const int ke = min(kb + 32, nsteps);
+#pragma unroll 1
+            for (int k = kb; k < ke; k++) step(k, true);
+        }
+        publish(min(w, kb + 1));
+    }
+}
+
+// One warp runs the whole pass (chunks one after the other, row buffer in place).
+// MODE 0: rows 1..capR, H and F of row capR into cap (columns 0..w).
+// MODE 1: all rows, traceback codes.
 template <int MODE>
 __device__ void mm_warp_dp(const MMArgs &g, const DpProb &P, int2 *rowbuf, int capR, int2 *cap, unsigned int *codes,
                            int lane)
 {
-    const int h = P.h, w = P.w, kind = P.kind;
-    const int rows = MODE == 0 ? capR : h;
-    const int HW = (h + 7) / 8;
+    const int w = P.w, kind = P.kind;
+    const int rows = MODE == 0 ? capR : P.h;
     for (int b = lane; b <= w; b += 32) {
         const int2 v = make_int2(b == 0 ? 0 : mm_row0(g, kind, b), (b == 0 && kind == 2) ? 0 : NEG);
         rowbuf[b] = v;
@@ -107,66 +203,11 @@ __device__ void mm_warp_dp(const MMArgs &g, const DpProb &P, int2 *rowbuf, int c
     if (MODE == 0 && capR > 0 && lane == 0) cap[0] = make_int2(mm_col0(g, kind, capR), mm_col0(g, kind, capR));
     __threadfence_block();
     __syncwarp();
-    const int diag00 = (kind == 3 || kind == 4) ? NEG : 0;
     for (int a0 = 0; a0 < rows; a0 += MM_CHUNK) {
-        const int r0 = a0 + lane * MM_ALPHA;  // this lane: rows r0 + 1 .. r0 + MM_ALPHA
-        int rc[MM_ALPHA], Hp[MM_ALPHA], Ep[MM_ALPHA];
-#pragma unroll
-        for (int r = 0; r < MM_ALPHA; r++) {
-            const int a = r0 + r + 1;
-            rc[r] = a <= h ? mm_up(P.rs[(long long)a * P.rstep]) : 0x100;  // pad rows never match
-            Hp[r] = mm_col0(g, kind, a);
-            Ep[r] = NEG;
-        }
-        int hdiag = r0 == 0 ? diag00 : mm_col0(g, kind, r0);  // H(r0, b - 1) for the next column
-        int hu = 0, fu = 0;
-        int2 cur = (1 + lane <= w) ? rowbuf[1 + lane] : make_int2(NEG, NEG);
-        int2 nxt = (33 + lane <= w) ? rowbuf[33 + lane] : make_int2(NEG, NEG);
-        const int nsteps = w + 31;
-        for (int k = 0; k < nsteps; k++) {
-            if (k > 0 && (k & 31) == 0) {
-                cur = nxt;
-                const int c = k + 33 + lane;
-                nxt = c <= w ? rowbuf[c] : make_int2(NEG, NEG);
-            }
-            int upH = __shfl_up_sync(0xffffffffu, hu, 1);
-            int upF = __shfl_up_sync(0xffffffffu, fu, 1);
-            const int rH = __shfl_sync(0xffffffffu, cur.x, k & 31);
-            const int rF = __shfl_sync(0xffffffffu, cur.y, k & 31);
-            if (lane == 0) { upH = rH; upF = rF; }
-            const int b = k - lane + 1;
-            if (b >= 1 && b <= w) {
-                const int cc = mm_up(P.cs[(long long)b * P.cstep]);
-                int hd = hdiag;
-                hdiag = upH;
-                unsigned int code = 0;
-                int capH = 0, capF = 0;
-#pragma unroll
-                for (int r = 0; r < MM_ALPHA; r++) {
-                    const int e = max(Ep[r] - g.ge, Hp[r] - g.gf);                // Eq. 2
-                    const int f = max(upF - g.ge, upH - g.gf);                    // Eq. 3
-                    const int d = hd + (rc[r] == cc ? g.ma : g.mi);               // Eq. 1 (no 0 term)
-                    const int hv = max(max(e, f), d);
-                    if (MODE == 1) {
-                        const unsigned int src = (d >= e && d >= f) ? 0u : (f >= e ? 1u : 2u);
-                        const unsigned int ext = (Ep[r] - g.ge >= Hp[r] - g.gf ? 4u : 0u) |
-                                                 (upF - g.ge >= upH - g.gf ? 8u : 0u);
-                        code |= (src | ext) << (4 * r);
-                    }
-                    if (MODE == 0 && r0 + r + 1 == capR) { capH = hv; capF = f; }
-                    hd = Hp[r];
-                    Hp[r] = max(hv, NEG);
-                    Ep[r] = max(e, NEG);
-                    upH = Hp[r];
-                    upF = max(f, NEG);
-                }
-                hu = upH;
-                fu = upF;
-                if (MODE == 1 && r0 < h) codes[(long long)b * HW + r0 / 8] = code;
-                if (MODE == 0 && capR > r0 && capR <= r0 + MM_ALPHA) cap[b] = make_int2(capH, capF);
-                if (lane == 31) rowbuf[b] = make_int2(hu, fu);
-            }
-        }
+        if (MODE == 0 && a0 + MM_CHUNK >= capR)
+            mm_chunk<MODE, true>(g, P, a0, rowbuf, rowbuf, capR, cap, codes, lane, [](int) {}, [](int) {});
+        else
+            mm_chunk<MODE, false>(g, P, a0, rowbuf, rowbuf, capR, cap, codes, lane, [](int) {}, [](int) {});
         __threadfence_block();
         __syncwarp();
     }
@@ -179,13 +220,13 @@ __device__ void mm_warp_dp(const MMArgs &g, const DpProb &P, int2 *rowbuf, int c
 // shared memory every 32 columns (after __threadfence_block), the reader's
 // lane 0 waits for it before each 32-column prefetch and loads through L2
 // (__ldcg).  A slot is reused by the same warp NWP chunks later, after its
-// reader (the next warp) is done with it.  Same arithmetic as mm_warp_dp.
+// reader (the next warp) is done with it.
 template <int NWP>
 __device__ void mm_cta_pass(const MMArgs &g, const DpProb &P, int2 *ring, long long rs, int capR, int2 *cap,
                             volatile int *s_gen, volatile int *s_cols, int warp, int lane)
 {
     constexpr int R = NWP + 1;
-    const int h = P.h, w = P.w, kind = P.kind;
+    const int w = P.w, kind = P.kind;
     for (int b = threadIdx.x; b <= w; b += blockDim.x) {
         const int2 v = make_int2(b == 0 ? 0 : mm_row0(g, kind, b), (b == 0 && kind == 2) ? 0 : NEG);
         ring[b] = v;
@@ -197,20 +238,16 @@ __device__ void mm_cta_pass(const MMArgs &g, const DpProb &P, int2 *ring, long l
     }
     if (capR > 0 && threadIdx.x == 0) cap[0] = make_int2(mm_col0(g, kind, capR), mm_col0(g, kind, capR));
     __syncthreads();
-    const int diag00 = (kind == 3 || kind == 4) ? NEG : 0;
     const int nchunks = (capR + MM_CHUNK - 1) / MM_CHUNK;
     for (int c = warp; c < nchunks; c += NWP) {
-        const int a0 = c * MM_CHUNK;
         const int in = c % R, out = (c + 1) % R;
-        const int2 *rin = ring + in * rs;
-        int2 *rout = ring + out * rs;
         if (lane == 0) {
             s_cols[out] = 0;
             __threadfence_block();
             s_gen[out] = c;
         }
         __syncwarp();
-        auto wait_cols = [&](int need) {
+        auto wait = [&](int need) {
             need = min(need, w);
             if (lane == 0 && (s_gen[in] != c - 1 || s_cols[in] < need)) {
                 const unsigned long long t0 = gtimer();
@@ -222,63 +259,15 @@ __device__ void mm_cta_pass(const MMArgs &g, const DpProb &P, int2 *ring, long l
             __syncwarp();
             __threadfence_block();
         };
-        const int r0 = a0 + lane * MM_ALPHA;
-        int rc[MM_ALPHA], Hp[MM_ALPHA], Ep[MM_ALPHA];
-#pragma unroll
-        for (int r = 0; r < MM_ALPHA; r++) {
-            const int a = r0 + r + 1;
-            rc[r] = a <= h ? mm_up(P.rs[(long long)a * P.rstep]) : 0x100;
-            Hp[r] = mm_col0(g, kind, a);
-            Ep[r] = NEG;
-        }
-        int hdiag = r0 == 0 ? diag00 : mm_col0(g, kind, r0);
-        int hu = 0, fu = 0;
-        wait_cols(64);
-        int2 cur = (1 + lane <= w) ? __ldcg(rin + 1 + lane) : make_int2(NEG, NEG);
-        int2 nxt = (33 + lane <= w) ? __ldcg(rin + 33 + lane) : make_int2(NEG, NEG);
-        int capH = 0, capF = 0;
-        const int nsteps = w + 31;
-        for (int k = 0; k < nsteps; k++) {
-            if (k > 0 && (k & 31) == 0) {
-                cur = nxt;
-                wait_cols(k + 64);
-                const int cc2 = k + 33 + lane;
-                nxt = cc2 <= w ? __ldcg(rin + cc2) : make_int2(NEG, NEG);
-            }
-            int upH = __shfl_up_sync(0xffffffffu, hu, 1);
-            int upF = __shfl_up_sync(0xffffffffu, fu, 1);
-            const int rH = __shfl_sync(0xffffffffu, cur.x, k & 31);
-            const int rF = __shfl_sync(0xffffffffu, cur.y, k & 31);
-            if (lane == 0) { upH = rH; upF = rF; }
-            const int b = k - lane + 1;
-            if (b >= 1 && b <= w) {
-                const int cc = mm_up(P.cs[(long long)b * P.cstep]);
-                int hd = hdiag;
-                hdiag = upH;
-#pragma unroll
-                for (int r = 0; r < MM_ALPHA; r++) {
-                    const int e = max(Ep[r] - g.ge, Hp[r] - g.gf);   // Eq. 2
-                    const int f = max(upF - g.ge, upH - g.gf);       // Eq. 3
-                    const int d = hd + (rc[r] == cc ? g.ma : g.mi);  // Eq. 1 (no 0 term)
-                    const int hv = max(max(e, f), d);
-                    if (r0 + r + 1 == capR) { capH = hv; capF = f; }
-                    hd = Hp[r];
-                    Hp[r] = max(hv, NEG);
-                    Ep[r] = max(e, NEG);
-                    upH = Hp[r];
-                    upF = max(f, NEG);
-                }
-                hu = upH;
-                fu = upF;
-                if (capR > r0 && capR <= r0 + MM_ALPHA) cap[b] = make_int2(capH, capF);
-                if (lane == 31) rout[b] = make_int2(hu, fu);
-            }
-            if ((k & 31) == 31 || k == nsteps - 1) {
-                __threadfence_block();
-                __syncwarp();
-                if (lane == 31) s_cols[out] = min(w, k - 30);
-            }
-        }
+        auto publish = [&](int cols) {
+            __threadfence_block();
+            __syncwarp();
+            if (lane == 31) s_cols[out] = cols;
+        };
+        if ((c + 1) * MM_CHUNK >= capR)
+            mm_chunk<0, true>(g, P, c * MM_CHUNK, ring + in * rs, ring + out * rs, capR, cap, nullptr, lane, wait, publish);
+        else
+            mm_chunk<0, false>(g, P, c * MM_CHUNK, ring + in * rs, ring + out * rs, capR, cap, nullptr, lane, wait, publish);
     }
     __syncthreads();
 }

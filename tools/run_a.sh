@@ -1,3 +1,2 @@
-python tools/mm_bench.py 20000
-SWB_MM_CTA_ROWS=100000000 python tools/mm_bench.py 20000
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:sw_mm_split_cta -c 1 -o gpurun_out/mm_cta -f python tools/mm_bench.py 20000 > gpurun_out/ncu_mm.log 2>&1
+timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+timeout 900 python tools/align_bench.py C1 C2 C4
