@@ -40,8 +40,11 @@ PAPER_GCUPS = {"C2": 21.419}
 # mix with the measured rates (profiles/r01_microbench_int.txt; half-rate ops
 # occupy the ALU pipe 2 cycles per warp instruction, full-rate ops 1):
 #   int32 kernel: 8 ALU cycles per 32 cells  -> 16.0 cells/clk/SM
-#   packed 16x2 : 9 ALU cycles per 64 cells  -> 28.44 cells/clk/SM
-ROOF_CELLS_PER_CLK_SM = {"int32": 16.0, "int16x2": 28.44}
+#   packed 16x2 : 11 ALU cycles per 64 cells -> 23.27 cells/clk/SM
+#     (SWB_FMODE 2 mix: VIMNMX3 E*, PRMT p, 3x VIADDMNMX D/t/F', 1/2 VIMNMX3 max;
+#      the earlier mix with 9 ALU cycles issued 2 more instructions per slot and
+#      ran 14-18 % slower)
+ROOF_CELLS_PER_CLK_SM = {"int32": 16.0, "int16x2": round(4 * 64 / 11, 2)}
 
 
 def parse():

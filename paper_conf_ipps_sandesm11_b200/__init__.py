@@ -20,7 +20,7 @@ import numpy as np
 from . import build as _build
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libcudalign_b200.so")
+LIB_PATH = os.environ.get("SWB_LIB") or os.path.join(_HERE, "libcudalign_b200.so")
 
 SW_OK = 0
 SW_EINVAL = -1

@@ -30,6 +30,9 @@
 namespace swb {
 
 constexpr int BIAS16 = 32768;
+#ifndef SWB_FMODE
+#define SWB_FMODE 2
+#endif
 
 __device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(lo & 0xffff) | ((uint32_t)hi << 16); }
 __device__ __forceinline__ int lo16(uint32_t v) { return (int)(v & 0xffffu); }
@@ -113,6 +116,39 @@ struct Fill16 {
     // recurrence (max(max(E,0) - G_ext, t, 0) = max(E - G_ext, t, 0)), and H
     // takes max(.., E, .., 0) anyway.  E only leaves the lane as a stripe's
     // right border, where the receiver's H and F are unchanged by the floor.
+    // H, t and the next row's F of one slot from D and the incoming F (both
+    // halves).  SWB_FMODE selects the instruction mix:
+    //   0: H = max(D, F); t = H - G_first; F' = max(F - G_ext, D - G_first)
+    //      (IMAD + VIMNMX on the F chain)
+    //   1: F' = VIADDMNMX(F, -G_ext, D - G_first): the F chain down the slots
+    //      is one same-pipe instruction per slot
+    //   2: as 1, and t = VIADDMNMX(F, -G_first, D - G_first) directly; the
+    //      tile maximum is then taken over t (= H - G_first) instead of H,
+    //      except in replays (TRACK), which need H.
+    // The u16x2 adds never wrap: every frame value stays far above G_first.
+    template <bool TRACK>
+    static __device__ __forceinline__ void cell_hf(uint32_t d, uint32_t &fu, uint32_t &h, uint32_t &t, int one,
+                                                   int nge2, int ngf2, uint32_t nge16, uint32_t ngf16)
+    {
+        if constexpr (SWB_FMODE == 0) {
+            h = __vmaxu2(d, fu);
+            t = (uint32_t)imad((int)h, one, ngf2);
+            fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d, one, ngf2));
+        } else {
+            const uint32_t dg = (uint32_t)imad((int)d, one, ngf2);
+            if constexpr (SWB_FMODE == 1 || TRACK) {
+                h = __vmaxu2(d, fu);
+                t = (uint32_t)imad((int)h, one, ngf2);
+            } else {
+                t = __viaddmax_u16x2(fu, ngf16, dg);
+                h = t;
+            }
+            fu = __viaddmax_u16x2(fu, nge16, dg);
+        }
+    }
+    // Offset from the tile maximum a non-replay tile returns to H (mode 2: t).
+    static __device__ __forceinline__ int tmax_off(const FillArgs &a) { return SWB_FMODE == 2 && !SPLIT ? a.gf : 0; }
+
     template <bool GUARD, bool TRACK, bool SP1, bool CAP>
     static __device__ __forceinline__ uint32_t step(const FillArgs &a, const StepInfo &X, Lane &L, int k, int lane,
                                                     uint32_t cr_a, uint32_t ro_a, uint32_t sel_a, uint32_t pt_sel,
@@ -137,6 +173,9 @@ struct Fill16 {
         uint32_t td = L.tprev;
         L.tprev = tu;
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
+        // per-half two's complements of -G_ext, -G_first for the u16x2 adds
+        const uint32_t nge16 = ((0x10000u - (uint32_t)a.ge) & 0xffffu) * 0x10001u;
+        const uint32_t ngf16 = ((0x10000u - (uint32_t)a.gf) & 0xffffu) * 0x10001u;
         uint32_t f15 = 0;  // F entering the last slot (row 2NS-1 in the high half)
         if constexpr (SPLIT) {
             // Same cells, shorter F chain for latency-bound warps: D of every slot
@@ -198,20 +237,18 @@ struct Fill16 {
                 const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
                 const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
                 const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
-                const uint32_t h0 = __vmaxu2(d0, fu);
                 td = L.t[s];
-                const uint32_t t0 = (uint32_t)imad((int)h0, one, ngf2);
-                fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d0, one, ngf2));
+                uint32_t h0, t0;
+                cell_hf<TRACK>(d0, fu, h0, t0, one, nge2, ngf2, nge16, ngf16);
                 L.e[s] = e0;
                 L.t[s] = t0;
                 if (s == NS - 2) f15 = fu;
                 const uint32_t e1 = __vimax3_u16x2((uint32_t)imad((int)L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
                 const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
                 const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
-                const uint32_t h1 = __vmaxu2(d1, fu);
                 td = L.t[s + 1];
-                const uint32_t t1 = (uint32_t)imad((int)h1, one, ngf2);
-                fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d1, one, ngf2));
+                uint32_t h1, t1;
+                cell_hf<TRACK>(d1, fu, h1, t1, one, nge2, ngf2, nge16, ngf16);
                 L.e[s + 1] = e1;
                 L.t[s + 1] = t1;
                 tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
@@ -643,7 +680,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     } else {
                         tm = F::template tile<false, false, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
                     }
-                    const int tmax = F::toabs(L, max(lo16(tm), hi16(tm)));
+                    const int tmax = F::toabs(L, max(lo16(tm), hi16(tm))) + F::tmax_off(a);
                     if (__any_sync(0xffffffffu, tmax >= thr)) {
                         F::restore(L, sv, lane);
                         const int obs = bs;
