@@ -88,6 +88,8 @@ typedef struct {
     int64_t special_rows;
     int64_t special_bytes_d2h;
     int32_t alpha, warps, width, grid; /* launch configuration */
+    int32_t patched;   /* 1: the packed kernel ran with the gap penalties patched in as
+                          instruction immediates; 0: runtime operands */
 } sw_stats;
 
 /* Create a context on the given CUDA devices.  Round 1 supports exactly one
@@ -210,6 +212,14 @@ int64_t sw_band_height(const sw_ctx *ctx);
  * qualifies (local mode, k % 16 == 0, small value window).  packed = 0 never
  * uses the packed kernel.  Results are identical for every choice. */
 int sw_set_kernel(sw_ctx *ctx, int variant, int packed);
+
+/* Immediate patching of the packed kernel (testing / tuning; default on).
+ * on = 1: the packed kernel runs from a copy of its cubin whose gap-penalty
+ * immediates are patched with the call's values, loaded once
+ * per (gap_open, gap_ext) and context; on = 0: the kernel that reads them from
+ * registers.  Results are identical; sw_stats.patched says which one ran.
+ * Returns SW_EINVAL for a NULL ctx or on outside {0, 1}. */
+int sw_set_patch(sw_ctx *ctx, int on);
 
 /* ---- Column-stripe pipeline ----
  * The matrix is split into column stripes; stripe g sweeps every band of its

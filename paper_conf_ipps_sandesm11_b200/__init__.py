@@ -43,6 +43,7 @@ EXPORTED = [
     "sw_row_granularity",
     "sw_band_height",
     "sw_set_kernel",
+    "sw_set_patch",
     "sw_set_virtual_stripes",
     "sw_stripe_export",
     "sw_stripe_connect",
@@ -95,6 +96,7 @@ class Stats(ctypes.Structure):
         ("warps", ctypes.c_int32),
         ("width", ctypes.c_int32),
         ("grid", ctypes.c_int32),
+        ("patched", ctypes.c_int32),
     ]
 
     def as_dict(self):
@@ -147,6 +149,8 @@ def load_library(path: str = LIB_PATH):
     lib.sw_band_height.restype = i64
     lib.sw_set_kernel.argtypes = [vp, ctypes.c_int, ctypes.c_int]
     lib.sw_set_kernel.restype = ctypes.c_int
+    lib.sw_set_patch.argtypes = [vp, ctypes.c_int]
+    lib.sw_set_patch.restype = ctypes.c_int
     lib.sw_set_virtual_stripes.argtypes = [vp, ctypes.c_int]
     lib.sw_set_virtual_stripes.restype = ctypes.c_int
     lib.sw_stripe_export.argtypes = [vp, i64, vp]
@@ -338,6 +342,11 @@ class Context:
     def set_kernel(self, variant: int = -1, packed: bool = True):
         """variant -1: automatic; 0..5: fixed geometry; packed: allow the 16x2 kernel."""
         self._check(self._lib.sw_set_kernel(self._h, variant, int(bool(packed))), "sw_set_kernel")
+
+    def set_patch(self, on: bool = True):
+        """Run the packed kernel with the gap penalties patched in as immediates
+        (default) or read from registers; results are identical."""
+        self._check(self._lib.sw_set_patch(self._h, int(bool(on))), "sw_set_patch")
 
     def set_virtual_stripes(self, nstripes: int):
         """Split the next Stage-1 calls into `nstripes` column stripes on this GPU

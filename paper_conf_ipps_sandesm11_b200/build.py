@@ -12,6 +12,11 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libcudalign_b200.so")
 SOURCES = [os.path.join(HERE, "csrc", "sw_api.cu")]
+# The packed kernels with magic immediates (csrc/sw_fill16_patch.cu), embedded
+# in the library and patched per scoring at run time.
+PATCH_SRC = os.path.join(HERE, "csrc", "sw_fill16_patch.cu")
+PATCH_CUBIN = os.path.join(HERE, "sw_fill16_patch.cubin")
+MAGIC = {"NGE2": 0x6B8B4567, "NGF2": 0x327B23C6, "NGE16": 0x643C9869, "NGF16": 0x66334873}
 import glob
 
 DEPS = sorted(glob.glob(os.path.join(HERE, "csrc", "*"))) + [os.path.join(ROOT, "include", "cudalign_b200.h")]
@@ -30,11 +35,40 @@ def stale() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS)
 
 
+def check_patch_sites(path: str) -> dict:
+    """Every occurrence of a magic word in the cubin must be a 32-bit
+    instruction immediate (byte 4 of a 16-byte SASS instruction); the loader
+    (sw_api.cu patch_sites) refuses to patch otherwise."""
+    import struct
+
+    data = open(path, "rb").read()
+    counts = {}
+    for name, v in MAGIC.items():
+        pat = struct.pack("<I", v)
+        offs, i = [], data.find(pat)
+        while i >= 0:
+            offs.append(i)
+            i = data.find(pat, i + 1)
+        bad = [o for o in offs if o % 16 != 4]
+        if bad:
+            raise RuntimeError(f"{path}: magic {name} at non-immediate offsets {bad[:4]}")
+        counts[name] = len(offs)
+    for name in ("NGE2", "NGE16", "NGF16"):
+        if counts[name] == 0:
+            raise RuntimeError(f"{path}: magic {name} not found (ptxas folded it?)")
+    return counts
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
+    ptmp = PATCH_CUBIN + f".tmp{os.getpid()}"
+    subprocess.check_call([NVCC, *[f for f in FLAGS if f not in ("-Xcompiler", "-fPIC", "-shared")], "-cubin",
+                           "-o", ptmp, PATCH_SRC])
+    check_patch_sites(ptmp)
+    os.replace(ptmp, PATCH_CUBIN)
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *FLAGS, "-o", tmp, *SOURCES]
+    cmd = [NVCC, *FLAGS, f'-DSWB_PATCH_CUBIN="{PATCH_CUBIN}"', "-o", tmp, *SOURCES]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd))

@@ -107,7 +107,15 @@ struct Variant {
     size_t smem16;
     int io_warps;           // 1, or 0 for the cooperative-I/O packed kernel (block = (nw + io) warps)
     int skew_tiles;         // int32 kernel: tiles past the last column lane 31 needs (ceil(62 / W))
+    char packed_name[96];   // mangled name of the packed kernel in the patchable cubin ("" : none)
 };
+
+template <int NW, int W, bool COOP, int NS>
+static void packed_name(Variant &v)
+{
+    snprintf(v.packed_name, sizeof(v.packed_name), "_ZN3swb16sw_fill16_kernelILi%dELi%dELb%dELi%dELb0EEEvNS_8FillArgsE",
+             NW, W, COOP ? 1 : 0, NS);
+}
 
 template <int ALPHA, int NW, int W, bool COOP = false, bool SPLIT = false>
 static Variant make_variant()
@@ -122,11 +130,13 @@ static Variant make_variant()
     v.smem16 = 0;
     v.io_warps = 1;
     v.skew_tiles = 1;
+    v.packed_name[0] = 0;
     if constexpr (ALPHA == 32) {
         // packed kernel only (16 slots per lane); int32 work falls back to the default geometry
         v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, 16, SPLIT>;
         v.io_warps = COOP ? 0 : 1;
         v.smem16 = Fill16<NW, W, 16, SPLIT>::smem_bytes();
+        if constexpr (!SPLIT) packed_name<NW, W, COOP, 16>(v);
         return v;
     } else {
         v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
@@ -138,8 +148,10 @@ static Variant make_variant()
         if constexpr (NW == 16) {
             v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, true>;
             v.io_warps = 0;
+            packed_name<NW, W, true, 8>(v);
         } else {
             v.packed_fn = (const void *)&sw_fill16_kernel<NW, W>;
+            packed_name<NW, W, false, 8>(v);
         }
         v.smem16 = Fill16<NW, W>::smem_bytes();
     }
@@ -199,6 +211,67 @@ struct S1Rows {
     int64_t ld = 0, stride = 0;  // row q at sp[0] + q * stride: H[0..n), F at + ld
 };
 
+// ---------------------------------------------------------------- patched packed kernels
+//
+// The packed cell update is bound by register reads: an add
+// whose constant is an instruction immediate reads one register, with the
+// constant in a register three.  The gap penalties are runtime values, so the
+// packed kernels are also built into a separate cubin (sw_fill16_patch.cu)
+// with magic immediates; per (G_ext, G_first) the library copies that image,
+// overwrites the immediates (32-bit field at byte 4 of each 16-byte SASS
+// instruction) and loads it with cudaLibraryLoadData.  The build checks that
+// every occurrence of the magic words is such a field (build.py).
+
+#if defined(SWB_PATCH_CUBIN) && !defined(__CUDA_ARCH__)
+asm(".section .rodata\n"
+    ".balign 16\n"
+    "swb_patch_cubin_begin:\n"
+    ".incbin \"" SWB_PATCH_CUBIN "\"\n"
+    "swb_patch_cubin_end:\n"
+    ".previous\n");
+extern "C" const unsigned char swb_patch_cubin_begin[] __asm__("swb_patch_cubin_begin");
+extern "C" const unsigned char swb_patch_cubin_end[] __asm__("swb_patch_cubin_end");
+static const unsigned char *patch_image() { return swb_patch_cubin_begin; }
+static size_t patch_image_size() { return (size_t)(swb_patch_cubin_end - swb_patch_cubin_begin); }
+#else
+static const unsigned char *patch_image() { return nullptr; }
+static size_t patch_image_size() { return 0; }
+#endif
+
+struct PatchedSet {
+    int ge = -1, gf = -1;
+    cudaLibrary_t lib = nullptr;
+    const void *fn[NVARIANTS] = {};
+};
+
+// Offsets of the magic immediates in the embedded image (computed once).
+struct PatchSites {
+    std::vector<size_t> off[4];
+    bool ok = false;
+};
+static const PatchSites &patch_sites()
+{
+    static PatchSites ps = [] {
+        PatchSites p;
+        const unsigned char *img = patch_image();
+        const size_t n = patch_image_size();
+        if (!img || n < 16) return p;
+        const uint32_t magic[4] = {SWB_K_NGE2, SWB_K_NGF2, SWB_K_NGE16, SWB_K_NGF16};
+        for (size_t o = 0; o + 4 <= n; o++) {
+            uint32_t w;
+            memcpy(&w, img + o, 4);
+            for (int k = 0; k < 4; k++)
+                if (w == magic[k]) {
+                    if (o % 16 != 4) return p;  // not an instruction immediate: refuse to patch
+                    p.off[k].push_back(o);
+                }
+        }
+        p.ok = !p.off[0].empty() && !p.off[2].empty() && !p.off[3].empty();
+        return p;
+    }();
+    return ps;
+}
+
 struct sw_ctx {
     int device = 0;
     int num_sms = 0;
@@ -227,6 +300,8 @@ struct sw_ctx {
     int vstripes = 1;           // virtual stripes for the single-process calls
     S1Rows s1;                  // special rows resident from the last Stage-1 call
     int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
+    int patch = 1;              // use the immediate-patched packed kernels (SWB_PATCH=0: runtime operands)
+    std::vector<PatchedSet> patched;  // loaded patched images, most recent last
     long long timeout_ns = 120ll * 1000000000ll;
 };
 
@@ -339,6 +414,7 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
         if (const char *vs = getenv("SWB_VSTRIPES")) ctx->vstripes = std::max(1, std::min(MAX_STRIPES, atoi(vs)));
         if (const char *to = getenv("SWB_TIMEOUT_S")) ctx->timeout_ns = (long long)(atof(to) * 1e9);
         if (const char *pk = getenv("SWB_PACKED")) ctx->packed = atoi(pk);
+        if (const char *pt = getenv("SWB_PATCH")) ctx->patch = atoi(pt);
     } while (0);
     if (rc) { sw_shutdown(ctx); return rc; }
     *out = ctx;
@@ -361,6 +437,8 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
         if (ctx->colp[s].p) cudaFreeHost(ctx->colp[s].p);
         if (ctx->vrecv[s].base) cudaFree(ctx->vrecv[s].base);
     }
+    for (auto &P : ctx->patched)
+        if (P.lib) cudaLibraryUnload(P.lib);
     if (ctx->right_base) cudaIpcCloseMemHandle(ctx->right_base);
     if (ctx->recv.base) cudaFree(ctx->recv.base);
     if (ctx->stage.p) cudaFreeHost(ctx->stage.p);
@@ -411,6 +489,13 @@ extern "C" int sw_set_kernel(sw_ctx *ctx, int variant, int packed)
     if (!ctx || variant < -1 || variant >= NVARIANTS || packed < 0 || packed > 1) return SW_EINVAL;
     ctx->variant_override = variant;
     ctx->packed = packed;
+    return SW_OK;
+}
+
+extern "C" int sw_set_patch(sw_ctx *ctx, int on)
+{
+    if (!ctx || on < 0 || on > 1) return SW_EINVAL;
+    ctx->patch = on;
     return SW_OK;
 }
 
@@ -508,6 +593,58 @@ static double model_fill_time(long long nb, long long P, long long n, long long 
     return (std::max(chain, waves) + (double)n) / cps;
 }
 
+// The patched packed kernel of variant V for (G_ext, G_first), loading the
+// image on first use (at most 4 images per context, oldest unloaded first).
+// nullptr: not available (no embedded image, SWB_PATCH=0, or a load error),
+// and the caller runs the runtime-operand kernel (same results).
+static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf)
+{
+    if (!ctx->patch || !V.packed_name[0]) return nullptr;
+    const PatchSites &ps = patch_sites();
+    if (!ps.ok) return nullptr;
+    const int vidx = (int)(&V - &variant_for(0));
+    if (vidx < 0 || vidx >= NVARIANTS) return nullptr;
+    PatchedSet *P = nullptr;
+    for (auto &q : ctx->patched)
+        if (q.ge == ge && q.gf == gf) P = &q;
+    if (!P) {
+        std::vector<unsigned char> img(patch_image(), patch_image() + patch_image_size());
+        const uint32_t val[4] = {(uint32_t)(-(ge * 0x10001)), (uint32_t)(-(gf * 0x10001)),
+                                 ((0x10000u - (uint32_t)ge) & 0xffffu) * 0x10001u,
+                                 ((0x10000u - (uint32_t)gf) & 0xffffu) * 0x10001u};
+        for (int k = 0; k < 4; k++)
+            for (size_t o : ps.off[k]) memcpy(img.data() + o, &val[k], 4);
+        PatchedSet q;
+        q.ge = ge;
+        q.gf = gf;
+        if (cudaLibraryLoadData(&q.lib, img.data(), nullptr, nullptr, 0, nullptr, nullptr, 0) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        if (ctx->patched.size() >= 4) {
+            cudaDeviceSynchronize();  // an older image may still run on a caller's stream
+            cudaLibraryUnload(ctx->patched.front().lib);
+            ctx->patched.erase(ctx->patched.begin());
+        }
+        ctx->patched.push_back(q);
+        P = &ctx->patched.back();
+    }
+    if (!P->fn[vidx]) {
+        cudaKernel_t k = nullptr;
+        if (cudaLibraryGetKernel(&k, P->lib, V.packed_name) != cudaSuccess || !k) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)V.smem16) !=
+            cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        P->fn[vidx] = (const void *)k;
+    }
+    return P->fn[vidx];
+}
+
 static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
 {
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
@@ -528,11 +665,11 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
     // profiles/r01_variants.txt; earlier entries win near-ties (3 %)
     static const Candidate cands[] = {
         {DEFAULT_VARIANT, false, 4.24e6, 4.24e6},  // int32, 8 warps + I/O warp
-        {1, true, 5.967e6, 6.04e6},                // packed alpha 16, 8 warps + I/O warp
-        {8, true, 3.180e6, 6.05e6},                // packed alpha 32, 4 warps + I/O warp (2 CTAs/SM)
-        {10, true, 3.349e6, 3.349e6},              // packed alpha 32, 8 warps + I/O warp
-        {5, true, 3.363e6, 3.363e6},               // packed alpha 16, 15 warps + I/O warp
-        {6, true, 3.084e6, 3.084e6},               // packed alpha 16, 16 warps, cooperative I/O
+        {1, true, 8.08e6, 7.74e6},                 // packed alpha 16, 8 warps + I/O warp
+        {8, true, 4.25e6, 7.86e6},                 // packed alpha 32, 4 warps + I/O warp (2 CTAs/SM)
+        {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
+        {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
+        {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
     };
     double best_t = 1e300;
     int best = 0;
@@ -620,6 +757,13 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     }
     const void *fill_fn = use16 ? V.packed_fn : (J.local ? V.local_fn : V.global_fn);
     const size_t fill_smem = use16 ? V.smem16 : V.smem;
+    bool patched = false;
+    if (use16) {
+        if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge)) {
+            fill_fn = pf;
+            patched = true;
+        }
+    }
     const int block = V.nw * 32 + (use16 ? V.io_warps : 1) * 32;
     int blocks_per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, fill_fn, block, fill_smem);
@@ -721,6 +865,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     a.ge = J.ge;
     a.gf = J.go + J.ge;
     a.one = 1;
+    a.nge2 = (uint32_t)(-(J.ge * 0x10001));
+    a.ngf2 = (uint32_t)(-(a.gf * 0x10001));
+    a.nge16 = ((0x10000u - (uint32_t)J.ge) & 0xffffu) * 0x10001u;
+    a.ngf16 = ((0x10000u - (uint32_t)a.gf) & 0xffffu) * 0x10001u;
     for (int x = 0; x < 4; x++) {
         uint32_t w = 0;
         for (int y = 0; y < 4; y++) {
@@ -929,6 +1077,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     ctx->stats.special_rows += nsp;
     ctx->stats.special_bytes_d2h += bytes;
     ctx->stats.alpha = use16 ? -V.alpha : V.alpha;  // negative: packed 16x2 kernel
+    ctx->stats.patched = patched ? 1 : 0;
     ctx->stats.warps = V.nw;
     ctx->stats.width = W;
     ctx->stats.grid = grid;

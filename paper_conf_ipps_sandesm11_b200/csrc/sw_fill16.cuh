@@ -33,6 +33,26 @@ constexpr int BIAS16 = 32768;
 #ifndef SWB_FMODE
 #define SWB_FMODE 2
 #endif
+// Magic immediates of the patchable build (sw_fill16_patch.cu): -G_ext and
+// -G_first in both halves as a 32-bit add (NGE2, NGF2) and per half (NGE16,
+// NGF16).  Arbitrary values, chosen not to occur elsewhere in the code.
+#define SWB_K_NGE2 0x6b8b4567u
+#define SWB_K_NGF2 0x327b23c6u
+#define SWB_K_NGE16 0x643c9869u
+#define SWB_K_NGF16 0x66334873u
+#ifndef SWB_ADDMODE
+#ifdef SWB_PATCH
+#define SWB_ADDMODE 1
+#else
+#define SWB_ADDMODE 0
+#endif
+#endif
+#ifndef SWB_UNR
+#define SWB_UNR 4     // lane steps per iteration of the fast tile loop
+#endif
+#ifndef SWB_TMTREE
+#define SWB_TMTREE 0  // 1: tile maximum as a per-step tree instead of a chain through the slots
+#endif
 
 __device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(lo & 0xffff) | ((uint32_t)hi << 16); }
 __device__ __forceinline__ int lo16(uint32_t v) { return (int)(v & 0xffffu); }
@@ -48,8 +68,24 @@ __device__ __forceinline__ uint32_t col_sel16(uint32_t code)
     return lo | (hi << 8);
 }
 
+// Maximum of N packed u16x2 values as a 3-ary tree (depth log3 N instead of a chain).
+template <int N>
+struct MaxTree {
+    static __device__ __forceinline__ uint32_t run(const uint32_t *v)
+    {
+        if constexpr (N == 1) return v[0];
+        else if constexpr (N == 2) return __vmaxu2(v[0], v[1]);
+        else if constexpr (N == 3) return __vimax3_u16x2(v[0], v[1], v[2]);
+        else {
+            constexpr int A = (N + 2) / 3, B = (N - A + 1) / 2, C = N - A - B;
+            return __vimax3_u16x2(MaxTree<A>::run(v), MaxTree<B>::run(v + A), MaxTree<C>::run(v + A + B));
+        }
+    }
+};
+
 template <int NW, int W, int NS = 8, bool SPLIT = false>
 struct Fill16 {
+    static constexpr bool TMTREE = SWB_FMODE == 2 && SWB_TMTREE;
     static constexpr int ALPHA = 2 * NS, BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
     static constexpr int SRING = Smem<W, NW>::SRING;
@@ -126,6 +162,15 @@ struct Fill16 {
     //      tile maximum is then taken over t (= H - G_first) instead of H,
     //      except in replays (TRACK), which need H.
     // The u16x2 adds never wrap: every frame value stays far above G_first.
+    // x + c (both halves; never borrows, see above).  SWB_ADDMODE 0: IMAD with
+    // a runtime 1 (forces the FMA pipe, 3 register reads); 1: a plain add,
+    // ptxas picks IMAD.IADD (FMA pipe, 2 reads) or IADD3 (ALU pipe).
+    static __device__ __forceinline__ uint32_t add_fma(uint32_t x, int one, int c)
+    {
+        if constexpr (SWB_ADDMODE == 0) return (uint32_t)imad((int)x, one, c);
+        else return x + (uint32_t)c;
+    }
+
     template <bool TRACK>
     static __device__ __forceinline__ void cell_hf(uint32_t d, uint32_t &fu, uint32_t &h, uint32_t &t, int one,
                                                    int nge2, int ngf2, uint32_t nge16, uint32_t ngf16)
@@ -135,7 +180,7 @@ struct Fill16 {
             t = (uint32_t)imad((int)h, one, ngf2);
             fu = __vmaxu2((uint32_t)imad((int)fu, one, nge2), (uint32_t)imad((int)d, one, ngf2));
         } else {
-            const uint32_t dg = (uint32_t)imad((int)d, one, ngf2);
+            const uint32_t dg = add_fma(d, one, ngf2);
             if constexpr (SWB_FMODE == 1 || TRACK) {
                 h = __vmaxu2(d, fu);
                 t = (uint32_t)imad((int)h, one, ngf2);
@@ -172,10 +217,25 @@ struct Fill16 {
         uint32_t fu = __byte_perm(lane == 0 ? cr : up_f, L.fn, 0x5432);  // F of slot 0's rows
         uint32_t td = L.tprev;
         L.tprev = tu;
+#if defined(SWB_PATCH)
+        // Instruction immediates that sw_api.cu patches in the cubin at load
+        // time with this call's values: an add with an
+        // immediate reads one register instead of three.
+        constexpr int nge2 = (int)SWB_K_NGE2, ngf2 = (int)SWB_K_NGF2;
+        constexpr uint32_t nge16 = SWB_K_NGE16, ngf16 = SWB_K_NGF16;
+#elif defined(SWB_FIXGE)  // timing experiment only: gap penalties as compile-time immediates
+        constexpr int nge2 = -(SWB_FIXGE * 0x10001), ngf2 = -(SWB_FIXGF * 0x10001);
+        constexpr uint32_t nge16 = ((0x10000u - (uint32_t)SWB_FIXGE) & 0xffffu) * 0x10001u;
+        constexpr uint32_t ngf16 = ((0x10000u - (uint32_t)SWB_FIXGF) & 0xffffu) * 0x10001u;
+#elif SWB_ADDMODE == 2  // the addends straight from the kernel parameters (constant bank)
+        const int nge2 = (int)a.nge2, ngf2 = (int)a.ngf2;
+        const uint32_t nge16 = a.nge16, ngf16 = a.ngf16;
+#else
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
         // per-half two's complements of -G_ext, -G_first for the u16x2 adds
         const uint32_t nge16 = ((0x10000u - (uint32_t)a.ge) & 0xffffu) * 0x10001u;
         const uint32_t ngf16 = ((0x10000u - (uint32_t)a.gf) & 0xffffu) * 0x10001u;
+#endif
         uint32_t f15 = 0;  // F entering the last slot (row 2NS-1 in the high half)
         if constexpr (SPLIT) {
             // Same cells, shorter F chain for latency-bound warps: D of every slot
@@ -188,7 +248,7 @@ struct Fill16 {
             uint32_t d[NS];
 #pragma unroll
             for (int s = 0; s < NS; s++) {
-                const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
+                const uint32_t e0 = __vimax3_u16x2(add_fma(L.e[s], one, nge2), L.t[s], L.FL);
                 const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
                 d[s] = __viaddmax_u16x2(td, p0, e0);
                 td = L.t[s];
@@ -234,7 +294,7 @@ struct Fill16 {
         } else {
 #pragma unroll
             for (int s = 0; s < NS; s += 2) {
-                const uint32_t e0 = __vimax3_u16x2((uint32_t)imad((int)L.e[s], one, nge2), L.t[s], L.FL);
+                const uint32_t e0 = __vimax3_u16x2(add_fma(L.e[s], one, nge2), L.t[s], L.FL);
                 const uint32_t p0 = (uint32_t)prmt(L.P[s], L.Q[s], sel);
                 const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
                 td = L.t[s];
@@ -243,7 +303,7 @@ struct Fill16 {
                 L.e[s] = e0;
                 L.t[s] = t0;
                 if (s == NS - 2) f15 = fu;
-                const uint32_t e1 = __vimax3_u16x2((uint32_t)imad((int)L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
+                const uint32_t e1 = __vimax3_u16x2(add_fma(L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
                 const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
                 const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
                 td = L.t[s + 1];
@@ -251,7 +311,7 @@ struct Fill16 {
                 cell_hf<TRACK>(d1, fu, h1, t1, one, nge2, ngf2, nge16, ngf16);
                 L.e[s + 1] = e1;
                 L.t[s + 1] = t1;
-                tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
+                if (TRACK || !TMTREE) tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
                 if (CAP) {
                     if (jl == X.jcap) {
                         X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
@@ -263,6 +323,14 @@ struct Fill16 {
                     }
                 }
             }
+        }
+        if constexpr (!SPLIT && !TRACK && TMTREE) {
+            // tile maximum as a 3-ary tree over this step's t (mode 2: t is what is tracked)
+            uint32_t v[NS + 1];
+#pragma unroll
+            for (int s = 0; s < NS; s++) v[s] = L.t[s];
+            v[NS] = tmax;
+            tmax = MaxTree<NS + 1>::run(v);
         }
         L.fn = fu;
         if (GUARD) {
@@ -358,17 +426,13 @@ struct Fill16 {
                                                     row1, bs, bi, bj, sp_ptr);
         } else {
 #pragma unroll 1
-            for (int kq = 0; kq < STEPS; kq += 4) {
+            for (int kq = 0; kq < STEPS; kq += SWB_UNR) {
                 const uint32_t sq = sel0 + 2u * kq, cq = cring + 4u * kq, oq = ro0 + 8u * kq;
-                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq, lane, cq, oq, sq, pt_sel, one, tmax,
-                                                      row1, bs, bi, bj, sp_ptr);
-                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + 1, lane, cq + 4u, oq + 8u, sq + 4u * HALF,
-                                                      pt_sel, one, tmax, row1, bs, bi, bj, sp_ptr);
-                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + 2, lane, cq + 8u, oq + 16u, sq + 4u,
-                                                      pt_sel, one, tmax, row1, bs, bi, bj, sp_ptr);
-                tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + 3, lane, cq + 12u, oq + 24u,
-                                                      sq + 4u + 4u * HALF, pt_sel, one, tmax, row1, bs, bi, bj,
-                                                      sp_ptr);
+#pragma unroll
+                for (int u = 0; u < SWB_UNR; u++)
+                    tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + u, lane, cq + 4u * u, oq + 8u * u,
+                                                          sq + 4u * ((u >> 1) + (u & 1) * HALF), pt_sel, one, tmax,
+                                                          row1, bs, bi, bj, sp_ptr);
             }
         }
         return tmax;

@@ -1,0 +1,23 @@
+// sw_fill16_patch.cu -- the packed Stage-1 kernels built with magic
+// instruction immediates for the gap penalties (SWB_PATCH, sw_fill16.cuh).
+// Compiled to a cubin that is embedded in libcudalign_b200.so; at run time
+// sw_api.cu replaces the magic immediates with the call's -G_ext / -G_first
+// encodings and loads the patched image (cudaLibraryLoadData).  An add with an
+// immediate reads one register instead of three, which is what the packed
+// cell update is bound by.
+#define SWB_PATCH 1
+#include "sw_fill16.cuh"
+
+namespace swb {
+// the packed geometries of the variant table (sw_api.cu variant_for)
+template __global__ void sw_fill16_kernel<4, 64, false, 8, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<8, 64, false, 8, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<12, 64, false, 8, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<14, 64, false, 8, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<15, 64, false, 8, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<16, 64, true, 8, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<4, 64, false, 16, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<4, 64, true, 16, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<8, 64, false, 16, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<16, 64, true, 16, false>(const __grid_constant__ FillArgs);
+}  // namespace swb

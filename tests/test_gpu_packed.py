@@ -41,6 +41,8 @@ def check(ctx, A, B, scoring, k, variant, stripes=1, expect_packed=True):
         ctx.set_kernel(-1, True)
         ctx.set_virtual_stripes(1)
     assert (st["alpha"] < 0) == expect_packed, st
+    # the immediate-patched image runs for every packed geometry but the split-F one (12)
+    assert st["patched"] == (1 if expect_packed and variant not in (12,) else 0), st
     want, orows = oracle.stage1(_s(A), _s(B), *scoring, k=k)
     assert got.astuple() == want, (len(A), len(B), scoring, k, variant, stripes)
     assert [r for r, _, _ in rows] == [r for r, _, _ in orows]
@@ -103,3 +105,27 @@ def test_packed_config_c1(ctx):
     cfg = synth.CONFIGS["C1"]
     A, B = synth.make_pair(cfg)
     check(ctx, A, B, PAPER, cfg.k, 5)
+
+
+@pytest.mark.parametrize("scoring", [PAPER, (2, -1, 0, 1), (5, -4, 10, 1), (1, -1, 1, 1), (3, -2, 2, 3)])
+def test_patch_on_off_identical(ctx, scoring):
+    """Patched immediates (per scoring) and register operands give identical
+    special rows and best cell, both equal to the oracle."""
+    A, B = synth.random_pair(77 + scoring[2], 4000, 3000, plant_len=1500, s=0.03, g=0.01)
+    out = []
+    for on in (True, False):
+        ctx.set_patch(on)
+        try:
+            got, rows = ctx.align_stage1(A, B, *scoring, k=64, keep_rows=True)
+            st = ctx.stats()
+        finally:
+            ctx.set_patch(True)
+        assert st["alpha"] < 0 and st["patched"] == int(on), st
+        out.append((got.astuple(), rows))
+    assert out[0][0] == out[1][0]
+    for (r, h, f), (r2, h2, f2) in zip(out[0][1], out[1][1]):
+        assert r == r2 and np.array_equal(h, h2) and np.array_equal(f, f2)
+    want, orows = oracle.stage1(_s(A), _s(B), *scoring, k=64)
+    assert out[0][0] == want
+    for (r, h, f), (_, oh, of) in zip(out[0][1], orows):
+        assert np.array_equal(h, oh) and np.array_equal(f, of), r
