@@ -16,7 +16,8 @@ SOURCES = [os.path.join(HERE, "csrc", "sw_api.cu")]
 # in the library and patched per scoring at run time.
 PATCH_SRC = os.path.join(HERE, "csrc", "sw_fill16_patch.cu")
 PATCH_CUBIN = os.path.join(HERE, "sw_fill16_patch.cubin")
-MAGIC = {"NGE2": 0x6B8B4567, "NGF2": 0x327B23C6, "NGE16": 0x643C9869, "NGF16": 0x66334873}
+MAGIC = {"NGE2": 0x6B8B4567, "NGF2": 0x327B23C6, "NGE16": 0x643C9869, "NGF16": 0x66334873,
+         "NGE1": 0x2AE8944A, "NGF1": 0x625558EC}
 import glob
 
 DEPS = sorted(glob.glob(os.path.join(HERE, "csrc", "*"))) + [os.path.join(ROOT, "include", "cudalign_b200.h")]
@@ -52,8 +53,11 @@ def check_patch_sites(path: str) -> dict:
         bad = [o for o in offs if o % 16 != 4]
         if bad:
             raise RuntimeError(f"{path}: magic {name} at non-immediate offsets {bad[:4]}")
+        # ptxas must use the constant as written: a negated copy (x - (-K)) could not be patched
+        if data.find(struct.pack("<I", (-v) & 0xFFFFFFFF)) >= 0:
+            raise RuntimeError(f"{path}: the negation of magic {name} occurs (an unpatchable form)")
         counts[name] = len(offs)
-    for name in ("NGE2", "NGE16", "NGF16"):
+    for name in ("NGE2", "NGE16", "NGF16", "NGE1", "NGF1"):
         if counts[name] == 0:
             raise RuntimeError(f"{path}: magic {name} not found (ptxas folded it?)")
     return counts

@@ -241,12 +241,13 @@ static size_t patch_image_size() { return 0; }
 struct PatchedSet {
     int ge = -1, gf = -1;
     cudaLibrary_t lib = nullptr;
-    const void *fn[NVARIANTS] = {};
+    const void *fn[3][NVARIANTS] = {};  // [packed, int32 local, int32 global][variant]
 };
 
 // Offsets of the magic immediates in the embedded image (computed once).
+constexpr int NMAGIC = 6;
 struct PatchSites {
-    std::vector<size_t> off[4];
+    std::vector<size_t> off[NMAGIC];
     bool ok = false;
 };
 static const PatchSites &patch_sites()
@@ -256,17 +257,18 @@ static const PatchSites &patch_sites()
         const unsigned char *img = patch_image();
         const size_t n = patch_image_size();
         if (!img || n < 16) return p;
-        const uint32_t magic[4] = {SWB_K_NGE2, SWB_K_NGF2, SWB_K_NGE16, SWB_K_NGF16};
+        const uint32_t magic[NMAGIC] = {SWB_K_NGE2, SWB_K_NGF2, SWB_K_NGE16, SWB_K_NGF16, SWB_K_NGE1, SWB_K_NGF1};
         for (size_t o = 0; o + 4 <= n; o++) {
             uint32_t w;
             memcpy(&w, img + o, 4);
-            for (int k = 0; k < 4; k++)
+            for (int k = 0; k < NMAGIC; k++)
                 if (w == magic[k]) {
                     if (o % 16 != 4) return p;  // not an instruction immediate: refuse to patch
                     p.off[k].push_back(o);
                 }
         }
-        p.ok = !p.off[0].empty() && !p.off[2].empty() && !p.off[3].empty();
+        p.ok = !p.off[0].empty() && !p.off[2].empty() && !p.off[3].empty() && !p.off[4].empty() &&
+               !p.off[5].empty();
         return p;
     }();
     return ps;
@@ -597,9 +599,18 @@ static double model_fill_time(long long nb, long long P, long long n, long long 
 // image on first use (at most 4 images per context, oldest unloaded first).
 // nullptr: not available (no embedded image, SWB_PATCH=0, or a load error),
 // and the caller runs the runtime-operand kernel (same results).
-static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf)
+static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf, int kind = 0)
 {
-    if (!ctx->patch || !V.packed_name[0]) return nullptr;
+    // kind 0: packed; 1: int32 local; 2: int32 global (default geometry only)
+    char name[96];
+    if (kind == 0) {
+        if (!V.packed_name[0]) return nullptr;
+        snprintf(name, sizeof(name), "%s", V.packed_name);
+    } else {
+        if (V.alpha != 16 || V.nw != 8 || V.w != 64) return nullptr;
+        snprintf(name, sizeof(name), "_ZN3swb14sw_fill_kernelILi16ELi8ELi64ELb%dEEEvNS_8FillArgsE", kind == 1 ? 1 : 0);
+    }
+    if (!ctx->patch) return nullptr;
     const PatchSites &ps = patch_sites();
     if (!ps.ok) return nullptr;
     const int vidx = (int)(&V - &variant_for(0));
@@ -609,10 +620,11 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf)
         if (q.ge == ge && q.gf == gf) P = &q;
     if (!P) {
         std::vector<unsigned char> img(patch_image(), patch_image() + patch_image_size());
-        const uint32_t val[4] = {(uint32_t)(-(ge * 0x10001)), (uint32_t)(-(gf * 0x10001)),
-                                 ((0x10000u - (uint32_t)ge) & 0xffffu) * 0x10001u,
-                                 ((0x10000u - (uint32_t)gf) & 0xffffu) * 0x10001u};
-        for (int k = 0; k < 4; k++)
+        const uint32_t val[NMAGIC] = {(uint32_t)(-(ge * 0x10001)), (uint32_t)(-(gf * 0x10001)),
+                                      ((0x10000u - (uint32_t)ge) & 0xffffu) * 0x10001u,
+                                      ((0x10000u - (uint32_t)gf) & 0xffffu) * 0x10001u, (uint32_t)(-ge),
+                                      (uint32_t)(-gf)};
+        for (int k = 0; k < NMAGIC; k++)
             for (size_t o : ps.off[k]) memcpy(img.data() + o, &val[k], 4);
         PatchedSet q;
         q.ge = ge;
@@ -629,20 +641,20 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf)
         ctx->patched.push_back(q);
         P = &ctx->patched.back();
     }
-    if (!P->fn[vidx]) {
+    if (!P->fn[kind][vidx]) {
         cudaKernel_t k = nullptr;
-        if (cudaLibraryGetKernel(&k, P->lib, V.packed_name) != cudaSuccess || !k) {
+        if (cudaLibraryGetKernel(&k, P->lib, name) != cudaSuccess || !k) {
             cudaGetLastError();
             return nullptr;
         }
-        if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)V.smem16) !=
-            cudaSuccess) {
+        if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)(kind == 0 ? V.smem16 : V.smem)) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
         }
-        P->fn[vidx] = (const void *)k;
+        P->fn[kind][vidx] = (const void *)k;
     }
-    return P->fn[vidx];
+    return P->fn[kind][vidx];
 }
 
 static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
@@ -758,11 +770,9 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     const void *fill_fn = use16 ? V.packed_fn : (J.local ? V.local_fn : V.global_fn);
     const size_t fill_smem = use16 ? V.smem16 : V.smem;
     bool patched = false;
-    if (use16) {
-        if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge)) {
-            fill_fn = pf;
-            patched = true;
-        }
+    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, use16 ? 0 : J.local ? 1 : 2)) {
+        fill_fn = pf;
+        patched = true;
     }
     const int block = V.nw * 32 + (use16 ? V.io_warps : 1) * 32;
     int blocks_per_sm = 0;

@@ -164,6 +164,21 @@ __device__ __forceinline__ int lane_id()
     return l;
 }
 
+// -G_ext and -G_first of the int32 cell update: instruction immediates in the
+// patched image (sw_fill16_patch.cu, SWB_PATCH), kernel arguments otherwise.
+#ifndef SWB_I32MODE
+#define SWB_I32MODE 1  // int32 cell update: 1 = D form (one VIADDMNMX per row on the F chain), 0 = H form
+#endif
+#define SWB_K_NGE1 0x2ae8944au
+#define SWB_K_NGF1 0x625558ecu
+#ifdef SWB_PATCH
+#define NGE(a) ((int)SWB_K_NGE1)
+#define NGF(a) ((int)SWB_K_NGF1)
+#else
+#define NGE(a) (-(a).ge)
+#define NGF(a) (-(a).gf)
+#endif
+
 // x * one + y through the FMA pipe (IMAD); `one` is a runtime 1 so ptxas
 // cannot fold the add into an ALU-pipe VIADDMNMX.
 __device__ __forceinline__ int imad(int x, int one, int y)
@@ -282,35 +297,110 @@ struct Fill {
         int tdA = L.tprev;  // t(r0-1, j0-1)
         int tdB = a_t;      // t(r0-1, j0)
         L.tprev = b_t;
+#if SWB_I32MODE == 1
+        // F of the lane's first row from the row above (t, F): Eq. 3
+        int fA = __viaddmax_s32(a_f, NGE(a), a_t), fB = __viaddmax_s32(b_f, NGE(a), b_t);
         int tuA = a_t, fuA = a_f, tuB = b_t, fuB = b_f;
-        const int nge = -a.ge;
         const int gf = a.gf;
+        int *spp = sp_ptr;
+#pragma unroll
+        for (int r = 0; r < ALPHA; r++) {
+            // column j0, with D = max(H_diag + p, E[, 0]) (Eq. 1 without F):
+            //   E  = max(E_left - G_ext, t_left)            Eq. 2 (t = H - G_first)
+            //   Dg = D - G_first
+            //   t  = max(F - G_first, Dg)                    (H = max(D, F), Eq. 1)
+            //   F' = max(F - G_ext, Dg)                      Eq. 3 for the next row
+            // F' = max(F - G_ext, t) = max(F - G_ext, D - G_first, F - G_first) and
+            // G_ext <= G_first, so the chain down the rows is one VIADDMNMX per row;
+            // the constants are immediates in the patched image.
+            const int eA = __viaddmax_s32(L.e[r], NGE(a), L.t[r]);
+            const int pA = prmt(L.P[r], PADPROF, sl.x);
+            const int xA = tdA + pA;
+            const int dA = LOCAL ? __vimax_s32_relu(eA, xA) : max(eA, xA);
+            const int dgA = dA + NGF(a);
+            const int tA = __viaddmax_s32(fA, NGF(a), dgA);
+            fuA = fA;  // F of this row
+            fA = __viaddmax_s32(fA, NGE(a), dgA);
+            tdA = L.t[r];
+            tuA = tA;
+            // column j0 + 1 (one row behind column j0 in the dependency chain)
+            const int eB = __viaddmax_s32(eA, NGE(a), tA);
+            const int pB = prmt(L.P[r], PADPROF, sl.y);
+            const int xB = tdB + pB;
+            const int dB = LOCAL ? __vimax_s32_relu(eB, xB) : max(eB, xB);
+            const int dgB = dB + NGF(a);
+            const int tB = __viaddmax_s32(fB, NGF(a), dgB);
+            fuB = fB;
+            fB = __viaddmax_s32(fB, NGE(a), dgB);
+            tdB = tA;
+            tuB = tB;
+            L.e[r] = eB;
+            L.t[r] = tB;
+            tmax = __vimax3_s32(tmax, tA, tB);  // the tile maximum of t = H - G_first
+            if (SPM == 2 || TRACK) {
+                const int hA = tA + gf, hB = tB + gf;
+                if (SPM == 2) {
+                    if (smask & (1u << r)) {
+                        if (j0 < X.w) { spp[j0] = hA; spp[X.sp_ld + j0] = fuA; }
+                        if (j0 + 1 < X.w) { spp[j0 + 1] = hB; spp[X.sp_ld + j0 + 1] = fuB; }
+                        spp += X.sp_stride;
+                    }
+                }
+                if (TRACK) {
+                    const int row = row1 + r;
+                    if (row <= a.m) {
+                        const int cA = X.col0 + j0 + 1, cB = cA + 1;  // global DP columns
+                        if (j0 + 1 <= X.hw) {
+                            if (LOCAL) {
+                                if (better(hA, row, cA, bs, bi, bj)) { bs = hA; bi = row; bj = cA; }
+                            } else if (hA == a.goal && (row < bi || (row == bi && cA < bj))) {
+                                bi = row; bj = cA;
+                            }
+                        }
+                        if (j0 + 2 <= X.hw) {
+                            if (LOCAL) {
+                                if (better(hB, row, cB, bs, bi, bj)) { bs = hB; bi = row; bj = cB; }
+                            } else if (hB == a.goal && (row < bi || (row == bi && cB < bj))) {
+                                bi = row; bj = cB;
+                            }
+                        }
+                    }
+                }
+            }
+            if (CAP) {  // the stripe's last column: hand (t, E) to the right neighbour
+                if (j0 == X.jcap) X.rbrow[r] = make_int2(tA, eA);
+                if (j0 + 1 == X.jcap) X.rbrow[r] = make_int2(tB, eB);
+            }
+        }
+#else
+        int tuA = a_t, fuA = a_f, tuB = b_t, fuB = b_f;
+                const int gf = a.gf;
         int *spp = sp_ptr;
 #pragma unroll
         for (int r = 0; r < ALPHA; r++) {
             // column j0: Eq. 2, Eq. 3, Eq. 1 (p' = p + G_first applied to t = H - G_first).
             // Instruction mix balanced over the ALU pipe (DPX max, PRMT) and the
             // FMA pipe (the adds, as IMAD with a runtime 1): DESIGN.md section 5.
-            const int eA = __viaddmax_s32(L.e[r], nge, L.t[r]);
-            fuA = max(imad(fuA, a.one, nge), tuA);
+            const int eA = __viaddmax_s32(L.e[r], NGE(a), L.t[r]);
+            fuA = max(fuA + NGE(a), tuA);
             const int pA = prmt(L.P[r], PADPROF, sl.x);
-            const int xA = imad(tdA, a.one, pA);
+            const int xA = tdA + pA;
             const int hA = LOCAL ? __vimax3_s32_relu(eA, fuA, xA) : __vimax3_s32(eA, fuA, xA);
             tdA = L.t[r];
-            const int tA = imad(hA, a.one, -gf);
+            const int tA = hA + NGF(a);
             tuA = tA;
             // column j0 + 1 (one row behind column j0 in the dependency chain)
-            const int eB = __viaddmax_s32(eA, nge, tA);
-            fuB = max(imad(fuB, a.one, nge), tuB);
+            const int eB = __viaddmax_s32(eA, NGE(a), tA);
+            fuB = max(fuB + NGE(a), tuB);
             const int pB = prmt(L.P[r], PADPROF, sl.y);
-            const int xB = imad(tdB, a.one, pB);
+            const int xB = tdB + pB;
             const int hB = LOCAL ? __vimax3_s32_relu(eB, fuB, xB) : __vimax3_s32(eB, fuB, xB);
             tdB = tA;
-            const int tB = imad(hB, a.one, -gf);
+            const int tB = hB + NGF(a);
             tuB = tB;
             L.e[r] = eB;
             L.t[r] = tB;
-            tmax = __vimax3_s32(tmax, hA, hB);
+            tmax = __vimax3_s32(tmax, tA, tB);  // tile maximum of t = H - G_first
             if (SPM == 2) {
                 if (smask & (1u << r)) {
                     if (j0 < X.w) { spp[j0] = hA; spp[X.sp_ld + j0] = fuA; }
@@ -343,6 +433,7 @@ struct Fill {
                 }
             }
         }
+#endif
         L.out_t0 = tuA; L.out_f0 = fuA;
         L.out_t1 = tuB; L.out_f1 = fuB;
         if (SPM == 1 && sp_ptr != nullptr) {
@@ -640,7 +731,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                     } else {
                         tmax = F::template tile_fast<false>(a, X, L, c, lane, rin, rout, selr_s, nullptr);
                     }
-                    if (__any_sync(0xffffffffu, tmax >= thr)) {
+                    if (__any_sync(0xffffffffu, tmax >= thr - a.gf)) {  // tmax is over t = H - G_first
                         // exact replay of this tile from the saved state (rare)
                         F::restore(L, sv, lane);
                         const int obs = bs, obi = bi, obj = bj;

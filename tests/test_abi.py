@@ -87,3 +87,16 @@ def test_flush_interval_helper_matches_table_viii(lib):
         assert pred == l2 if gib in (10, 30, 50) else abs(pred - l2) <= 1
     assert lib.sw_special_row_interval_for_budget(0, 5, 256, 1) == 0
     assert lib.sw_special_row_interval_for_budget(10, 10, 256, 1 << 40) == 256  # at least one block
+
+
+def test_patch_cubin_immediates(lib):
+    """The embedded patchable image: every magic gap-penalty
+    word is a 32-bit SASS immediate field (byte 4 of a 16-byte instruction),
+    no negated copy exists, and the library embeds exactly this image."""
+    from paper_conf_ipps_sandesm11_b200 import build
+
+    counts = build.check_patch_sites(build.PATCH_CUBIN)
+    for name in ("NGE2", "NGE16", "NGF16", "NGE1", "NGF1"):
+        assert counts[name] > 0, counts
+    so = open(os.path.join(ROOT, "paper_conf_ipps_sandesm11_b200", "libcudalign_b200.so"), "rb").read()
+    assert open(build.PATCH_CUBIN, "rb").read() in so
