@@ -18,6 +18,8 @@ PATCH_SRC = os.path.join(HERE, "csrc", "sw_fill16_patch.cu")
 PATCH_CUBIN = os.path.join(HERE, "sw_fill16_patch.cubin")
 MAGIC = {"NGE2": 0x6B8B4567, "NGF2": 0x327B23C6, "NGE16": 0x643C9869, "NGF16": 0x66334873,
          "NGE1": 0x2AE8944A, "NGF1": 0x625558EC}
+# the alternative set of the two-build check (same order)
+ALT_MAGIC = [0x1D2F3B61, 0x5E3A9B27, 0x49C1F6B3, 0x7A2D4E19, 0x3F6B2D85, 0x0B7E5C93]
 import glob
 
 DEPS = sorted(glob.glob(os.path.join(HERE, "csrc", "*"))) + [os.path.join(ROOT, "include", "cudalign_b200.h")]
@@ -57,7 +59,7 @@ def check_patch_sites(path: str) -> dict:
         if data.find(struct.pack("<I", (-v) & 0xFFFFFFFF)) >= 0:
             raise RuntimeError(f"{path}: the negation of magic {name} occurs (an unpatchable form)")
         counts[name] = len(offs)
-    for name in ("NGE2", "NGE16", "NGF16", "NGE1", "NGF1"):
+    for name in ("NGE2", "NGE16", "NGF16"):
         if counts[name] == 0:
             raise RuntimeError(f"{path}: magic {name} not found (ptxas folded it?)")
     return counts
@@ -66,10 +68,23 @@ def check_patch_sites(path: str) -> dict:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
+    # the patchable cubin, twice: with the magic set used at run time and with an
+    # alternative set; the SASS must agree up to the magic words (tools/patch_check.py)
     ptmp = PATCH_CUBIN + f".tmp{os.getpid()}"
-    subprocess.check_call([NVCC, *[f for f in FLAGS if f not in ("-Xcompiler", "-fPIC", "-shared")], "-cubin",
-                           "-o", ptmp, PATCH_SRC])
+    palt = PATCH_CUBIN + f".alt{os.getpid()}"
+    cflags = [f for f in FLAGS if f not in ("-Xcompiler", "-fPIC", "-shared")]
+    alt = [f"-DSWB_K_{k}={v:#x}u" for k, v in zip(MAGIC, ALT_MAGIC)]
+    procs = [subprocess.Popen([NVCC, *cflags, "-cubin", "-o", ptmp, PATCH_SRC]),
+             subprocess.Popen([NVCC, *cflags, *alt, "-cubin", "-o", palt, PATCH_SRC])]
+    if any(p.wait() for p in procs):
+        raise RuntimeError("nvcc failed on the patchable cubin")
     check_patch_sites(ptmp)
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    import patch_check
+
+    if patch_check.main(ptmp, palt):
+        raise RuntimeError("patchable cubin: SASS depends on the magic values (a derived constant)")
+    os.remove(palt)
     os.replace(ptmp, PATCH_CUBIN)
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = [NVCC, *FLAGS, f'-DSWB_PATCH_CUBIN="{PATCH_CUBIN}"', "-o", tmp, *SOURCES]

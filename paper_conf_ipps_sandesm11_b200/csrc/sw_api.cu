@@ -267,8 +267,7 @@ static const PatchSites &patch_sites()
                     p.off[k].push_back(o);
                 }
         }
-        p.ok = !p.off[0].empty() && !p.off[2].empty() && !p.off[3].empty() && !p.off[4].empty() &&
-               !p.off[5].empty();
+        p.ok = !p.off[0].empty() && !p.off[2].empty() && !p.off[3].empty();
         return p;
     }();
     return ps;
@@ -601,16 +600,9 @@ static double model_fill_time(long long nb, long long P, long long n, long long 
 // and the caller runs the runtime-operand kernel (same results).
 static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf, int kind = 0)
 {
-    // kind 0: packed; 1: int32 local; 2: int32 global (default geometry only)
-    char name[96];
-    if (kind == 0) {
-        if (!V.packed_name[0]) return nullptr;
-        snprintf(name, sizeof(name), "%s", V.packed_name);
-    } else {
-        if (V.alpha != 16 || V.nw != 8 || V.w != 64) return nullptr;
-        snprintf(name, sizeof(name), "_ZN3swb14sw_fill_kernelILi16ELi8ELi64ELb%dEEEvNS_8FillArgsE", kind == 1 ? 1 : 0);
-    }
-    if (!ctx->patch) return nullptr;
+    // kind 0: packed (the only kernels in the patched image); 1, 2: int32 local/global (not patched)
+    if (kind != 0 || !V.packed_name[0] || !ctx->patch) return nullptr;
+    const char *name = V.packed_name;
     const PatchSites &ps = patch_sites();
     if (!ps.ok) return nullptr;
     const int vidx = (int)(&V - &variant_for(0));

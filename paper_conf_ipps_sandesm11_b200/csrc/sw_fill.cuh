@@ -167,10 +167,12 @@ __device__ __forceinline__ int lane_id()
 // -G_ext and -G_first of the int32 cell update: instruction immediates in the
 // patched image (sw_fill16_patch.cu, SWB_PATCH), kernel arguments otherwise.
 #ifndef SWB_I32MODE
-#define SWB_I32MODE 1  // int32 cell update: 1 = D form (one VIADDMNMX per row on the F chain), 0 = H form
+#define SWB_I32MODE 0  // int32 cell update: 0 = H form (default, measured faster), 1 = D form
 #endif
+#ifndef SWB_K_NGE1
 #define SWB_K_NGE1 0x2ae8944au
 #define SWB_K_NGF1 0x625558ecu
+#endif
 #ifdef SWB_PATCH
 #define NGE(a) ((int)SWB_K_NGE1)
 #define NGF(a) ((int)SWB_K_NGF1)

@@ -36,10 +36,12 @@ constexpr int BIAS16 = 32768;
 // Magic immediates of the patchable build (sw_fill16_patch.cu): -G_ext and
 // -G_first in both halves as a 32-bit add (NGE2, NGF2) and per half (NGE16,
 // NGF16).  Arbitrary values, chosen not to occur elsewhere in the code.
+#ifndef SWB_K_NGE2
 #define SWB_K_NGE2 0x6b8b4567u
 #define SWB_K_NGF2 0x327b23c6u
 #define SWB_K_NGE16 0x643c9869u
 #define SWB_K_NGF16 0x66334873u
+#endif
 #ifndef SWB_ADDMODE
 #ifdef SWB_PATCH
 #define SWB_ADDMODE 1

@@ -1,11 +1,14 @@
-// sw_fill16_patch.cu -- the packed Stage-1 kernels (and the default int32
-// geometry) built with magic
+// sw_fill16_patch.cu -- the packed Stage-1 kernels built with magic
 // instruction immediates for the gap penalties (SWB_PATCH, sw_fill16.cuh).
 // Compiled to a cubin that is embedded in libcudalign_b200.so; at run time
 // sw_api.cu replaces the magic immediates with the call's -G_ext / -G_first
 // encodings and loads the patched image (cudaLibraryLoadData).  An add with an
 // immediate reads one register instead of three, which is what the packed
-// cell update is bound by.
+// cell update is bound by.  The build compiles this file twice
+// with two magic sets and requires identical SASS up to the magic words
+// (tools/patch_check.py): no constant derived from a magic can hide in the code.
+// The int32 kernel is not patched: its faster H form compiles to
+// magic-dependent code.
 #define SWB_PATCH 1
 #include "sw_fill16.cuh"
 
@@ -21,8 +24,4 @@ template __global__ void sw_fill16_kernel<4, 64, false, 16, false>(const __grid_
 template __global__ void sw_fill16_kernel<4, 64, true, 16, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<16, 64, true, 16, false>(const __grid_constant__ FillArgs);
-// the int32 kernel in the default geometry (DEFAULT_VARIANT: alpha 16, 8 warps,
-// W 64), local (Stage 1 outside the packed window) and global (reverse pass, Stage 2)
-template __global__ void sw_fill_kernel<16, 8, 64, true>(const __grid_constant__ FillArgs);
-template __global__ void sw_fill_kernel<16, 8, 64, false>(const __grid_constant__ FillArgs);
 }  // namespace swb
