@@ -129,3 +129,18 @@ def test_patch_on_off_identical(ctx, scoring):
     assert out[0][0] == want
     for (r, h, f), (_, oh, of) in zip(out[0][1], orows):
         assert np.array_equal(h, oh) and np.array_equal(f, of), r
+
+
+def test_patch_image_cache_eviction(ctx):
+    """More distinct (G_open, G_ext) pairs than the per-context image cache
+    holds (4): images are evicted and reloaded, results stay exact."""
+    A, B = synth.random_pair(4242, 2500, 2200, plant_len=1200, s=0.04, g=0.01)
+    scorings = [(1, -3, 3, 2), (1, -2, 2, 1), (2, -3, 4, 1), (1, -1, 1, 2), (3, -2, 0, 3), (2, -2, 5, 2), (1, -3, 3, 2)]
+    for sc in scorings:
+        got, rows = ctx.align_stage1(A, B, *sc, k=32, keep_rows=True)
+        st = ctx.stats()
+        assert st["alpha"] < 0 and st["patched"] == 1, (sc, st)
+        want, orows = oracle.stage1(_s(A), _s(B), *sc, k=32)
+        assert got.astuple() == want, sc
+        for (r, h, f), (_, oh, of) in zip(rows, orows):
+            assert np.array_equal(h, oh) and np.array_equal(f, of), (sc, r)
