@@ -108,12 +108,14 @@ struct Variant {
     int io_warps;           // 1, or 0 for the cooperative-I/O packed kernel (block = (nw + io) warps)
     int skew_tiles;         // int32 kernel: tiles past the last column lane 31 needs (ceil(62 / W))
     char packed_name[96];   // mangled name of the packed kernel in the patchable cubin ("" : none)
+    const void *packed_global_fn;  // packed kernel in global (reverse-pass) mode, alpha 32 x 8 warps only
+    char packed_global_name[96];
 };
 
 template <int NW, int W, bool COOP, int NS>
 static void packed_name(Variant &v)
 {
-    snprintf(v.packed_name, sizeof(v.packed_name), "_ZN3swb16sw_fill16_kernelILi%dELi%dELb%dELi%dELb0EEEvNS_8FillArgsE",
+    snprintf(v.packed_name, sizeof(v.packed_name), "_ZN3swb16sw_fill16_kernelILi%dELi%dELb%dELi%dELb0ELb1EEEvNS_8FillArgsE",
              NW, W, COOP ? 1 : 0, NS);
 }
 
@@ -131,12 +133,20 @@ static Variant make_variant()
     v.io_warps = 1;
     v.skew_tiles = 1;
     v.packed_name[0] = 0;
+    v.packed_global_fn = nullptr;
+    v.packed_global_name[0] = 0;
     if constexpr (ALPHA == 32) {
         // packed kernel only (16 slots per lane); int32 work falls back to the default geometry
         v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, 16, SPLIT>;
         v.io_warps = COOP ? 0 : 1;
         v.smem16 = Fill16<NW, W, 16, SPLIT>::smem_bytes();
         if constexpr (!SPLIT) packed_name<NW, W, COOP, 16>(v);
+        if constexpr (NW == 8 && !COOP && !SPLIT) {
+            // the reverse pass (a8) on the packed kernel
+            v.packed_global_fn = (const void *)&sw_fill16_kernel<NW, W, false, 16, false, false>;
+            snprintf(v.packed_global_name, sizeof(v.packed_global_name),
+                     "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi16ELb0ELb0EEEvNS_8FillArgsE", NW, W);
+        }
         return v;
     } else {
         v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
@@ -241,7 +251,7 @@ static size_t patch_image_size() { return 0; }
 struct PatchedSet {
     int ge = -1, gf = -1;
     cudaLibrary_t lib = nullptr;
-    const void *fn[3][NVARIANTS] = {};  // [packed, int32 local, int32 global][variant]
+    const void *fn[4][NVARIANTS] = {};  // [packed, int32 local, int32 global, packed global][variant]
 };
 
 // Offsets of the magic immediates in the embedded image (computed once).
@@ -409,6 +419,8 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
             if (v.local_fn) cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
             if (v.global_fn) cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
             if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
+            if (v.packed_global_fn)
+                cudaFuncSetAttribute(v.packed_global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
         }
         if ((e = cudaGetLastError()) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaFuncSetAttribute"); break; }
         if (const char *ov = getenv("SWB_VARIANT")) ctx->variant_override = atoi(ov);
@@ -600,9 +612,11 @@ static double model_fill_time(long long nb, long long P, long long n, long long 
 // and the caller runs the runtime-operand kernel (same results).
 static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf, int kind = 0)
 {
-    // kind 0: packed (the only kernels in the patched image); 1, 2: int32 local/global (not patched)
-    if (kind != 0 || !V.packed_name[0] || !ctx->patch) return nullptr;
-    const char *name = V.packed_name;
+    // kind 0: packed local, 3: packed global (the kernels in the patched image);
+    // 1, 2: int32 local/global (not patched)
+    if ((kind != 0 && kind != 3) || !ctx->patch) return nullptr;
+    const char *name = kind == 0 ? V.packed_name : V.packed_global_name;
+    if (!name[0]) return nullptr;
     const PatchSites &ps = patch_sites();
     if (!ps.ok) return nullptr;
     const int vidx = (int)(&V - &variant_for(0));
@@ -640,7 +654,7 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf,
             return nullptr;
         }
         if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)(kind == 0 ? V.smem16 : V.smem)) != cudaSuccess) {
+                                 (int)(kind == 0 || kind == 3 ? V.smem16 : V.smem)) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
         }
@@ -660,6 +674,16 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         return ctx->packed && J.local && V.packed_fn && (J.k == 0 || J.k % V.alpha == 0) &&
                span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
     };
+    if (!J.local) {
+        // reverse pass (a8): the packed kernel in global mode when it qualifies
+        // (alpha 32 x 8 warps geometry; one stripe, no Stage-2 matching or gap anchor)
+        const Variant &V = variant_for(10);
+        const long long span = 32ll * V.alpha + 140;
+        *use16 = ctx->packed && V.packed_global_fn && !J.match && !J.anchor_gap && J.k == 0 && !J.rank_mode &&
+                 J.nv == 1 && (ctx->variant_override < 0 || ctx->variant_override == 10) &&
+                 span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
+        if (*use16) return V;
+    }
     if (ctx->variant_override >= 0) {
         const Variant &V = variant_for(ctx->variant_override);
         *use16 = packed_ok(V);
@@ -759,10 +783,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             return SW_EINVAL;
         }
     }
-    const void *fill_fn = use16 ? V.packed_fn : (J.local ? V.local_fn : V.global_fn);
+    const void *fill_fn = use16 ? (J.local ? V.packed_fn : V.packed_global_fn) : (J.local ? V.local_fn : V.global_fn);
     const size_t fill_smem = use16 ? V.smem16 : V.smem;
     bool patched = false;
-    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, use16 ? 0 : J.local ? 1 : 2)) {
+    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, use16 ? (J.local ? 0 : 3) : J.local ? 1 : 2)) {
         fill_fn = pf;
         patched = true;
     }
@@ -945,7 +969,11 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     }
     {
         void *args[] = {&a};
-        CK(cudaLaunchKernel(fill_fn, dim3(grid), dim3(block), args, fill_smem, st));
+        const cudaError_t le = cudaLaunchKernel(fill_fn, dim3(grid), dim3(block), args, fill_smem, st);
+        if (le != cudaSuccess) {
+            cudaGetLastError();  // not sticky: do not fail the context's next call
+            return cuda_fail(ctx, le, "cudaLaunchKernel(fill)");
+        }
     }
     CK(cudaEventRecord(ctx->ev[2], st));
     sw_reduce_kernel<<<1, 256, 0, st>>>((const int4 *)ctx->slots.p, grid, J.local ? 1 : 0, d_hit_key, J.goal, d_res);

@@ -85,7 +85,7 @@ struct MaxTree {
     }
 };
 
-template <int NW, int W, int NS = 8, bool SPLIT = false>
+template <int NW, int W, int NS = 8, bool SPLIT = false, bool LOCAL = true>
 struct Fill16 {
     static constexpr bool TMTREE = SWB_FMODE == 2 && SWB_TMTREE;
     static constexpr int ALPHA = 2 * NS, BH = ALPHA * 32 * NW;
@@ -349,6 +349,34 @@ struct Fill16 {
             }
             tmax = (tmax & keep) | (tmax_in & ~keep);
         }
+        if (TRACK && !LOCAL) {
+            // Replay of a reverse (global) pass: the first cell in row-major
+            // order with H == goal (reading S10).  Within a step a row occurs
+            // once and the low half's rows precede the high half's; across
+            // steps the running (bi, bj) keeps the lexicographic minimum.
+            // Columns past X.hw cannot hold a start.
+            const int gq = a.goal - a.gf - L.B + BIAS16;  // goal's t in this warp's frame
+            if (gq >= 0 && gq <= 0xffff) {
+                const uint32_t Gt = (uint32_t)gq * 0x10001u;
+                const bool lo_ok = jl >= 0 && jl < X.hw, hi_ok = jl >= 1 && jl - 1 < X.hw;
+                uint32_t lob = 0u, hib = 0u;
+#pragma unroll
+                for (int s = 0; s < NS; s++) {
+                    const uint32_t eq = __vcmpeq2(L.t[s], Gt);
+                    lob |= (eq & 1u) << s;
+                    hib |= (eq >> 31) << s;
+                }
+                lob = lo_ok ? lob : 0u;
+                hib = hi_ok ? hib : 0u;
+                if (lob | hib) {
+                    int row, col;
+                    if (lob) { row = row1 + __ffs(lob) - 1; col = X.col0 + jl + 1; }
+                    else { row = row1 + NS + __ffs(hib) - 1; col = X.col0 + jl; }
+                    if (row <= a.m && (row < bi || (row == bi && col < bj))) { bi = row; bj = col; }
+                }
+            }
+            return 0;
+        }
         if (TRACK) {
             // Replay: the step's cells are t[s] + G_first now.  The best cell
             // of the step (max, then min row; a row occurs once per step) is
@@ -455,7 +483,7 @@ struct Fill16 {
         L.B += d;
         L.adj = BIAS16 - L.B;
         L.Bm = L.B - BIAS16;
-        const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
+        const int fl = LOCAL ? min(max(BIAS16 - L.B, 0), 0xffff) : 0;  // global: no 0 floor
         L.FL = (uint32_t)fl * 0x10001u;
     }
 
@@ -482,7 +510,7 @@ struct Fill16 {
         L.B = sv[(2 * NS + 2) * 32 + lane];
         L.adj = BIAS16 - L.B;
         L.Bm = L.B - BIAS16;
-        const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
+        const int fl = LOCAL ? min(max(BIAS16 - L.B, 0), 0xffff) : 0;
         L.FL = (uint32_t)fl * 0x10001u;
     }
 };
@@ -491,10 +519,14 @@ struct Fill16 {
 // warps that also share the I/O (each loads and drains W / NW columns per
 // tile), so all four SMSPs carry the same number of compute warps (16 warps:
 // 4 each) -- the lockstep interval otherwise waits for the busier SMSPs.
-template <int NW, int W, bool COOP = false, int NS = 8, bool SPLIT = false>
+// LOCAL = false: the reverse pass of sw_reverse_goal (a8): anchored global
+// recurrence with no 0 floor (FL = 0), global boundaries, first-hit tracking of
+// the goal and the early exit after the band with the first hit, as in the
+// int32 kernel; one stripe, no special rows, no Stage-2 matching (host checks).
+template <int NW, int W, bool COOP = false, int NS = 8, bool SPLIT = false, bool LOCAL = true>
 __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
 {
-    using F = Fill16<NW, W, NS, SPLIT>;
+    using F = Fill16<NW, W, NS, SPLIT, LOCAL>;
     constexpr int ALPHA = F::ALPHA;
     constexpr int BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS;
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -514,12 +546,12 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         return (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
     };
     const bool has_left = S.lb != nullptr, has_right = S.rb != nullptr;
-    int bs = 0, bi = 0, bj = 0;
+    int bs = 0, bi = LOCAL ? 0 : INT_MAX, bj = LOCAL ? 0 : INT_MAX;
     long long nrep = 0;
     if (*a.err) return;
     StepInfo X;
     X.w = S.w;
-    X.hw = S.w;
+    X.hw = LOCAL ? S.w : min(S.w, a.hit_w);
     X.col0 = S.col0;
     X.sp_ld = S.sp_ld;
     X.sp_stride = S.sp_stride;
@@ -531,6 +563,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
     for (;;) {
         if (threadIdx.x == 0) {
             int b = atomicAdd(S.ticket, 1);
+            if (!LOCAL && b > ld_relaxed(a.hit_band)) b = a.nb;
             if (ld_relaxed(a.err)) b = a.nb;
             s_band = b;
             s_abort = 0;
@@ -554,13 +587,18 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     tv[r] = v.x;
                     ev[r] = v.y;
                 }
-            } else {
+            } else if (LOCAL) {
 #pragma unroll
                 for (int r = 0; r < ALPHA; r++) { tv[r] = -a.gf; ev[r] = -a.gf; }  // E(i,0) := t(i,0), exact
+            } else {
+                // global: H(i,0) = -(G_open + i G_ext) (reading S9); E(i,0) := t(i,0), exact
+#pragma unroll
+                for (int r = 0; r < ALPHA; r++) { tv[r] = -(a.go + (row0 + r + 1) * a.ge) - a.gf; ev[r] = tv[r]; }
             }
             int tp;
             if (from_left && row0 > 0) tp = ld_sys_int2(S.lb + row0).x;
-            else tp = -a.gf;
+            else if (LOCAL || row0 == 0) tp = -a.gf;  // t(0,0): H(0,0) = 0
+            else tp = -(a.go + row0 * a.ge) - a.gf;
             L.B = __shfl_sync(0xffffffffu, tv[0], 0);
             L.adj = BIAS16 - L.B;
             L.Bm = L.B - BIAS16;
@@ -571,7 +609,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             }
             L.tprev = pk(F::tofr(L, tp), F::tofr(L, tp));
             L.fn = L.t[NS - 1];  // only feeds the high half at column -1 (kept by GUARD)
-            const int fl = min(max(BIAS16 - L.B, 0), 0xffff);
+            const int fl = LOCAL ? min(max(BIAS16 - L.B, 0), 0xffff) : 0;
             L.FL = (uint32_t)fl * 0x10001u;
         };
         if (warp < NW) {
@@ -601,6 +639,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 if (lane == 0) {
                     const unsigned long long t0 = gtimer();
                     while (ld_acquire(S.progress + b - 1) < need) {
+                        if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
                         if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                         __nanosleep(64);
                     }
@@ -610,7 +649,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = c * W + x;
-                rings[F::ridx(col)] = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
+                rings[F::ridx(col)] = (b == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb + col);
                 // pad columns: code 0 (harmless, see header)
                 F::put_sel(selr, col, code_at(col), code_at(col - 1));
             }
@@ -670,7 +709,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         };
         auto coop_fetch = [&](int c, int2 &v, uint32_t &code) {  // issue the loads (results used after compute)
             const int col = c * W + warp * CPW + lane;
-            v = (b == 0) ? top_boundary<true>(a, S.col0 + col) : __ldcg(S.rowb + col);
+            v = (b == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb + col);
             code = code_at(col) | (code_at(col - 1) << 2);
         };
         auto coop_put = [&](int c, int2 v, uint32_t code) {
@@ -726,7 +765,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     }
                     if (c > 0) F::rebase(a, L);
                     F::convert_ring(a, L, rings + warp * F::RS, crings + warp * W, c, lane);
-                    const int thr = max(max(bs, ld_relaxed(a.gbest)), 1);
+                    const int thr = LOCAL ? max(max(bs, ld_relaxed(a.gbest)), 1) : a.goal;
                     F::save(L, sv, lane);
                     uint32_t tm;
                     const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
@@ -749,16 +788,22 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     const int tmax = F::toabs(L, max(lo16(tm), hi16(tm))) + F::tmax_off(a);
                     if (__any_sync(0xffffffffu, tmax >= thr)) {
                         F::restore(L, sv, lane);
-                        const int obs = bs;
+                        const int obs = bs, obi = bi, obj = bj;
                         F::template tile<true, true, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
                         if (lane == 0) nrep++;
-                        if (bs > obs) atomicMax(a.gbest, bs);
+                        if (LOCAL) {
+                            if (bs > obs) atomicMax(a.gbest, bs);
+                        } else if (bi != obi || bj != obj) {
+                            atomicMin(a.hit_key, ((unsigned long long)(unsigned)bi << 32) | (unsigned)bj);
+                            atomicMin(a.hit_band, b);
+                        }
                     }
                 }
             } else {
                 if (s + 1 < NT) io_load(s + 1);
                 const int cd = s - 1 - 2 * (NW - 1);
                 if (cd >= 0) io_drain(cd);
+                if (!LOCAL && lane == 0 && ld_relaxed(a.hit_band) < b) s_abort = 1;
             }
             const int cdc = s - 1 - 2 * (NW - 1);
             if constexpr (COOP) {
@@ -793,20 +838,22 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
     }
 
     if (lane == 0 && nrep) atomicAdd(a.replays, (unsigned long long)nrep);
-    __shared__ int4 red[NW + 1];
-    for (int o = 16; o > 0; o >>= 1) {
-        const int s2 = __shfl_down_sync(0xffffffffu, bs, o);
-        const int i2 = __shfl_down_sync(0xffffffffu, bi, o);
-        const int j2 = __shfl_down_sync(0xffffffffu, bj, o);
-        if (better(s2, i2, j2, bs, bi, bj)) { bs = s2; bi = i2; bj = j2; }
-    }
-    if (lane == 0) red[warp] = make_int4(bs, bi, bj, 0);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int4 r = make_int4(0, 0, 0, 0);
-        for (int w = 0; w < NW; w++)
-            if (red[w].x > 0 && better(red[w].x, red[w].y, red[w].z, r.x, r.y, r.z)) r = red[w];
-        a.slots[blockIdx.x] = r;
+    if constexpr (LOCAL) {  // global: the hits went to hit_key / hit_band
+        __shared__ int4 red[NW + 1];
+        for (int o = 16; o > 0; o >>= 1) {
+            const int s2 = __shfl_down_sync(0xffffffffu, bs, o);
+            const int i2 = __shfl_down_sync(0xffffffffu, bi, o);
+            const int j2 = __shfl_down_sync(0xffffffffu, bj, o);
+            if (better(s2, i2, j2, bs, bi, bj)) { bs = s2; bi = i2; bj = j2; }
+        }
+        if (lane == 0) red[warp] = make_int4(bs, bi, bj, 0);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int4 r = make_int4(0, 0, 0, 0);
+            for (int w = 0; w < NW; w++)
+                if (red[w].x > 0 && better(red[w].x, red[w].y, red[w].z, r.x, r.y, r.z)) r = red[w];
+            a.slots[blockIdx.x] = r;
+        }
     }
 }
 

@@ -22,4 +22,10 @@ for rep in range(2):
 print(f"m={m} best={r.astuple()} start={s.astuple()} int32 stage1 fill {st1['fill_ms']:.1f} ms "
       f"({len(A) * len(B) / st1['fill_ms'] / 1e6:.0f} GCUPS, patched={st1['patched']}); reverse fill {st2['fill_ms']:.1f} ms "
       f"({r.i * r.j / st2['fill_ms'] / 1e6:.0f} GCUPS, patched={st2['patched']})")
+ctx.set_kernel(-1, True)  # automatic: the packed kernel in global mode
+for rep in range(2):
+    s = ctx.reverse_goal(A, r.i, B, r.j, r.score, 1, -3, 3, 2)
+    st3 = ctx.stats()
+print(f"  packed reverse fill {st3['fill_ms']:.1f} ms ({r.i * r.j / st3['fill_ms'] / 1e6:.0f} GCUPS, alpha={st3['alpha']}, "
+      f"patched={st3['patched']}) start={s.astuple()}")
 ctx.close()
