@@ -314,7 +314,10 @@ class Context:
         (P:281), partitions, mm_levels."""
         pa, m, ka = _as_bytes_ptr(A)
         pb, n, kb = _as_bytes_ptr(B)
-        cap1 = cap2 = 1024
+        # gap-run buffers sized for typical alignments (a run every >= 64 columns),
+        # so the call is not repeated; sw_align reports SW_ERANGE with the counts
+        # if they are too small, and the call is retried with exact sizes
+        cap1 = cap2 = max(1024, min(m, n) // 64)
         while True:
             g1 = (_Gap * cap1)()
             g2 = (_Gap * cap2)()

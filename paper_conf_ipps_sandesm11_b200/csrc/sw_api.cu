@@ -1315,7 +1315,11 @@ static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, c
     const long long BH = (long long)V.alpha * 32 * V.nw;
     long long L = std::max<long long>(BH, pmax > 0 ? (goal + pmax - 1) / pmax : i_end);
     for (;;) {
+        // A rectangle of at least half the rows costs a large fraction of the
+        // full one: take all rows at once instead of filling it twice (a
+        // whole-length alignment starts with L = goal / pmax ~ i_end).
         L = std::min<long long>(L, i_end);
+        if (2 * L >= i_end) L = i_end;
         long long Jc = j_end;
         if (ge > 0 && pmax > 0) {
             const long long slack = pmax * L - go - goal;
