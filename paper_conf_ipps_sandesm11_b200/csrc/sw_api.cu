@@ -891,10 +891,6 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     a.ge = J.ge;
     a.gf = J.go + J.ge;
     a.one = 1;
-    a.nge2 = (uint32_t)(-(J.ge * 0x10001));
-    a.ngf2 = (uint32_t)(-(a.gf * 0x10001));
-    a.nge16 = ((0x10000u - (uint32_t)J.ge) & 0xffffu) * 0x10001u;
-    a.ngf16 = ((0x10000u - (uint32_t)a.gf) & 0xffffu) * 0x10001u;
     for (int x = 0; x < 4; x++) {
         uint32_t w = 0;
         for (int y = 0; y < 4; y++) {

@@ -72,10 +72,6 @@ struct FillArgs {
     int nb;              // number of bands
     int go, ge, gf;      // G_open, G_ext, G_first = go + ge
     int one;             // always 1 (see imad())
-    // packed-kernel addends, precomputed so the cell update can take them
-    // straight from the constant bank (one register read per add):
-    // -G_ext and -G_first in both halves, as a 32-bit add (no borrow) and per half
-    uint32_t nge2, ngf2, nge16, ngf16;
     uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
     const uint32_t *A2;  // S0 codes, 2 bits each, 16 per word
     const uint32_t *B2;  // S1 codes (global columns)

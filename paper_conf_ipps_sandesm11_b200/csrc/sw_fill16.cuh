@@ -43,18 +43,12 @@ constexpr int BIAS16 = 32768;
 #define SWB_K_NGF16 0x66334873u
 #endif
 #ifndef SWB_ADDMODE
-#ifdef SWB_PATCH
-#define SWB_ADDMODE 1
-#else
-#define SWB_ADDMODE 0
-#endif
+#define SWB_ADDMODE 1  // plain adds; 0: IMAD with a runtime 1
 #endif
 #ifndef SWB_UNR
 #define SWB_UNR 4     // lane steps per iteration of the fast tile loop
 #endif
-#ifndef SWB_TMTREE
-#define SWB_TMTREE 0  // 1: tile maximum as a per-step tree instead of a chain through the slots
-#endif
+
 
 __device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(lo & 0xffff) | ((uint32_t)hi << 16); }
 __device__ __forceinline__ int lo16(uint32_t v) { return (int)(v & 0xffffu); }
@@ -70,24 +64,8 @@ __device__ __forceinline__ uint32_t col_sel16(uint32_t code)
     return lo | (hi << 8);
 }
 
-// Maximum of N packed u16x2 values as a 3-ary tree (depth log3 N instead of a chain).
-template <int N>
-struct MaxTree {
-    static __device__ __forceinline__ uint32_t run(const uint32_t *v)
-    {
-        if constexpr (N == 1) return v[0];
-        else if constexpr (N == 2) return __vmaxu2(v[0], v[1]);
-        else if constexpr (N == 3) return __vimax3_u16x2(v[0], v[1], v[2]);
-        else {
-            constexpr int A = (N + 2) / 3, B = (N - A + 1) / 2, C = N - A - B;
-            return __vimax3_u16x2(MaxTree<A>::run(v), MaxTree<B>::run(v + A), MaxTree<C>::run(v + A + B));
-        }
-    }
-};
-
 template <int NW, int W, int NS = 8, bool SPLIT = false, bool LOCAL = true>
 struct Fill16 {
-    static constexpr bool TMTREE = SWB_FMODE == 2 && SWB_TMTREE;
     static constexpr int ALPHA = 2 * NS, BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
     static constexpr int SRING = Smem<W, NW>::SRING;
@@ -164,9 +142,10 @@ struct Fill16 {
     //      tile maximum is then taken over t (= H - G_first) instead of H,
     //      except in replays (TRACK), which need H.
     // The u16x2 adds never wrap: every frame value stays far above G_first.
-    // x + c (both halves; never borrows, see above).  SWB_ADDMODE 0: IMAD with
-    // a runtime 1 (forces the FMA pipe, 3 register reads); 1: a plain add,
-    // ptxas picks IMAD.IADD (FMA pipe, 2 reads) or IADD3 (ALU pipe).
+    // x + c (both halves; never borrows, see above).  SWB_ADDMODE 1 (default):
+    // a plain add -- an immediate-form VIADD (FMA pipe, one register read) in
+    // the patched image, IMAD R, R, imm, R (two reads) otherwise; 0: IMAD with
+    // a runtime 1 (three reads, measured 4-10 % slower).
     static __device__ __forceinline__ uint32_t add_fma(uint32_t x, int one, int c)
     {
         if constexpr (SWB_ADDMODE == 0) return (uint32_t)imad((int)x, one, c);
@@ -225,13 +204,6 @@ struct Fill16 {
         // immediate reads one register instead of three.
         constexpr int nge2 = (int)SWB_K_NGE2, ngf2 = (int)SWB_K_NGF2;
         constexpr uint32_t nge16 = SWB_K_NGE16, ngf16 = SWB_K_NGF16;
-#elif defined(SWB_FIXGE)  // timing experiment only: gap penalties as compile-time immediates
-        constexpr int nge2 = -(SWB_FIXGE * 0x10001), ngf2 = -(SWB_FIXGF * 0x10001);
-        constexpr uint32_t nge16 = ((0x10000u - (uint32_t)SWB_FIXGE) & 0xffffu) * 0x10001u;
-        constexpr uint32_t ngf16 = ((0x10000u - (uint32_t)SWB_FIXGF) & 0xffffu) * 0x10001u;
-#elif SWB_ADDMODE == 2  // the addends straight from the kernel parameters (constant bank)
-        const int nge2 = (int)a.nge2, ngf2 = (int)a.ngf2;
-        const uint32_t nge16 = a.nge16, ngf16 = a.ngf16;
 #else
         const int nge2 = -(a.ge * 0x10001), ngf2 = -(a.gf * 0x10001);
         // per-half two's complements of -G_ext, -G_first for the u16x2 adds
@@ -313,7 +285,7 @@ struct Fill16 {
                 cell_hf<TRACK>(d1, fu, h1, t1, one, nge2, ngf2, nge16, ngf16);
                 L.e[s + 1] = e1;
                 L.t[s + 1] = t1;
-                if (TRACK || !TMTREE) tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
+                tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
                 if (CAP) {
                     if (jl == X.jcap) {
                         X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
@@ -325,14 +297,6 @@ struct Fill16 {
                     }
                 }
             }
-        }
-        if constexpr (!SPLIT && !TRACK && TMTREE) {
-            // tile maximum as a 3-ary tree over this step's t (mode 2: t is what is tracked)
-            uint32_t v[NS + 1];
-#pragma unroll
-            for (int s = 0; s < NS; s++) v[s] = L.t[s];
-            v[NS] = tmax;
-            tmax = MaxTree<NS + 1>::run(v);
         }
         L.fn = fu;
         if (GUARD) {
