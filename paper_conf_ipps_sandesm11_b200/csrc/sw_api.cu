@@ -1307,9 +1307,10 @@ static int reverse_common(sw_ctx *ctx, const unsigned char *dA, int64_t i_end, c
                           cudaStream_t us, sw_result *out)
 {
     const long long pmax = std::max(ma, mi);
-    const Variant &V = ctx_variant(ctx);
-    const long long BH = (long long)V.alpha * 32 * V.nw;
-    long long L = std::max<long long>(BH, pmax > 0 ? (goal + pmax - 1) / pmax : i_end);
+    // First rectangle: twice the fewest rows a score of `goal` needs.  The fill
+    // sweeps Jc columns band by band, so a short alignment (C2: 93 rows) costs
+    // a few hundred columns instead of a whole band height of them.
+    long long L = std::max<long long>(256, pmax > 0 ? 2 * ((goal + pmax - 1) / pmax) : i_end);
     for (;;) {
         // A rectangle of at least half the rows costs a large fraction of the
         // full one: take all rows at once instead of filling it twice (a
