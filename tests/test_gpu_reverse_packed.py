@@ -87,3 +87,20 @@ def test_reverse_packed_ties_and_edges(ctx):
     X = synth.random_pair(4, 3000, 1)[0]
     p, q, _ = both(ctx, X, 3000, X, 3000, 3000, PAPER)
     assert p == q == (3000, 0, 0)
+
+
+@pytest.mark.parametrize("scoring", [(5, -4, 10, 5), (1, -1, 0, 1), (4, -5, 0, 7)])
+def test_reverse_packed_window_edges(ctx, scoring):
+    """Scorings near the packed kernel's 16-bit window bound (DESIGN.md 4.7:
+    (32 alpha + 140)(|p|max + G_first) + 1024 < 30000) and the smallest
+    penalties, on a whole-length pair: Stage 1 and the reverse pass both
+    packed, bit-exact."""
+    A, B = synth.random_pair(31 + scoring[2], 6000, 5800, plant_len=6000, s=0.03, g=0.006)
+    got, _ = ctx.align_stage1(A, B, *scoring, k=0)
+    assert ctx.stats()["alpha"] < 0
+    (s, ie, je), _ = oracle.stage1(_s(A), _s(B), *scoring)
+    assert got.astuple() == (s, ie, je)
+    want = oracle.reverse_goal(_s(A), ie, _s(B), je, *scoring, s)
+    p, q, st = both(ctx, A, ie, B, je, s, scoring)
+    assert p == want and q == want, (scoring, p, q, want)
+    assert st["alpha"] < 0
