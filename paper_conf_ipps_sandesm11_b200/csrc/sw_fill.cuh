@@ -110,7 +110,7 @@ struct StepInfo {
 __device__ __forceinline__ unsigned long long gtimer()
 {
     unsigned long long t;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t) : : "memory");  // ordered with barriers (debug stamps)
     return t;
 }
 

@@ -535,6 +535,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         __syncthreads();
         const int b = s_band;
         if (b >= a.nb) break;
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b] = gtimer();  // debug: band start
 
         typename F::Lane L;
         const int row0 = b * BH + (warp * 32 + lane) * ALPHA;
@@ -602,10 +603,22 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             if (b > 0) {
                 if (lane == 0) {
                     const unsigned long long t0 = gtimer();
+                    unsigned long long spins = 0;
                     while (ld_acquire(S.progress + b - 1) < need) {
                         if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
                         if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                         __nanosleep(64);
+                        spins++;
+                    }
+                    if (a.dbg && S.col0 == 0 && spins) {  // debug: total wait ns, spin loops, waits
+                        a.dbg[80 * b + 5] += gtimer() - t0;
+                        a.dbg[80 * b + 6] += spins;
+                        a.dbg[80 * b + 7] += 1;
+                    }
+                    if (a.dbg && S.col0 == 0 && c == 0) {  // debug: tile 0's border wait
+                        a.dbg[80 * b + 2] = gtimer();
+                        a.dbg[80 * b + 3] = (unsigned long long)ld_acquire(S.progress + b - 1);
+                        a.dbg[80 * b + 4] = spins;
                     }
                 }
                 __syncwarp();
@@ -787,6 +800,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             if (s_abort) break;
         }
         if (threadIdx.x == (COOP ? 0 : NW * 32) && !s_abort) st_release(S.progress + b, INT_MAX);
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 15] = gtimer();  // debug: band end
         if (a.k > 0) {
             __threadfence();
             __syncthreads();

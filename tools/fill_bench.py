@@ -68,11 +68,12 @@ def main():
             import numpy as np
             t = band_times(ctx)
             np.set_printoptions(linewidth=250, precision=1, suppress=True)
-            print("  slots: 0 start | 1..8 warp first chunk | 10 io first load | 11 io first drain | 12,13 chunk2 | 14 last warp done | 15 end")
+            print("  slots: 0 start | 1 first tile | 15 end (int32 kernel: 2-4 quarter intervals; packed: 2 tile-0 border ready, 3 upstream progress, 4 spins) | 5-7 border waits")
             for i in list(range(0, min(len(t), 3))) + [len(t) // 2]:
                 print("   band", i, t[i][:16])
             lag = np.diff(t[:, 1])
-            print(f"  start lag us mean={np.nanmean(lag):.1f}; band dur us mean={np.nanmean(t[:,15]-t[:,1]):.0f}")
+            print(f"  start lag us mean={np.nanmean(lag):.1f} median={np.nanmedian(lag):.1f}; band dur us mean={np.nanmean(t[:,15]-t[:,1]):.0f}; "
+                  f"first tile of the last band at {np.nanmax(t[:,1]):.0f} us, last band end {np.nanmax(t[:,15]):.0f} us")
         print(f"{wl} v{v} k={k} result={r.astuple()} fill_ms={best['fill_ms']:.2f} total_ms={best['total_ms']:.2f} "
               f"GCUPS(fill)={cells / best['fill_ms'] / 1e6:.1f} alpha={best['alpha']} warps={best['warps']} "
               f"grid={best['grid']} replays={best['replays']}", flush=True)
