@@ -312,6 +312,7 @@ struct sw_ctx {
     S1Rows s1;                  // special rows resident from the last Stage-1 call
     int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
     int patch = 1;              // use the immediate-patched packed kernels (SWB_PATCH=0: runtime operands)
+    bool patch_warned = false;
     std::vector<PatchedSet> patched;  // loaded patched images, most recent last
     long long timeout_ns = 120ll * 1000000000ll;
 };
@@ -651,6 +652,10 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf,
         cudaKernel_t k = nullptr;
         if (cudaLibraryGetKernel(&k, P->lib, name) != cudaSuccess || !k) {
             cudaGetLastError();
+            if (!ctx->patch_warned) {  // a name/instantiation mismatch: say so once, run unpatched
+                fprintf(stderr, "[cudalign_b200] patched kernel %s not in the embedded image; using register operands\n", name);
+                ctx->patch_warned = true;
+            }
             return nullptr;
         }
         if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize,
