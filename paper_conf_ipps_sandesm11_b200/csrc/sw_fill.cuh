@@ -709,8 +709,9 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                     const uint32_t selr_s = pin(selr_base);
                     if (c == 0 && has_left) load_left();
                     int thr;
-                    if (LOCAL) thr = max(max(bs, ld_relaxed(a.gbest)), 1);
-                    else thr = a.goal;
+                    // loaded here, used after the tile (the L2 round trip overlaps it)
+                    const int gbest = LOCAL ? ld_relaxed(a.gbest) : 0;
+                    const int bs0 = bs;
                     F::save(L, sv, lane);
                     int tmax;
                     const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
@@ -729,6 +730,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                     } else {
                         tmax = F::template tile_fast<false>(a, X, L, c, lane, rin, rout, selr_s, nullptr);
                     }
+                    thr = LOCAL ? max(max(bs0, gbest), 1) : a.goal;
                     if (__any_sync(0xffffffffu, tmax >= thr - a.gf)) {  // tmax is over t = H - G_first
                         // exact replay of this tile from the saved state (rare)
                         F::restore(L, sv, lane);

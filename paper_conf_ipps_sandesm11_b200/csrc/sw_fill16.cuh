@@ -742,7 +742,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     }
                     if (c > 0) F::rebase(a, L);
                     F::convert_ring(a, L, rings + warp * F::RS, crings + warp * W, c, lane);
-                    const int thr = LOCAL ? max(max(bs, ld_relaxed(a.gbest)), 1) : a.goal;
+                    // the running best of all CTAs: loaded here, used after the tile
+                    // (so the L2 round trip overlaps the tile instead of stalling it)
+                    const int gbest = LOCAL ? ld_relaxed(a.gbest) : 0;
+                    const int bs0 = bs;
                     F::save(L, sv, lane);
                     uint32_t tm;
                     const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
@@ -763,6 +766,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                         tm = F::template tile<false, false, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
                     }
                     const int tmax = F::toabs(L, max(lo16(tm), hi16(tm))) + F::tmax_off(a);
+                    const int thr = LOCAL ? max(max(bs0, gbest), 1) : a.goal;
                     if (__any_sync(0xffffffffu, tmax >= thr)) {
                         F::restore(L, sv, lane);
                         const int obs = bs, obi = bi, obj = bj;
