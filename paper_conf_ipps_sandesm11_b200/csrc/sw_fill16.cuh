@@ -3,20 +3,25 @@
 // Same band pipeline, I/O warp, row border, special rows, stripes and exact
 // best-cell replay as sw_fill.cuh (read that first); what changes is the lane:
 //
-//  * A lane owns 16 rows as 8 packed slots: slot s holds row s in its low
-//    half at column j and row s+8 in its high half at column j-1, so ONE
-//    instruction updates two cells that do not depend on each other.  Slot 0's
-//    high half takes row 7's values of the previous step (a PRMT), so the
-//    vertical chain is 8 slots long instead of 16.
+//  * A lane owns 2 NS rows (NS = 8 or 16) as NS packed slots: slot s holds
+//    row s in its low half at column j and row s+NS in its high half at
+//    column j-1, so ONE instruction updates two cells that do not depend on
+//    each other.  Slot 0's high half takes row NS-1's values of the previous
+//    step (a PRMT), so the vertical chain is NS slots long instead of 2 NS.
 //  * Values are biased unsigned 16-bit numbers in a warp-uniform frame
 //    q = x - B + 32768 (x the int32 value), re-based at every tile.  Within a
 //    warp all live values lie within ~650 (p_max + G_first) of each other
 //    (|H(i,j) - H(i-1,j)| <= p_max + G_first), far inside
 //    16 bits for the supported scorings, so the frame never wraps.
-//  * Adds that cannot borrow across halves use IMAD on the FMA pipe
-//    (q - G_ext, q - G_first); the signed substitution score is added with the
-//    per-half VIADDMNMX.U16x2; maxima use VIMNMX(3).U16x2.  The local 0 floor
-//    is the frame's image of 0.
+//  * Adds that cannot borrow across halves are plain 32-bit adds on the FMA
+//    pipe (q - G_ext, q - G_first); the signed substitution score is added
+//    with the per-half VIADDMNMX.U16x2; t and the next row's F are one
+//    VIADDMNMX.U16x2 each from (F, D - G_first) (cell_hf, SWB_FMODE 2); maxima
+//    use VIMNMX3.U16x2.  The local 0 floor is the frame's image of 0; the
+//    global (reverse-pass) instantiation has no floor.
+//  * The gap penalties are compile-time magic immediates in the patchable
+//    build (SWB_PATCH, sw_fill16_patch.cu) that the library rewrites per
+//    scoring: an add with an immediate reads one register instead of three.
 //  * Everything that leaves the lane (warp ring, special rows, the right
 //    border of a stripe, replay tracking) is converted back to int32.
 //
