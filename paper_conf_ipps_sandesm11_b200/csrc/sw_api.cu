@@ -162,6 +162,12 @@ static Variant make_variant()
         } else {
             v.packed_fn = (const void *)&sw_fill16_kernel<NW, W>;
             packed_name<NW, W, false, 8>(v);
+            if constexpr (NW == 8) {
+                // Stage-2 partitions (global mode with matching) on the packed kernel
+                v.packed_global_fn = (const void *)&sw_fill16_kernel<NW, W, false, 8, false, false>;
+                snprintf(v.packed_global_name, sizeof(v.packed_global_name),
+                         "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi8ELb0ELb0EEEvNS_8FillArgsE", NW, W);
+            }
         }
         v.smem16 = Fill16<NW, W>::smem_bytes();
     }
@@ -679,6 +685,17 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         return ctx->packed && J.local && V.packed_fn && (J.k == 0 || J.k % V.alpha == 0) &&
                span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
     };
+    if (!J.local && J.match && !J.anchor_gap && ctx->variant_override < 0) {
+        // Stage-2 partitions: the packed kernel in global mode with the band-end
+        // matching, alpha 16 x 8 warps (4096-row bands, the int32 default's
+        // geometry: these one-wave fills stop after the band with the first event).
+        // Gap anchors (S20) put -inf in column 0, outside the 16-bit frame: int32.
+        const Variant &V = variant_for(1);
+        const long long span = 32ll * V.alpha + 140;
+        *use16 = ctx->packed && V.packed_global_fn && J.k == 0 && !J.rank_mode && J.nv == 1 &&
+                 span * (pmax_abs + J.go + J.ge) + 1024 < 30000 && !(getenv("SWB_S2PACKED") && atoi(getenv("SWB_S2PACKED")) == 0);
+        if (*use16) return V;
+    }
     if (!J.local) {
         // reverse pass (a8): the packed kernel in global mode when it qualifies
         // (alpha 32 x 8 warps geometry; one stripe, no Stage-2 matching or gap anchor)

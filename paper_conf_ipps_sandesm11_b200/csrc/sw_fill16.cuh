@@ -760,7 +760,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                         if (c == cap_t1) {
                             __threadfence_system();
                             __syncwarp();
-                            if (lane == 0) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
+                            if (lane == 0 && S.rready != nullptr) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
                         }
                     } else if (c == 0) {
                         tm = warp_sp ? F::template tile<true, false, true, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr)
@@ -810,6 +810,32 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         }
         if (threadIdx.x == (COOP ? 0 : NW * 32) && !s_abort) st_release(S.progress + b, INT_MAX);
         if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 15] = gtimer();  // debug: band end
+        if constexpr (!LOCAL) {
+            if (a.match && !s_abort) {
+                // Stage-2 goal-based matching, as in the
+                // int32 kernel: the capture tiles left (t, E) of the special row's DP
+                // column for every row of the band in S.rb (int32, absolute); row j'
+                // is original column j = j_c - j', t + G_first the reverse H there,
+                // E the reverse F.  Once per band, coalesced.
+                __syncthreads();
+                unsigned long long key = ~0ull;
+                const int hi = min((b + 1) * BH, a.m);
+                for (int row = b * BH + 1 + (int)threadIdx.x; row <= hi; row += (int)blockDim.x) {
+                    const int2 v = __ldcg(S.rb + row);
+                    const int j = a.mjc - row;
+                    const long long hs = (a.mH != nullptr && j > 0) ? (long long)__ldg(a.mH + j - 1) : 0ll;
+                    const long long fs = (a.mH != nullptr && j > 0) ? (long long)__ldg(a.mF + j - 1) : (long long)NEG;
+                    int kind = -1;
+                    if (hs + v.x + a.gf == a.goal) kind = 0;                                          // H junction
+                    else if (fs > NEG / 2 && v.y > NEG / 2 && fs + v.y + a.go == a.goal) kind = 1;  // gap junction (S18)
+                    if (kind >= 0) key = min(key, ((unsigned long long)(unsigned)row << 32) | (unsigned)(S.w + kind));
+                }
+                if (key != ~0ull) {
+                    atomicMin(a.hit_key, key);
+                    atomicMin(a.hit_band, b);
+                }
+            }
+        }
         if (a.k > 0) {
             __threadfence();
             __syncthreads();

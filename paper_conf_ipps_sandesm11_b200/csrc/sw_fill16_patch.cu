@@ -26,4 +26,6 @@ template __global__ void sw_fill16_kernel<8, 64, false, 16, false>(const __grid_
 template __global__ void sw_fill16_kernel<16, 64, true, 16, false>(const __grid_constant__ FillArgs);
 // the reverse pass (global mode), variant 10's geometry
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false, false>(const __grid_constant__ FillArgs);
+// Stage-2 partitions (global mode with matching), variant 1's geometry
+template __global__ void sw_fill16_kernel<8, 64, false, 8, false, false>(const __grid_constant__ FillArgs);
 }  // namespace swb
