@@ -135,13 +135,14 @@ static Variant make_variant()
     v.packed_name[0] = 0;
     v.packed_global_fn = nullptr;
     v.packed_global_name[0] = 0;
-    if constexpr (ALPHA == 32) {
-        // packed kernel only (16 slots per lane); int32 work falls back to the default geometry
-        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, 16, SPLIT>;
+    if constexpr (ALPHA == 32 || ALPHA == 30) {
+        // packed kernel only (16 or 15 slots per lane); int32 work falls back to the default geometry
+        constexpr int NS = ALPHA / 2;
+        v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, NS, SPLIT>;
         v.io_warps = COOP ? 0 : 1;
-        v.smem16 = Fill16<NW, W, 16, SPLIT>::smem_bytes();
-        if constexpr (!SPLIT) packed_name<NW, W, COOP, 16>(v);
-        if constexpr (NW == 8 && !COOP && !SPLIT) {
+        v.smem16 = Fill16<NW, W, NS, SPLIT>::smem_bytes();
+        if constexpr (!SPLIT) packed_name<NW, W, COOP, NS>(v);
+        if constexpr (ALPHA == 32 && NW == 8 && !COOP && !SPLIT) {
             // the reverse pass (a8) on the packed kernel
             v.packed_global_fn = (const void *)&sw_fill16_kernel<NW, W, false, 16, false, false>;
             snprintf(v.packed_global_name, sizeof(v.packed_global_name),
@@ -175,7 +176,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 13;
+static constexpr int NVARIANTS = 14;
 static constexpr int NINT32_VARIANTS = 8;  // variants 0..7 have int32 kernels; 8.. are packed-only (alpha 32)
 
 static const Variant &variant_for(int idx)
@@ -194,6 +195,7 @@ static const Variant &variant_for(int idx)
         make_variant<32, 8, 64>(),
         make_variant<32, 16, 64, true>(),
         make_variant<32, 4, 64, false, true>(),  // split F chain (latency-bound one-wave fills)
+        make_variant<30, 4, 64>(),  // 3840-row bands: one-wave matrices of up to 148 bands (C2: 142)
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -717,6 +719,7 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         {DEFAULT_VARIANT, false, 4.24e6, 4.24e6},  // int32, 8 warps + I/O warp
         {1, true, 8.08e6, 7.74e6},                 // packed alpha 16, 8 warps + I/O warp
         {8, true, 4.25e6, 7.86e6},                 // packed alpha 32, 4 warps + I/O warp (2 CTAs/SM)
+        {13, true, 4.45e6, 8.17e6},                // packed alpha 30, 4 warps + I/O warp (2 CTAs/SM)
         {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
         {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
         {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
@@ -1237,9 +1240,12 @@ extern "C" int sw_align_stage1_dev(sw_ctx *ctx, const char *dseqA, int64_t m, co
 // last band of the tallest band height, flags (band, warp) the finest split.
 static size_t recv_rows(int64_t max_rows)
 {
-    int64_t bh_max = 0;
-    for (int i = 0; i < NVARIANTS; i++) bh_max = std::max<int64_t>(bh_max, (int64_t)variant_for(i).alpha * 32 * variant_for(i).nw);
-    return (size_t)(((max_rows + bh_max - 1) / bh_max) * bh_max + 2);
+    int64_t rows = 0;  // the largest padded row count over the band heights (not all powers of two)
+    for (int i = 0; i < NVARIANTS; i++) {
+        const int64_t bh = (int64_t)variant_for(i).alpha * 32 * variant_for(i).nw;
+        rows = std::max<int64_t>(rows, ((max_rows + bh - 1) / bh) * bh);
+    }
+    return (size_t)(rows + 2);
 }
 static size_t recv_flags(int64_t max_rows)
 {

@@ -3,7 +3,7 @@
 // Same band pipeline, I/O warp, row border, special rows, stripes and exact
 // best-cell replay as sw_fill.cuh (read that first); what changes is the lane:
 //
-//  * A lane owns 2 NS rows (NS = 8 or 16) as NS packed slots: slot s holds
+//  * A lane owns 2 NS rows (NS = 8, 15 or 16) as NS packed slots: slot s holds
 //    row s in its low half at column j and row s+NS in its high half at
 //    column j-1, so ONE instruction updates two cells that do not depend on
 //    each other.  Slot 0's high half takes row NS-1's values of the previous
@@ -278,9 +278,18 @@ struct Fill16 {
                 const uint32_t d0 = __viaddmax_u16x2(td, p0, e0);
                 td = L.t[s];
                 uint32_t h0, t0;
+                if (s == NS - 1) f15 = fu;  // odd NS: the last slot is unpaired
                 cell_hf<TRACK>(d0, fu, h0, t0, one, nge2, ngf2, nge16, ngf16);
                 L.e[s] = e0;
                 L.t[s] = t0;
+                if (s + 1 == NS) {
+                    tmax = __vmaxu2(tmax, h0);
+                    if (CAP) {
+                        if (jl == X.jcap) X.rbrow[s] = make_int2(toabs(L, lo16(t0)), toabs(L, lo16(e0)));
+                        if (jl - 1 == X.jcap) X.rbrow[s + NS] = make_int2(toabs(L, hi16(t0)), toabs(L, hi16(e0)));
+                    }
+                    break;
+                }
                 if (s == NS - 2) f15 = fu;
                 const uint32_t e1 = __vimax3_u16x2(add_fma(L.e[s + 1], one, nge2), L.t[s + 1], L.FL);
                 const uint32_t p1 = (uint32_t)prmt(L.P[s + 1], L.Q[s + 1], sel);
@@ -583,15 +592,26 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             L.FL = (uint32_t)fl * 0x10001u;
         };
         if (warp < NW) {
-            // row r's code: bits 2 (r & 15) of word r >> 4 (row0 is a multiple of 16)
-            uint32_t wv[ALPHA / 16];
+            if constexpr (ALPHA % 16 == 0) {
+                // row r's code: bits 2 (r & 15) of word r >> 4 (row0 is a multiple of 16)
+                uint32_t wv[ALPHA / 16];
 #pragma unroll
-            for (int q = 0; q < ALPHA / 16; q++) wv[q] = row0 + 16 * q < a.m ? a.A2[(row0 >> 4) + q] : 0u;
+                for (int q = 0; q < ALPHA / 16; q++) wv[q] = row0 + 16 * q < a.m ? a.A2[(row0 >> 4) + q] : 0u;
 #pragma unroll
-            for (int s = 0; s < NS; s++) {
-                const int rp = s, rq = s + NS;
-                L.P[s] = (row0 + rp < a.m) ? a.prof[(wv[rp >> 4] >> (2 * (rp & 15))) & 3u] : PADPROF;
-                L.Q[s] = (row0 + rq < a.m) ? a.prof[(wv[rq >> 4] >> (2 * (rq & 15))) & 3u] : PADPROF;
+                for (int s = 0; s < NS; s++) {
+                    const int rp = s, rq = s + NS;
+                    L.P[s] = (row0 + rp < a.m) ? a.prof[(wv[rp >> 4] >> (2 * (rp & 15))) & 3u] : PADPROF;
+                    L.Q[s] = (row0 + rq < a.m) ? a.prof[(wv[rq >> 4] >> (2 * (rq & 15))) & 3u] : PADPROF;
+                }
+            } else {
+                // alpha 30: strips straddle the 16-code words; one word per row
+                auto code_row = [&](int r) -> uint32_t { return (a.A2[r >> 4] >> (2 * (r & 15))) & 3u; };
+#pragma unroll
+                for (int s = 0; s < NS; s++) {
+                    const int rp = row0 + s, rq = row0 + s + NS;
+                    L.P[s] = rp < a.m ? a.prof[code_row(rp)] : PADPROF;
+                    L.Q[s] = rq < a.m ? a.prof[code_row(rq)] : PADPROF;
+                }
             }
             init_state(false);
             if (a.k > 0) {

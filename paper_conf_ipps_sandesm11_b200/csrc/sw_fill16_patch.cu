@@ -22,6 +22,7 @@ template __global__ void sw_fill16_kernel<15, 64, false, 8, false>(const __grid_
 template __global__ void sw_fill16_kernel<16, 64, true, 8, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<4, 64, false, 16, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<4, 64, true, 16, false>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<4, 64, false, 15, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<16, 64, true, 16, false>(const __grid_constant__ FillArgs);
 // the reverse pass (global mode), variant 10's geometry

@@ -106,9 +106,10 @@ CONFIGS = {
     "C1": Config("C1", 50_000, 50_000, 1, 1024, "plant",
                  dict(L=2000, a0=24_000, b0=10_000, s=0.05, g=0.002, mu=3.0, ins_frac=0.5),
                  note="BASELINE configs[0]: 50 KBP x 50 KBP, one planted 2 KBP region"),
-    "C2": Config("C2", 542_868, 536_165, 2, 4096, "gapless",
+    "C2": Config("C2", 542_868, 536_165, 2, 3840, "gapless",
                  dict(L=92, n_sub=11, a0=308_466, b0=455_042),
-                 note="BASELINE configs[1]: Table II 543K x 536K sizes; Table III row 2 shape (P:392)"),
+                 note="BASELINE configs[1]: Table II 543K x 536K sizes; Table III row 2 shape (P:392); "
+                      "k = 3840, a multiple of every packed strip height (16, 30, 32)"),
     "C3": Config("C3", 5_000_000, 5_000_000, 3, 65_536, "whole",
                  dict(s=5e-5, g=3e-5, mu=10.0, ins_frac=0.5, b0=0),
                  gpus=(1, 2), note="BASELINE configs[2]: whole-length homology (B. anthracis shape, P:395)"),

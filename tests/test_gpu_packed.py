@@ -101,6 +101,27 @@ def test_packed_alpha32(ctx, variant):
     check(ctx, A, B, PAPER, 32, variant, stripes=3)
 
 
+@pytest.mark.parametrize("m,n", [(1, 1), (29, 40), (31, 300), (3839, 700), (3841, 1000), (9000, 2049)])
+def test_packed_alpha30_shapes(ctx, m, n):
+    """Variant 13: 15 slots per lane (odd slot count, unpaired last slot) and
+    3840-row bands whose strips straddle the 16-code words of A; special rows
+    at strip bottoms (k % 30 == 0), bands, ragged tails."""
+    A, B = synth.random_pair(130 + m + n, m, n, plant_len=min(m, n) // 2, s=0.05, g=0.01)
+    check(ctx, A, B, PAPER, 30, 13)
+    check(ctx, A, B, PAPER, 0, 13)
+
+
+def test_packed_alpha30(ctx):
+    A, B = synth.random_pair(131, 8000, 2100, plant_len=1500, s=0.04, g=0.01)
+    for scoring in (PAPER, (2, -1, 4, 1), (1, -1, 0, 2), (5, -4, 10, 1), (3, -2, 0, 1)):
+        check(ctx, A, B, scoring, 3840, 13)
+    check(ctx, A, B, PAPER, 90, 13)
+    check(ctx, A, B, PAPER, 32, 13, expect_packed=False)  # k not a multiple of 30: int32 kernel
+    check(ctx, A, B, PAPER, 60, 13, stripes=3)
+    X = synth.random_pair(5, 500, 1)[0]
+    check(ctx, np.concatenate([X, X, X, X]), X, PAPER, 30, 13)
+
+
 def test_packed_config_c1(ctx):
     cfg = synth.CONFIGS["C1"]
     A, B = synth.make_pair(cfg)

@@ -62,7 +62,7 @@ def ctx():
 
 
 def test_c2_full_band_induction(ctx):
-    """BASELINE configs[1] (543K x 536K, k = 4096): every special row and the
+    """BASELINE configs[1] (543K x 536K, k = 3840): every special row and the
     best cell, bit-exact, plus the reverse-pass start cell."""
     cfg = synth.CONFIGS["C2"]
     A, B = synth.make_pair(cfg)
