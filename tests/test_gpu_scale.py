@@ -72,6 +72,9 @@ def test_c2_full_band_induction(ctx):
         rows[row] = (H.copy(), F.copy())
 
     got, _ = ctx.align_stage1(A, B, *PAPER, k=cfg.k, sink=sink)
+    # the kernel bench.py times: the alpha-30 packed geometry (142 bands of 3840 rows)
+    s1 = ctx.stats()
+    assert (s1["alpha"], s1["warps"], s1["grid"], s1["patched"]) == (-30, 4, 142, 1), s1
     assert sorted(rows) == list(range(cfg.k, cfg.m + 1, cfg.k))
     bounds = list(range(0, cfg.m, cfg.k)) + [cfg.m]
     jobs = [(q, bounds[q], bounds[q + 1]) for q in range(len(bounds) - 1)]
