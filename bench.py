@@ -161,7 +161,7 @@ def reference_arm(args, cfg, k, rank, world):
         "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GCUPS",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
-        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
         "config": {"workload": cfg.name, "m": cfg.m, "n": cfg.n, "k": k, "scoring": list(SCORING)},
         "cpu_baseline": {"value": round(value, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": samples},
         "e2e": {"value": round(value, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -391,7 +391,7 @@ def main():
     line = {
         "metric": METRIC, "value": round(value, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
-        "scaling": "strong" if world > 1 else "weak",
+        "scaling": "strong",
         "vs_baseline": (round(value / PAPER_GCUPS[cfg.name], 2) if cfg.name in PAPER_GCUPS else None),
         "dtype": "int16x2" if s1["alpha"] < 0 else "int32", "data": "synthetic",
         "config": {"workload": cfg.name, "m": m, "n": n, "k": k, "scoring": list(SCORING),
