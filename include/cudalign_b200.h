@@ -209,8 +209,10 @@ int64_t sw_band_height(const sw_ctx *ctx);
 /* Kernel selection (testing / tuning).  variant = -1: automatic choice per
  * call; 0..7: a fixed geometry (alpha, warps, tile width) of
  * the int32 kernel (DESIGN.md 4.1 lists them), or of the packed 16x2 kernel when packed = 1 and the call
- * qualifies (local mode, k % 16 == 0, small value window).  packed = 0 never
- * uses the packed kernel.  Results are identical for every choice. */
+ * qualifies (local mode, k % alpha == 0, small value window); 8..13: packed-only
+ * geometries (alpha 32, or alpha 30 for 13) that fall back to the default int32
+ * geometry when the call does not qualify.  packed = 0 never uses the packed
+ * kernel.  Results are identical for every choice.  SW_EINVAL outside -1..13. */
 int sw_set_kernel(sw_ctx *ctx, int variant, int packed);
 
 /* Immediate patching of the packed kernel (testing / tuning; default on).
