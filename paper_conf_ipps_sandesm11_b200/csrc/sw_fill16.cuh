@@ -50,8 +50,11 @@ constexpr int BIAS16 = 32768;
 #ifndef SWB_ADDMODE
 #define SWB_ADDMODE 1  // plain adds; 0: IMAD with a runtime 1
 #endif
+// Lane steps per iteration of the fast tile loop: 8 for the local-mode
+// geometries with 15 or 16 slots except 4 warps x 16 slots, 4 otherwise
+// (measured); SWB_UNR overrides it for every geometry.
 #ifndef SWB_UNR
-#define SWB_UNR 4     // lane steps per iteration of the fast tile loop
+#define SWB_UNR 0
 #endif
 
 
@@ -76,6 +79,7 @@ struct Fill16 {
     static constexpr int SRING = Smem<W, NW>::SRING;
     static constexpr int SKEW = 63;     // lane 31's output column lags lane 0's by 2*31 + 1
     static constexpr int STEPS = W;     // one column per lane step
+    static constexpr int UNR = SWB_UNR > 0 ? SWB_UNR : (LOCAL && NS >= 15 && !(NW == 4 && NS == 16)) ? 8 : 4;
     static constexpr int NSAVE = 2 * NS + 3;
     static constexpr int HALF = SRING / 2 + 32;  // selector ring: one parity half + a 32-entry mirror
     // Warp-to-warp rings of (t, F): column col lives at ridx(col) in [1, RING]
@@ -434,10 +438,10 @@ struct Fill16 {
                                                     row1, bs, bi, bj, sp_ptr);
         } else {
 #pragma unroll 1
-            for (int kq = 0; kq < STEPS; kq += SWB_UNR) {
+            for (int kq = 0; kq < STEPS; kq += UNR) {
                 const uint32_t sq = sel0 + 2u * kq, cq = cring + 4u * kq, oq = ro0 + 8u * kq;
 #pragma unroll
-                for (int u = 0; u < SWB_UNR; u++)
+                for (int u = 0; u < UNR; u++)
                     tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + u, lane, cq + 4u * u, oq + 8u * u,
                                                           sq + 4u * ((u >> 1) + (u & 1) * HALF), pt_sel, one, tmax,
                                                           row1, bs, bi, bj, sp_ptr);
