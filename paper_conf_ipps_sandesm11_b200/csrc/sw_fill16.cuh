@@ -51,8 +51,9 @@ constexpr int BIAS16 = 32768;
 #define SWB_ADDMODE 1  // plain adds; 0: IMAD with a runtime 1
 #endif
 // Lane steps per iteration of the fast tile loop: 8 for the local-mode
-// geometries with 15 or 16 slots except 4 warps x 16 slots, 4 otherwise
-// (measured); SWB_UNR overrides it for every geometry.
+// geometries with 8 or more warps or 15 slots, 4 otherwise (4 warps x 16
+// slots: 9.2 -> 14.0 ms on C1 at 8; measured); SWB_UNR
+// overrides it for every geometry.
 #ifndef SWB_UNR
 #define SWB_UNR 0
 #endif
@@ -79,7 +80,7 @@ struct Fill16 {
     static constexpr int SRING = Smem<W, NW>::SRING;
     static constexpr int SKEW = 63;     // lane 31's output column lags lane 0's by 2*31 + 1
     static constexpr int STEPS = W;     // one column per lane step
-    static constexpr int UNR = SWB_UNR > 0 ? SWB_UNR : (LOCAL && NS >= 15 && !(NW == 4 && NS == 16)) ? 8 : 4;
+    static constexpr int UNR = SWB_UNR > 0 ? SWB_UNR : (LOCAL && (NW >= 8 || NS == 15)) ? 8 : 4;
     static constexpr int NSAVE = 2 * NS + 3;
     static constexpr int HALF = SRING / 2 + 32;  // selector ring: one parity half + a 32-entry mirror
     // Warp-to-warp rings of (t, F): column col lives at ridx(col) in [1, RING]
