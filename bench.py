@@ -50,9 +50,12 @@ ROOF_CELLS_PER_CLK_SM = {"int32": 16.0, "int16x2": round(4 * 64 / 11, 2)}
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--steps", type=int, default=3)
     p.add_argument("--warmup", type=int, default=3)
-    p.add_argument("--workload", default=os.environ.get("SWB_WORKLOAD", "C2"))
+    # C4 (10M x 10M): the largest BASELINE config that fits one GPU's bench
+    # window (the metric's C5 pair takes ~5 min per step; tools/c5_align.py)
+    p.add_argument("--workload", default=os.environ.get("SWB_WORKLOAD", "C4"))
+    p.add_argument("--e2e-steps", type=int, default=3, help="host-API steps timed for e2e (<= --steps)")
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--k", type=int, default=None, help="special_row_interval override")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -117,28 +120,60 @@ class ClockSampler:
 
 # ---------------------------------------------------------------- oracle (CPU) timing
 
-def oracle_sample(A, B, target_s=12.0):
-    """Time the oracle's band recompute (the same loop as its Stage 1) on a
-    bounded sample of rows of the workload: single-threaded, as it stands."""
+def host_cpu():
+    """(logical CPUs usable by this process, CPU model string)."""
+    try:
+        ncpu = len(os.sched_getaffinity(0))
+    except Exception:
+        ncpu = os.cpu_count() or 1
+    model = "unknown"
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return ncpu, model
+
+
+def oracle_sample(A, B, target_s=12.0, threads=None):
+    """Time the oracle's band recompute (oracle.band: the same row loop as its
+    Stage 1 and as the band-induction checker) on a bounded sample of the
+    workload, as it stands: `threads` concurrent bands of distinct rows (the
+    band-induction driver's parallelism; ctypes releases the GIL), each a full
+    sweep of all n columns.  Returns (GCUPS over all threads, sample text, s, threads)."""
+    from multiprocessing.pool import ThreadPool
+
     import numpy as np
 
     import oracle
 
-    n = len(B)
+    n, m = len(B), len(A)
     ma, mi, go, ge = SCORING
+    ncpu, model = host_cpu()
+    # one band's working set is 4 int64 rows of n + 1 entries: cap the threads at ~16 GB
+    T = threads or max(1, min(ncpu, 64, int(16e9 // (32 * (n + 1)))))
     Htop = np.zeros(n + 1, np.int64)
     Ftop = np.full(n + 1, oracle.NEG, np.int64)
-    r = max(1, int(2e8 // max(n, 1)))
+    r = max(1, min(m, int(2e8 // max(n, 1))))
     t0 = time.perf_counter()
-    oracle.band(A, B, ma, mi, go, ge, 0, min(r, len(A)), Htop, Ftop)
-    dt = time.perf_counter() - t0
-    rate = (min(r, len(A)) * n) / max(dt, 1e-9)
-    rows = int(min(len(A), max(1, target_s * rate / n)))
+    oracle.band(A, B, ma, mi, go, ge, 0, r, Htop, Ftop)
+    rate1 = r * n / max(time.perf_counter() - t0, 1e-9)
+    rows = int(max(1, min(m // T, target_s * rate1 / n)))
+
+    def job(t):
+        r0 = t * rows
+        oracle.band(A, B, ma, mi, go, ge, r0, r0 + rows, Htop, Ftop)
+
     t0 = time.perf_counter()
-    oracle.band(A, B, ma, mi, go, ge, 0, rows, Htop, Ftop)
+    with ThreadPool(T) as pool:
+        pool.map(job, range(T), chunksize=1)
     dt = time.perf_counter() - t0
-    cells = rows * n
-    return cells / dt / 1e9, f"oracle.band rows 1..{rows} x all {n} columns of the workload ({cells:.3g} cells, {dt:.1f} s, 1 thread)", dt
+    cells = float(T) * rows * n
+    sample = (f"oracle.band on {T} threads (of {ncpu} logical CPUs, {model}), each rows r0+1..r0+{rows} x all "
+              f"{n} columns of the workload ({cells:.3g} cells, {dt:.1f} s)")
+    return cells / dt / 1e9, sample, dt, T, rate1 / 1e9
 
 
 def reference_arm(args, cfg, k, rank, world):
@@ -149,21 +184,23 @@ def reference_arm(args, cfg, k, rank, world):
 
     A, B = synth.make_pair(cfg)
     oracle.build()
-    vals, samples, times = [], "", []
+    vals, samples, times, T = [], "", [], 1
     for _ in range(args.warmup):
-        oracle_sample(A, B, target_s=2.0)
+        oracle_sample(A, B, target_s=1.0)
     for _ in range(args.steps):
-        v, samples, dt = oracle_sample(A, B, target_s=10.0)
+        v, samples, dt, T, _ = oracle_sample(A, B, target_s=8.0)
         vals.append(v)
         times.append(dt)
     value = statistics.median(vals)
     line = {
-        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GCUPS",
+        "impl": "reference", "metric": METRIC, "workload": f"{cfg.name} ({cfg.m} x {cfg.n}, k={k})",
+        "value": round(value, 4), "unit": "GCUPS",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
         "config": {"workload": cfg.name, "m": cfg.m, "n": cfg.n, "k": k, "scoring": list(SCORING)},
-        "cpu_baseline": {"value": round(value, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": samples},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GCUPS", "cores": T, "kind": "oracle", "sample": samples,
+                         "nproc": host_cpu()[0], "cpu_model": host_cpu()[1]},
         "e2e": {"value": round(value, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -320,7 +357,7 @@ def main():
         e2e_step()
         torch.cuda.synchronize()
         ts = []
-        for s in range(args.steps):
+        for s in range(max(1, min(args.steps, args.e2e_steps))):
             flush.fill_(s & 0xFF)
             torch.cuda.synchronize()
             if world > 1:
@@ -334,13 +371,14 @@ def main():
         h2d = m + n + ((best[1] + best[2]) if rank == 0 else 0)
         d2h = sp_bytes // args.steps + 3 * 16
         e2e = {"value": round(cells / e2e_s / 1e9, 3), "unit": "GCUPS", "h2d_bytes_per_step": int(h2d),
-               "d2h_bytes_per_step": int(d2h), "ms_per_step": round(1e3 * e2e_s, 3)}
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": round(1e3 * e2e_s, 3), "steps": len(ts)}
 
     # ---- the full alignment (Stages 1-5, sw_align) once, outside the timed region:
     # the N2/N3 rows of SURVEY 8(f) measured on the same workload
     full = None
     if not args.no_align and world == 1:
-        ctx.align(A, B, *SCORING, k=k)  # warm-up: first use of the Stage 2-5 kernels and their buffers
+        if m * n < 1e12:
+            ctx.align(A, B, *SCORING, k=k)  # warm-up: first use of the Stage 2-5 kernels and their buffers
         t0 = time.perf_counter()
         ra = ctx.align(A, B, *SCORING, k=k)
         full = {"ms": round(1e3 * (time.perf_counter() - t0), 2),
@@ -385,11 +423,14 @@ def main():
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
-        v, sample, _ = oracle_sample(A, B, target_s=12.0)
-        cpu = {"value": round(v, 4), "unit": "GCUPS", "cores": 1, "kind": "oracle", "sample": sample}
+        v, sample, _, T, v1 = oracle_sample(A, B, target_s=10.0)
+        ncpu, model = host_cpu()
+        cpu = {"value": round(v, 4), "unit": "GCUPS", "cores": T, "kind": "oracle", "sample": sample,
+               "nproc": ncpu, "cpu_model": model, "single_thread_value": round(v1, 4)}
 
     line = {
-        "metric": METRIC, "value": round(value, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
+        "metric": METRIC, "workload": f"{cfg.name} ({m} x {n}, k={k})",
+        "value": round(value, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
         "scaling": "strong",
         "vs_baseline": (round(value / PAPER_GCUPS[cfg.name], 2) if cfg.name in PAPER_GCUPS else None),

@@ -223,6 +223,14 @@ int sw_set_kernel(sw_ctx *ctx, int variant, int packed);
  * Returns SW_EINVAL for a NULL ctx or on outside {0, 1}. */
 int sw_set_patch(sw_ctx *ctx, int on);
 
+/* Persistent-grid cap (testing / tuning; default 0).  ctas > 0: every fill
+ * launch of the following calls runs at most `ctas` CTAs (at least one per
+ * stripe) instead of the resident capacity, so bands outnumber CTAs and each
+ * CTA takes several bands from the ticket (the band pipeline's multi-wave
+ * path, P:134's grid of blocks over an arbitrary number of rows).  Results are
+ * identical for every value.  SW_EINVAL for a NULL ctx or ctas < 0. */
+int sw_set_grid(sw_ctx *ctx, int ctas);
+
 /* ---- Column-stripe pipeline ----
  * The matrix is split into column stripes; stripe g sweeps every band of its
  * columns and hands the band's right-edge (t = H - G_first, E) column to stripe

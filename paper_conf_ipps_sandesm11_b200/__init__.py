@@ -45,6 +45,7 @@ EXPORTED = [
     "sw_set_kernel",
     "sw_set_patch",
     "sw_set_virtual_stripes",
+    "sw_set_grid",
     "sw_stripe_export",
     "sw_stripe_connect",
     "sw_align_stage1_stripe",
@@ -153,6 +154,8 @@ def load_library(path: str = LIB_PATH):
     lib.sw_set_patch.restype = ctypes.c_int
     lib.sw_set_virtual_stripes.argtypes = [vp, ctypes.c_int]
     lib.sw_set_virtual_stripes.restype = ctypes.c_int
+    lib.sw_set_grid.argtypes = [vp, ctypes.c_int]
+    lib.sw_set_grid.restype = ctypes.c_int
     lib.sw_stripe_export.argtypes = [vp, i64, vp]
     lib.sw_stripe_export.restype = ctypes.c_int
     lib.sw_stripe_connect.argtypes = [vp, vp, i64]
@@ -355,6 +358,11 @@ class Context:
         """Split the next Stage-1 calls into `nstripes` column stripes on this GPU
         (the multi-GPU border protocol, run inside one launch)."""
         self._check(self._lib.sw_set_virtual_stripes(self._h, nstripes), "sw_set_virtual_stripes")
+
+    def set_grid(self, ctas: int = 0):
+        """Cap the CTAs of every fill launch (0: resident capacity), so bands
+        outnumber CTAs and the multi-wave band pipeline runs on small inputs."""
+        self._check(self._lib.sw_set_grid(self._h, ctas), "sw_set_grid")
 
     def stripe_export(self, max_rows: int) -> bytes:
         """Allocate this rank's left-border receive area; returns its 64-byte CUDA IPC handle."""

@@ -316,6 +316,7 @@ struct sw_ctx {
     sw_stats stats{};
     char errbuf[512] = {0};
     int variant_override = -1;
+    int grid_cap = 0;           // sw_set_grid: CTAs per fill launch (0 = resident capacity; testing)
     int vstripes = 1;           // virtual stripes for the single-process calls
     S1Rows s1;                  // special rows resident from the last Stage-1 call
     int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
@@ -518,6 +519,13 @@ extern "C" int sw_set_patch(sw_ctx *ctx, int on)
 {
     if (!ctx || on < 0 || on > 1) return SW_EINVAL;
     ctx->patch = on;
+    return SW_OK;
+}
+
+extern "C" int sw_set_grid(sw_ctx *ctx, int ctas)
+{
+    if (!ctx || ctas < 0) return SW_EINVAL;
+    ctx->grid_cap = ctas;
     return SW_OK;
 }
 
@@ -826,6 +834,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     // every CTA of every stripe must be co-resident (stripes wait on each other)
     int per_stripe = std::max(1, std::min(nb, blocks_per_sm * ctx->num_sms / NS));
     if (const char *g = getenv("SWB_GRID")) per_stripe = std::max(1, std::min(per_stripe, atoi(g) / NS));
+    if (ctx->grid_cap > 0) per_stripe = std::max(1, std::min(per_stripe, ctx->grid_cap / NS));
     const int grid = per_stripe * NS;
     hck[1] = hnow();
     if ((rc = grow(ctx, ctx->slots, (size_t)grid * sizeof(int4)))) return rc;

@@ -9,8 +9,8 @@ under (max, min i, min j) into the GPU's best cell.  Bands run in parallel on
 the host cores.  C2 is checked completely (every row, the global best); C3 is
 checked on a seeded sample of bands plus the band that holds the end cell.
 """
-import multiprocessing as mp
 import os
+from multiprocessing.pool import ThreadPool
 
 import numpy as np
 import pytest
@@ -44,10 +44,12 @@ def _band_job(args):
 
 
 def _run_bands(A, B, rows, jobs):
+    """Bands in parallel on the host cores: threads, since the oracle's C band
+    loop runs inside a ctypes call that releases the GIL (no fork of this
+    CUDA-initialised process)."""
     _G.update(A=A.tobytes(), B=B.tobytes(), rows=rows)
     oracle.build()
-    ctx = mp.get_context("fork")
-    with ctx.Pool(min(len(jobs), os.cpu_count() or 4)) as pool:
+    with ThreadPool(min(len(jobs), os.cpu_count() or 4)) as pool:
         return pool.map(_band_job, jobs, chunksize=1)
 
 
@@ -89,15 +91,11 @@ def test_c2_full_band_induction(ctx):
     assert (st.i, st.j) == (cfg.params["a0"], cfg.params["b0"])  # the planted segment's start (Table III shape)
 
 
-@pytest.mark.skipif(not os.environ.get("SWB_SLOW"), reason="set SWB_SLOW=1 (several minutes of host CPU)")
-def test_c3_sampled_band_induction(ctx):
-    cfg = synth.CONFIGS["C3"]
+def _sampled_induction(ctx, cfg, k, sample, expect_kernel):
+    """Stage 1 of `cfg` at special-row spacing k; the oracle recomputes the
+    sampled bands [q k, (q + 1) k) from the GPU's row q k and must reproduce row
+    (q + 1) k bit for bit; the band holding the end cell must hold the best."""
     A, B = synth.make_pair(cfg)
-    k = 2048  # verification spacing (the kernel configuration is the bench's)
-    rng = np.random.default_rng(3)
-    nbands = cfg.m // k
-    sample = set(int(x) for x in rng.choice(nbands, size=12, replace=False))
-    sample.update({nbands - 1, nbands})  # the last full band and the ragged tail (holds the end cell)
     keep = set()
     for q in sample:
         keep.update({q * k, (q + 1) * k})
@@ -108,10 +106,51 @@ def test_c3_sampled_band_induction(ctx):
             rows[row] = (H.copy(), F.copy())
 
     got, _ = ctx.align_stage1(A, B, *PAPER, k=k, sink=sink)
+    s1 = ctx.stats()
+    assert (s1["alpha"], s1["warps"], s1["patched"]) == expect_kernel, s1
+    assert s1["special_rows"] == cfg.m // k
     jobs = [(q, q * k, min((q + 1) * k, cfg.m)) for q in sorted(sample) if q * k < cfg.m]
     res = _run_bands(A, B, rows, jobs)
     assert all(ok for _, ok, _ in res), [q for q, ok, _ in res if not ok]
     qe = (got.i - 1) // k
-    assert qe in sample
+    assert qe in sample, (qe, sorted(sample))
     band_best = {q: b for q, _, b in res}[qe]
     assert band_best == got.astuple()
+    # no sampled band may hold a better cell than the reported best (the total order)
+    for q, _, b in res:
+        assert b[0] < got.score or (b[0] == got.score and (b[1], b[2]) >= (got.i, got.j)), (q, b, got)
+    return got
+
+
+def test_c3_sampled_band_induction(ctx):
+    """C3 (5M x 5M, whole-length homology) in the geometry its bench line runs
+    (alpha 16 x 8 warps, 1221 bands of 4096 rows on 148 CTAs: 8+ waves):
+    special rows every 4096 rows (one per band, drained by the I/O warp); a
+    seeded sample of bands plus the last full band and the ragged tail, where
+    the end cell lies."""
+    cfg = synth.CONFIGS["C3"]
+    k = 4096
+    rng = np.random.default_rng(3)
+    nbands = cfg.m // k
+    sample = set(int(x) for x in rng.choice(nbands, size=10, replace=False))
+    sample.update({nbands - 1, nbands})
+    got = _sampled_induction(ctx, cfg, k, sample, (-16, 8, 1))
+    assert got.i > cfg.m - 2 * k  # whole-length alignment ends near the corner
+
+
+def test_c4_sampled_band_induction(ctx):
+    """C4 (10M x 10M, the scaling config) in the geometry bench.py times
+    (alpha 32 x 8 warps, 8192-row bands: 1221 bands on 148 CTAs, 8 full waves
+    and a partial ninth): special rows every 8192 rows; a seeded sample of
+    bands from every wave, the bands around the planted homology (the end
+    cell) and the ragged last band."""
+    cfg = synth.CONFIGS["C4"]
+    k = 8192
+    rng = np.random.default_rng(4)
+    nbands = cfg.m // k
+    sample = set(int(x) for x in rng.choice(nbands, size=4, replace=False))
+    a0, L = cfg.params["a0"], cfg.params["L"]
+    sample.update(range(a0 // k, (a0 + 2 * L) // k + 1))
+    sample.add(nbands)  # the ragged last band
+    got = _sampled_induction(ctx, cfg, k, sample, (-32, 8, 1))
+    assert a0 < got.i <= a0 + 2 * L
