@@ -90,12 +90,38 @@ typedef struct {
     int32_t alpha, warps, width, grid; /* launch configuration */
     int32_t patched;   /* 1: the packed kernel ran with the gap penalties patched in as
                           instruction immediates; 0: runtime operands */
+    int32_t devices;   /* device entries that ran bands (band-cyclic multi-GPU Stage 1) */
+    int32_t sp_slots;  /* special-row ring slots per unit (= the row count when all stayed resident) */
+    int32_t tail_alpha, tail_warps, tail_grid; /* tail segment geometry (0: none; alpha < 0: packed) */
+    int64_t tail_rows; /* rows of the tail segment */
 } sw_stats;
 
-/* Create a context on the given CUDA devices.  Round 1 supports exactly one
- * device per context (one process per GPU); device_ids[0] is used.
- * Allocates the library's streams.  Returns SW_EINVAL / SW_ECUDA. */
+/* Create a context on n_devices in {1, 2, 4, 8} CUDA devices.
+ * device_ids[0] is the primary device: the reverse pass, Stage 2 and Stages
+ * 3-5 run there.  With n_devices > 1, Stage 1 (sw_align_stage1*) runs as one
+ * band pipeline across the devices (band-cyclic: device d takes bands d,
+ * d + n, ...; each band's bottom row goes to the next device by peer stores
+ * over NVLink), or as column stripes (sw_set_multi_gpu); the
+ * library combines the per-device best cells under the total order of reading
+ * S4 and hands the sink whole special rows.  Peer access is enabled between
+ * every pair of distinct devices (SW_EINVAL if a pair has no P2P path).  An id
+ * may repeat ("virtual peers" on one GPU, for testing): its entries share that
+ * GPU's SMs.  Allocates the library's streams.  Returns SW_EINVAL / SW_ECUDA. */
 int sw_init(const int *device_ids, int n_devices, sw_ctx **out);
+
+/* Number of device entries of the context (sw_init's n_devices). */
+int sw_device_count(const sw_ctx *ctx);
+
+/* Multi-device Stage-1 partition (testing / tuning; default 1).  cyclic = 1:
+ * band-cyclic rows (one pipeline of every device's CTAs); 0: the virtual
+ * column stripes of one device (the entries beyond the first idle).
+ * SW_EINVAL outside {0, 1}. */
+int sw_set_multi_gpu(sw_ctx *ctx, int cyclic);
+
+/* Total order of best cells (reading S4: higher score, then smaller i, then
+ * smaller j; (0, 0, 0) when every score is 0) over `count` results, e.g. the
+ * per-rank results of a multi-process stripe run.  SW_EINVAL on NULL. */
+int sw_combine_best(const sw_result *results, int count, sw_result *out);
 
 /* Stage 1 on host sequences.
  *   seqA : S0, m bytes of ACGTacgt (not NUL-terminated, borrowed for the call)
@@ -231,6 +257,24 @@ int sw_set_patch(sw_ctx *ctx, int on);
  * identical for every value.  SW_EINVAL for a NULL ctx or ctas < 0. */
 int sw_set_grid(sw_ctx *ctx, int ctas);
 
+/* Tail segment of a multi-wave Stage-1 fill (testing /
+ * tuning).  mode -1 (default): automatic -- when the last wave of bands is
+ * partial, the rows after the last full wave run as a second launch with a
+ * shorter band height, if the band-pipeline model says it is faster; 0: never;
+ * v + 1 (v a packed geometry of sw_set_kernel with a shorter band): always
+ * that geometry when the fill has a partial last wave.  Results are identical.
+ * SW_EINVAL outside -1 .. 14. */
+int sw_set_tail(sw_ctx *ctx, int mode);
+
+/* Device-memory budget of the special-row ring in bytes (testing / tuning;
+ * 0 = default, 80 % of the free HBM).  Special rows that do not all fit stay
+ * in a ring of as many slots as the budget holds (at least one band's rows);
+ * a band waits for its slots until the host has copied the rows that used them
+ * (back-pressure, P:178's bounded SRA), and the library keeps the rows in a
+ * host store for Stage 2.  Any k >= 1 runs under any budget.
+ * SW_EINVAL for bytes < 0. */
+int sw_set_row_budget(sw_ctx *ctx, int64_t bytes);
+
 /* ---- Column-stripe pipeline ----
  * The matrix is split into column stripes; stripe g sweeps every band of its
  * columns and hands the band's right-edge (t = H - G_first, E) column to stripe
@@ -249,10 +293,23 @@ int sw_set_virtual_stripes(sw_ctx *ctx, int nstripes);
 int sw_stripe_export(sw_ctx *ctx, int64_t max_rows, void *handle_out);
 int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t max_rows);
 
+/* Highest epoch this context has run a stripe call with (0: none).  A group
+ * of ranks agrees on the next epoch as 1 + the maximum over its ranks, so a
+ * new group on a reused context never repeats an epoch its receive area has
+ * seen. */
+int32_t sw_stripe_epoch(const sw_ctx *ctx);
+
+/* The kernel geometry the next stripe call with these arguments would run
+ * (alpha < 0: the packed kernel; warps per CTA): ranks of one group must agree
+ * on it (the per-(band, warp) border flags), which the caller checks before
+ * the call. */
+int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+            int64_t special_row_interval, int32_t *alpha, int32_t *warps);
+
 /* Stage 1 on this rank's stripe: global columns [c_lo, c_hi) of S1 (0-based),
  * all m rows.  dseqA / dseqB are the WHOLE sequences in this device's memory.
- * `epoch` (>= 1) must be the same on all ranks for one alignment and grow by
- * one per alignment.  `sink` receives this stripe's slice of each special row:
+ * `epoch` must be the same on all ranks for one alignment and above
+ * sw_stripe_epoch() of every rank (else SW_EINVAL).  `sink` receives this stripe's slice of each special row:
  * H, F = columns c_lo+1 .. c_hi, n = c_hi - c_lo.  `out` is this stripe's best
  * (score, i, j) in global coordinates; the global best is the maximum over
  * ranks under the same order (score, then smallest i, then smallest j). */

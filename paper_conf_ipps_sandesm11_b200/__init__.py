@@ -46,6 +46,13 @@ EXPORTED = [
     "sw_set_patch",
     "sw_set_virtual_stripes",
     "sw_set_grid",
+    "sw_set_tail",
+    "sw_set_row_budget",
+    "sw_set_multi_gpu",
+    "sw_device_count",
+    "sw_combine_best",
+    "sw_stripe_epoch",
+    "sw_plan",
     "sw_stripe_export",
     "sw_stripe_connect",
     "sw_align_stage1_stripe",
@@ -98,6 +105,12 @@ class Stats(ctypes.Structure):
         ("width", ctypes.c_int32),
         ("grid", ctypes.c_int32),
         ("patched", ctypes.c_int32),
+        ("devices", ctypes.c_int32),
+        ("sp_slots", ctypes.c_int32),
+        ("tail_alpha", ctypes.c_int32),
+        ("tail_warps", ctypes.c_int32),
+        ("tail_grid", ctypes.c_int32),
+        ("tail_rows", ctypes.c_int64),
     ]
 
     def as_dict(self):
@@ -156,6 +169,20 @@ def load_library(path: str = LIB_PATH):
     lib.sw_set_virtual_stripes.restype = ctypes.c_int
     lib.sw_set_grid.argtypes = [vp, ctypes.c_int]
     lib.sw_set_grid.restype = ctypes.c_int
+    lib.sw_set_tail.argtypes = [vp, ctypes.c_int]
+    lib.sw_set_tail.restype = ctypes.c_int
+    lib.sw_set_row_budget.argtypes = [vp, i64]
+    lib.sw_set_row_budget.restype = ctypes.c_int
+    lib.sw_set_multi_gpu.argtypes = [vp, ctypes.c_int]
+    lib.sw_set_multi_gpu.restype = ctypes.c_int
+    lib.sw_device_count.argtypes = [vp]
+    lib.sw_device_count.restype = ctypes.c_int
+    lib.sw_combine_best.argtypes = [R, ctypes.c_int, R]
+    lib.sw_combine_best.restype = ctypes.c_int
+    lib.sw_stripe_epoch.argtypes = [vp]
+    lib.sw_stripe_epoch.restype = i32
+    lib.sw_plan.argtypes = [vp, i64, i64, i32, i32, i32, i32, i64, ctypes.POINTER(i32), ctypes.POINTER(i32)]
+    lib.sw_plan.restype = ctypes.c_int
     lib.sw_stripe_export.argtypes = [vp, i64, vp]
     lib.sw_stripe_export.restype = ctypes.c_int
     lib.sw_stripe_connect.argtypes = [vp, vp, i64]
@@ -202,17 +229,33 @@ class Result:
         return (self.score, self.i, self.j)
 
 
-class Context:
-    """One engine context on one CUDA device (one process per GPU)."""
+def combine_best(results) -> tuple:
+    """The library's total order of best cells (sw_combine_best) over (score, i, j) triples."""
+    lib = load_library()
+    rs = list(results)
+    arr = (_Result * max(1, len(rs)))(*[_Result(int(a), int(b), int(c)) for a, b, c in rs])
+    out = _Result()
+    rc = lib.sw_combine_best(arr, len(rs), ctypes.byref(out))
+    if rc != SW_OK:
+        raise SwError(rc, "sw_combine_best")
+    return (out.score, out.i, out.j)
 
-    def __init__(self, device: int = 0):
+
+class Context:
+    """One engine context on one CUDA device (one process per GPU), or on
+    several devices (``devices=[0, 1, ...]``: Stage 1 runs as one band pipeline
+    across them)."""
+
+    def __init__(self, device: int = 0, devices=None):
         self._lib = load_library()
         self._h = ctypes.c_void_p()
-        ids = (ctypes.c_int * 1)(device)
-        rc = self._lib.sw_init(ids, 1, ctypes.byref(self._h))
+        ids_list = list(devices) if devices is not None else [device]
+        ids = (ctypes.c_int * len(ids_list))(*ids_list)
+        rc = self._lib.sw_init(ids, len(ids_list), ctypes.byref(self._h))
         if rc != SW_OK:
-            raise SwError(rc, f"sw_init(device={device}) failed: {self._lib.sw_strerror(rc).decode()}")
-        self.device = device
+            raise SwError(rc, f"sw_init(devices={ids_list}) failed: {self._lib.sw_strerror(rc).decode()}")
+        self.device = ids_list[0]
+        self.devices = ids_list
 
     # ------------------------------------------------------------------ helpers
     def _check(self, rc, what):
@@ -359,10 +402,37 @@ class Context:
         (the multi-GPU border protocol, run inside one launch)."""
         self._check(self._lib.sw_set_virtual_stripes(self._h, nstripes), "sw_set_virtual_stripes")
 
+    def set_tail(self, mode: int = -1):
+        """Tail segment: -1 automatic, 0 off, v + 1 force packed geometry v (testing)."""
+        self._check(self._lib.sw_set_tail(self._h, mode), "sw_set_tail")
+
+    def set_row_budget(self, nbytes: int = 0):
+        """Device bytes for the special-row ring (0: default); smaller budgets
+        stream the rows through a ring with back-pressure."""
+        self._check(self._lib.sw_set_row_budget(self._h, nbytes), "sw_set_row_budget")
+
+    def set_multi_gpu(self, cyclic: bool = True):
+        """Multi-device Stage 1: band-cyclic (default) or column stripes on the first device."""
+        self._check(self._lib.sw_set_multi_gpu(self._h, int(bool(cyclic))), "sw_set_multi_gpu")
+
+    def device_count(self) -> int:
+        return int(self._lib.sw_device_count(self._h))
+
     def set_grid(self, ctas: int = 0):
         """Cap the CTAs of every fill launch (0: resident capacity), so bands
         outnumber CTAs and the multi-wave band pipeline runs on small inputs."""
         self._check(self._lib.sw_set_grid(self._h, ctas), "sw_set_grid")
+
+    def stripe_epoch(self) -> int:
+        """Highest epoch this context ran a stripe call with (sw_stripe_epoch)."""
+        return int(self._lib.sw_stripe_epoch(self._h))
+
+    def plan(self, m, n, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0):
+        """(alpha, warps) of the geometry the next stripe call would run (alpha < 0: packed)."""
+        a, w = ctypes.c_int32(0), ctypes.c_int32(0)
+        self._check(self._lib.sw_plan(self._h, m, n, match, mismatch, gap_open, gap_ext, k, ctypes.byref(a),
+                                      ctypes.byref(w)), "sw_plan")
+        return (a.value, w.value)
 
     def stripe_export(self, max_rows: int) -> bytes:
         """Allocate this rank's left-border receive area; returns its 64-byte CUDA IPC handle."""

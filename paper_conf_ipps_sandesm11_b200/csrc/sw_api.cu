@@ -177,7 +177,10 @@ static Variant make_variant()
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
 static constexpr int NVARIANTS = 14;
-static constexpr int NINT32_VARIANTS = 8;  // variants 0..7 have int32 kernels; 8.. are packed-only (alpha 32)
+static constexpr int NINT32_VARIANTS = 8;
+// Dynamic shared memory the tail launch requests: more than
+// half an SM's 228 KB, so its CTAs take one SM each as the main launch frees them.
+static constexpr int TAIL_SMEM = 120 * 1024;  // variants 0..7 have int32 kernels; 8.. are packed-only (alpha 32)
 
 static const Variant &variant_for(int idx)
 {
@@ -221,12 +224,30 @@ struct RecvArea {
     int *lready() const { return (int *)((char *)base + rows * sizeof(int2)); }
 };
 
-// Where the special rows of the last Stage-1 call live (for Stage 2).
+// Where the special rows of the last Stage-1 call live (for Stage 2): in the
+// device ring (every row resident when the ring never wrapped), else in the
+// library's host store (the paper's SRA).
 struct S1Rows {
     bool valid = false;
+    bool resident = false;       // row q at sp[0] + q * stride (H[0..n), F at + ld)
+    bool stored = false;         // row q in host_rows[q] (H[0..n), F[n..2n))
     int64_t m = 0, n = 0, k = 0;
     int32_t ma = 0, mi = 0, go = 0, ge = 0;
-    int64_t ld = 0, stride = 0;  // row q at sp[0] + q * stride: H[0..n), F at + ld
+    int64_t ld = 0, stride = 0;
+};
+
+constexpr int MAX_DEV = 8;
+
+// Device entries 1.. of a multi-device context (entry 0 is the context's own
+// fields).  Entries may repeat a physical device ("virtual peers", testing):
+// their CTAs then share the GPU, and each launch is capped to its share.
+struct Peer {
+    int device = 0;
+    cudaStream_t stream = nullptr, side = nullptr;
+    cudaEvent_t ev[4] = {};
+    std::vector<cudaEvent_t> ev_row;
+    DevBuf a2, b2, misc, slots;
+    int4 *res_h = nullptr;
 };
 
 // ---------------------------------------------------------------- patched packed kernels
@@ -294,8 +315,13 @@ static const PatchSites &patch_sites()
 struct sw_ctx {
     int device = 0;
     int num_sms = 0;
+    int ndev = 1;               // device entries (sw_init's n_devices)
+    int share[MAX_DEV] = {1};   // entries on the same physical GPU as entry d (grid share)
+    Peer peer[MAX_DEV - 1];     // entries 1 .. ndev-1
     cudaStream_t stream = nullptr, side = nullptr;
+    cudaStream_t aux = nullptr; // tail-segment launches (device 0)
     cudaEvent_t ev[6] = {};
+    cudaEvent_t ev_aux[2] = {};
     std::vector<cudaEvent_t> ev_row;  // one per staging slot: the slot's final copy is done
     int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
@@ -317,6 +343,15 @@ struct sw_ctx {
     char errbuf[512] = {0};
     int variant_override = -1;
     int grid_cap = 0;           // sw_set_grid: CTAs per fill launch (0 = resident capacity; testing)
+    int tail_mode = -1;         // sw_set_tail: -1 automatic, 0 off, v >= 0 + 1: force variant v-1 for the tail
+    int cyclic = 1;             // multi-device Stage 1: 1 band-cyclic, 0 column stripes
+    size_t sp_budget = 0;       // sw_set_row_budget: device bytes for the special-row ring (0: 0.8 x free)
+    int pepoch = 0;             // tag of the last call's band-progress words
+    HostBuf released;           // mapped, portable: special rows 0 .. value-1 have left the device ring
+    std::vector<std::vector<int32_t>> host_rows;  // host store of special rows (ring mode)
+    DevBuf s2row;               // Stage 2: one special row uploaded from the host store
+    int unit_dev[MAX_STRIPES] = {-1, -1, -1, -1, -1, -1, -1, -1};  // physical device of unit u's rowb / progress / sp / vrecv (-1: none)
+    int stripe_epoch = 0;       // highest epoch of a rank-mode stripe call (sw_stripe_epoch)
     int vstripes = 1;           // virtual stripes for the single-process calls
     S1Rows s1;                  // special rows resident from the last Stage-1 call
     int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
@@ -361,7 +396,8 @@ static int grow_host(sw_ctx *ctx, HostBuf &b, size_t bytes, bool mapped)
     if (b.p) cudaFreeHost(b.p);
     b.p = nullptr;
     b.cap = 0;
-    if (cudaHostAlloc(&b.p, std::max<size_t>(bytes, 64), mapped ? cudaHostAllocMapped : cudaHostAllocDefault) != cudaSuccess) {
+    // portable: the mapped flags are read by every device of a multi-device context
+    if (cudaHostAlloc(&b.p, std::max<size_t>(bytes, 64), cudaHostAllocPortable | (mapped ? cudaHostAllocMapped : 0)) != cudaSuccess) {
         cudaGetLastError();
         snprintf(ctx->errbuf, sizeof(ctx->errbuf), "cudaHostAlloc(%zu) failed", bytes);
         return SW_ENOMEM;
@@ -405,14 +441,51 @@ extern "C" const char *sw_strerror(int code)
 
 extern "C" const char *sw_last_error(const sw_ctx *ctx) { return ctx ? ctx->errbuf : ""; }
 
+// Per-device view of a context entry (entry 0: the context's own fields).
+struct DevView {
+    int device;
+    cudaStream_t stream, side;
+    cudaEvent_t *ev;
+    std::vector<cudaEvent_t> *ev_row;
+    DevBuf *a2, *b2, *misc, *slots;
+    int4 *res_h;
+};
+static DevView dview(sw_ctx *ctx, int d)
+{
+    if (d == 0)
+        return DevView{ctx->device, ctx->stream, ctx->side, ctx->ev, &ctx->ev_row, &ctx->a2, &ctx->b2, &ctx->misc,
+                       &ctx->slots, ctx->res_h};
+    Peer &P = ctx->peer[d - 1];
+    return DevView{P.device, P.stream, P.side, P.ev, &P.ev_row, &P.a2, &P.b2, &P.misc, &P.slots, P.res_h};
+}
+
+static void set_kernel_attrs()
+{
+    for (int i = 0; i < NVARIANTS; i++) {
+        const Variant &v = variant_for(i);
+        if (v.local_fn) cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+        if (v.global_fn) cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+        if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, TAIL_SMEM);
+        if (v.packed_global_fn)
+            cudaFuncSetAttribute(v.packed_global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
+    }
+}
+
 extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
 {
-    if (!out || n_devices != 1 || !device_ids) return SW_EINVAL;
+    if (!out || !device_ids || !(n_devices == 1 || n_devices == 2 || n_devices == 4 || n_devices == 8)) return SW_EINVAL;
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0) { cudaGetLastError(); return SW_ECUDA; }
-    if (device_ids[0] < 0 || device_ids[0] >= ndev) return SW_EINVAL;
+    for (int d = 0; d < n_devices; d++)
+        if (device_ids[d] < 0 || device_ids[d] >= ndev) return SW_EINVAL;
     sw_ctx *ctx = new sw_ctx();
     ctx->device = device_ids[0];
+    ctx->ndev = n_devices;
+    for (int d = 1; d < n_devices; d++) ctx->peer[d - 1].device = device_ids[d];
+    for (int d = 0; d < n_devices; d++) {
+        ctx->share[d] = 0;
+        for (int e = 0; e < n_devices; e++) ctx->share[d] += device_ids[e] == device_ids[d];
+    }
     int rc = SW_OK;
     do {
         cudaError_t e;
@@ -420,24 +493,55 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
         cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, ctx->device);
         if ((e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
         if ((e = cudaStreamCreateWithFlags(&ctx->side, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
+        if ((e = cudaStreamCreateWithFlags(&ctx->aux, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
         for (auto &ev : ctx->ev)
             if ((e = cudaEventCreate(&ev)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
+        for (auto &ev : ctx->ev_aux)
+            if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
         if (rc) break;
         if ((e = cudaHostAlloc(&ctx->res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
-        for (int i = 0; i < NVARIANTS; i++) {
-            const Variant &v = variant_for(i);
-            if (v.local_fn) cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
-            if (v.global_fn) cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
-            if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
-            if (v.packed_global_fn)
-                cudaFuncSetAttribute(v.packed_global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
-        }
+        if (cudaHostAlloc(&ctx->released.p, 64, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) { rc = SW_ENOMEM; break; }
+        ctx->released.cap = 64;
+        ctx->released.mapped = true;
+        set_kernel_attrs();
         if ((e = cudaGetLastError()) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaFuncSetAttribute"); break; }
+        // entries 1..: streams, events and peer access in both directions with
+        // every other physical device of the context (the band-cyclic pipeline
+        // stores each band's bottom row into the next entry's memory)
+        for (int d = 1; d < n_devices && !rc; d++) {
+            Peer &P = ctx->peer[d - 1];
+            if ((e = cudaSetDevice(P.device)) != cudaSuccess) { rc = cuda_fail(ctx, e, "cudaSetDevice(peer)"); break; }
+            if ((e = cudaStreamCreateWithFlags(&P.stream, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
+            if ((e = cudaStreamCreateWithFlags(&P.side, cudaStreamNonBlocking)) != cudaSuccess) { rc = cuda_fail(ctx, e, "stream"); break; }
+            for (auto &ev : P.ev)
+                if ((e = cudaEventCreate(&ev)) != cudaSuccess) { rc = cuda_fail(ctx, e, "event"); break; }
+            if (rc) break;
+            if ((e = cudaHostAlloc(&P.res_h, 4 * sizeof(int4), cudaHostAllocDefault)) != cudaSuccess) { rc = SW_ENOMEM; break; }
+            set_kernel_attrs();
+        }
+        for (int d = 0; d < n_devices && !rc; d++)
+            for (int f = 0; f < n_devices && !rc; f++) {
+                if (device_ids[d] == device_ids[f]) continue;
+                int can = 0;
+                cudaDeviceCanAccessPeer(&can, device_ids[d], device_ids[f]);
+                if (!can) {
+                    snprintf(ctx->errbuf, sizeof(ctx->errbuf), "device %d cannot access device %d (no P2P)", device_ids[d], device_ids[f]);
+                    rc = SW_EINVAL;
+                    break;
+                }
+                cudaSetDevice(device_ids[d]);
+                e = cudaDeviceEnablePeerAccess(device_ids[f], 0);
+                if (e == cudaErrorPeerAccessAlreadyEnabled) { cudaGetLastError(); e = cudaSuccess; }
+                if (e != cudaSuccess) rc = cuda_fail(ctx, e, "cudaDeviceEnablePeerAccess");
+            }
+        cudaSetDevice(ctx->device);
+        if (rc) break;
         if (const char *ov = getenv("SWB_VARIANT")) ctx->variant_override = atoi(ov);
         if (const char *vs = getenv("SWB_VSTRIPES")) ctx->vstripes = std::max(1, std::min(MAX_STRIPES, atoi(vs)));
         if (const char *to = getenv("SWB_TIMEOUT_S")) ctx->timeout_ns = (long long)(atof(to) * 1e9);
         if (const char *pk = getenv("SWB_PACKED")) ctx->packed = atoi(pk);
         if (const char *pt = getenv("SWB_PATCH")) ctx->patch = atoi(pt);
+        if (const char *tl = getenv("SWB_TAIL")) ctx->tail_mode = atoi(tl);
     } while (0);
     if (rc) { sw_shutdown(ctx); return rc; }
     *out = ctx;
@@ -447,31 +551,53 @@ extern "C" int sw_init(const int *device_ids, int n_devices, sw_ctx **out)
 extern "C" void sw_shutdown(sw_ctx *ctx)
 {
     if (!ctx) return;
+    for (int d = 1; d < ctx->ndev; d++) {
+        Peer &P = ctx->peer[d - 1];
+        if (cudaSetDevice(P.device) != cudaSuccess) continue;
+        if (P.stream) cudaStreamSynchronize(P.stream);
+        if (P.side) cudaStreamSynchronize(P.side);
+        for (DevBuf *b : {&P.a2, &P.b2, &P.misc, &P.slots})
+            if (b->p) cudaFree(b->p);
+        if (P.res_h) cudaFreeHost(P.res_h);
+        for (auto &ev : P.ev)
+            if (ev) cudaEventDestroy(ev);
+        for (auto &ev : P.ev_row)
+            if (ev) cudaEventDestroy(ev);
+        if (P.stream) cudaStreamDestroy(P.stream);
+        if (P.side) cudaStreamDestroy(P.side);
+    }
     cudaSetDevice(ctx->device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
     if (ctx->side) cudaStreamSynchronize(ctx->side);
+    if (ctx->aux) cudaStreamSynchronize(ctx->aux);
     for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg, &ctx->capbuf, &ctx->mm_parts,
-                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves, &ctx->mm_err})
+                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves, &ctx->mm_err, &ctx->s2row})
         if (b->p) cudaFree(b->p);
     for (int s = 0; s < MAX_STRIPES; s++) {
+        cudaSetDevice(ctx->unit_dev[s] >= 0 ? ctx->unit_dev[s] : ctx->device);  // a unit's buffers live on its entry's device
         for (DevBuf *b : {&ctx->rowb[s], &ctx->progress[s], &ctx->sp[s]})
             if (b->p) cudaFree(b->p);
         if (ctx->flags[s].p) cudaFreeHost(ctx->flags[s].p);
         if (ctx->colp[s].p) cudaFreeHost(ctx->colp[s].p);
         if (ctx->vrecv[s].base) cudaFree(ctx->vrecv[s].base);
     }
+    cudaSetDevice(ctx->device);
     for (auto &P : ctx->patched)
         if (P.lib) cudaLibraryUnload(P.lib);
     if (ctx->right_base) cudaIpcCloseMemHandle(ctx->right_base);
     if (ctx->recv.base) cudaFree(ctx->recv.base);
     if (ctx->stage.p) cudaFreeHost(ctx->stage.p);
+    if (ctx->released.p) cudaFreeHost(ctx->released.p);
     if (ctx->res_h) cudaFreeHost(ctx->res_h);
     for (auto &ev : ctx->ev)
+        if (ev) cudaEventDestroy(ev);
+    for (auto &ev : ctx->ev_aux)
         if (ev) cudaEventDestroy(ev);
     for (auto &ev : ctx->ev_row)
         if (ev) cudaEventDestroy(ev);
     if (ctx->stream) cudaStreamDestroy(ctx->stream);
     if (ctx->side) cudaStreamDestroy(ctx->side);
+    if (ctx->aux) cudaStreamDestroy(ctx->aux);
     delete ctx;
 }
 
@@ -519,6 +645,44 @@ extern "C" int sw_set_patch(sw_ctx *ctx, int on)
 {
     if (!ctx || on < 0 || on > 1) return SW_EINVAL;
     ctx->patch = on;
+    return SW_OK;
+}
+
+extern "C" int sw_set_tail(sw_ctx *ctx, int mode)
+{
+    if (!ctx || mode < -1 || mode > NVARIANTS) return SW_EINVAL;
+    ctx->tail_mode = mode;
+    return SW_OK;
+}
+
+extern "C" int sw_set_row_budget(sw_ctx *ctx, int64_t bytes)
+{
+    if (!ctx || bytes < 0) return SW_EINVAL;
+    ctx->sp_budget = (size_t)bytes;
+    return SW_OK;
+}
+
+extern "C" int sw_set_multi_gpu(sw_ctx *ctx, int cyclic)
+{
+    if (!ctx || cyclic < 0 || cyclic > 1) return SW_EINVAL;
+    ctx->cyclic = cyclic;
+    return SW_OK;
+}
+
+extern "C" int sw_device_count(const sw_ctx *ctx) { return ctx ? ctx->ndev : 0; }
+
+extern "C" int32_t sw_stripe_epoch(const sw_ctx *ctx) { return ctx ? ctx->stripe_epoch : 0; }
+
+extern "C" int sw_combine_best(const sw_result *results, int count, sw_result *out)
+{
+    if (!out || count < 0 || (count > 0 && !results)) return SW_EINVAL;
+    sw_result b{0, 0, 0};
+    for (int x = 0; x < count; x++) {
+        const sw_result &r = results[x];
+        if (r.score <= 0) continue;
+        if (r.score > b.score || (r.score == b.score && (r.i < b.i || (r.i == b.i && r.j < b.j)))) b = r;
+    }
+    *out = b;
     return SW_OK;
 }
 
@@ -608,6 +772,26 @@ struct Candidate {
     double cps_solo;  // columns/s of a CTA alone on its SM (C2: 133 bands on 148 SMs)
 };
 
+// profiles/r01_variants.txt; earlier entries win near-ties (3 %)
+static const Candidate kCands[] = {
+    {DEFAULT_VARIANT, false, 4.24e6, 4.24e6},  // int32, 8 warps + I/O warp
+    {1, true, 8.08e6, 7.74e6},                 // packed alpha 16, 8 warps + I/O warp
+    {8, true, 4.25e6, 7.86e6},                 // packed alpha 32, 4 warps + I/O warp (2 CTAs/SM)
+    {13, true, 4.45e6, 8.17e6},                // packed alpha 30, 4 warps + I/O warp (2 CTAs/SM)
+    {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
+    {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
+    {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
+};
+static constexpr int NCANDS = (int)(sizeof(kCands) / sizeof(kCands[0]));
+// Tail-segment candidates: column speed of one CTA alone on
+// its SM (the tail launch holds one CTA per SM).
+static const Candidate kTailCands[] = {
+    {0, true, 12.0e6, 12.0e6},   // packed alpha 16, 4 warps + I/O warp: 2048-row bands
+    {13, true, 8.17e6, 8.17e6},  // packed alpha 30, 4 warps: 3840-row bands
+    {8, true, 7.86e6, 7.86e6},   // packed alpha 32, 4 warps: 4096-row bands
+    {1, true, 7.74e6, 7.74e6},   // packed alpha 16, 8 warps: 4096-row bands
+};
+
 // Modelled fill time of a candidate: band b starts when its CTA is free and
 // band b-1 is `lag` columns ahead,
 //   start(b) = max(start(b - P) + n / cps, start(b - 1) + lag / cps),
@@ -675,7 +859,7 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf,
             return nullptr;
         }
         if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)(kind == 0 || kind == 3 ? V.smem16 : V.smem)) != cudaSuccess) {
+                                 (int)(kind == 0 ? std::max<size_t>(V.smem16, TAIL_SMEM) : kind == 3 ? V.smem16 : V.smem)) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
         }
@@ -684,7 +868,16 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf,
     return P->fn[kind][vidx];
 }
 
-static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
+// The packed kernel's preconditions for a local-mode fill.
+static bool packed_qualifies(const sw_ctx *ctx, const Job &J, const Variant &V)
+{
+    const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
+    const long long span = 32ll * V.alpha + 140;
+    return ctx->packed && J.local && V.packed_fn && (J.k == 0 || J.k % V.alpha == 0) &&
+           span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
+}
+
+static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16, int gpus = 1)
 {
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
     // packed preconditions: local mode, special rows at strip
@@ -722,19 +915,10 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         if (!*use16 && !V.local_fn) return variant_for(DEFAULT_VARIANT);  // packed-only geometry
         return V;
     }
-    // profiles/r01_variants.txt; earlier entries win near-ties (3 %)
-    static const Candidate cands[] = {
-        {DEFAULT_VARIANT, false, 4.24e6, 4.24e6},  // int32, 8 warps + I/O warp
-        {1, true, 8.08e6, 7.74e6},                 // packed alpha 16, 8 warps + I/O warp
-        {8, true, 4.25e6, 7.86e6},                 // packed alpha 32, 4 warps + I/O warp (2 CTAs/SM)
-        {13, true, 4.45e6, 8.17e6},                // packed alpha 30, 4 warps + I/O warp (2 CTAs/SM)
-        {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
-        {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
-        {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
-    };
+    const Candidate *cands = kCands;
     double best_t = 1e300;
     int best = 0;
-    for (int c = 0; c < (int)(sizeof(cands) / sizeof(cands[0])); c++) {
+    for (int c = 0; c < NCANDS; c++) {
         const Candidate &C = cands[c];
         const Variant &V = variant_for(C.variant);
         if (C.packed && !packed_ok(V)) continue;
@@ -744,10 +928,11 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
         int per_sm = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, V.nw * 32 + (C.packed ? V.io_warps : 1) * 32,
                                                       C.packed ? V.smem16 : V.smem);
-        const long long P = (long long)std::max(1, per_sm) * ctx->num_sms;
+        // band-cyclic multi-GPU: one pipeline of `gpus` x the resident CTAs
+        const long long P = (long long)std::max(1, per_sm) * ctx->num_sms * gpus;
         const long long bh = (long long)V.alpha * 32 * V.nw;
         const long long nb = std::max<long long>(1, (J.m + bh - 1) / bh);
-        const double cps = nb <= ctx->num_sms ? C.cps_solo : C.cps_full;
+        const double cps = nb <= (long long)ctx->num_sms * gpus ? C.cps_solo : C.cps_full;
         double t = model_fill_time(nb, P, std::max<long long>(J.n, 1), (2ll * V.nw + 2) * V.w, cps);
         // special rows that are not band bottoms are written by the compute
         // warps (SP1 tiles) instead of the I/O warp: measured +7.7 % on C2
@@ -762,54 +947,212 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16)
     return variant_for(cands[best].variant);
 }
 
+// One fill SEGMENT: a launch (per device entry) of one kernel geometry over
+// rows [row_base, row_base + nb BH).
+struct Seg {
+    const Variant *V = nullptr;
+    bool use16 = false;
+    int row_base = 0, band_base = 0, nb = 0, BH = 0;
+    const void *fn = nullptr;
+    size_t smem = 0;
+    int block = 0;
+    bool patched = false;
+    int grid[MAX_DEV] = {};
+};
+
+static bool distinct_devices(const sw_ctx *ctx)
+{
+    for (int d = 1; d < ctx->ndev; d++)
+        if (ctx->peer[d - 1].device != ctx->device) return true;
+    return false;
+}
+
+// Resolve a segment's kernel (patched image when available) and its per-entry grid.
+static int setup_seg(sw_ctx *ctx, const Job &J, Seg &G, int P, int NS, bool tail)
+{
+    const Variant &V = *G.V;
+    G.BH = V.alpha * 32 * V.nw;
+    G.fn = G.use16 ? (J.local ? V.packed_fn : V.packed_global_fn) : (J.local ? V.local_fn : V.global_fn);
+    G.smem = G.use16 ? V.smem16 : V.smem;
+    G.patched = false;
+    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, G.use16 ? (J.local ? 0 : 3) : J.local ? 1 : 2)) {
+        G.fn = pf;
+        G.patched = true;
+    }
+    // the tail launch asks for enough shared memory to hold one CTA per SM:
+    // its CTAs take the SMs the main launch frees one by one
+    if (tail) G.smem = std::max<size_t>(G.smem, (size_t)TAIL_SMEM);
+    G.block = V.nw * 32 + (G.use16 ? V.io_warps : 1) * 32;
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, G.fn, G.block, G.smem);
+    if (per_sm < 1) per_sm = 1;
+    for (int d = 0; d < P; d++) {
+        // every CTA of every stripe / entry must be co-resident (they wait on each other)
+        const int cap = std::max(1, per_sm * ctx->num_sms / (NS * (P > 1 ? ctx->share[d] : 1)));
+        const int bands_d = (G.nb - d + P - 1) / P;  // bands b = t P + d of this entry
+        int g = std::max(1, std::min(bands_d, cap));
+        if (const char *e = getenv("SWB_GRID")) g = std::max(1, std::min(g, atoi(e) / NS));
+        if (ctx->grid_cap > 0) g = std::max(1, std::min(g, ctx->grid_cap / NS));
+        G.grid[d] = g * NS;
+    }
+    return SW_OK;
+}
+
+// Tail segment: when a multi-wave fill leaves a partial last
+// wave (C4: 1221 bands of 8192 rows on 148 CTAs, the ninth wave a quarter
+// full), run the rows after the last full wave as a second launch of a
+// geometry with shorter bands, so they spread over every SM instead of a
+// quarter of them.  Returns the tail geometry and the main launch's band count,
+// or nullptr.  Automatic choice by the band-pipeline model; sw_set_tail forces.
+static const Variant *choose_tail(sw_ctx *ctx, const Job &J, const Seg &S0, int *nb1_out)
+{
+    if (ctx->tail_mode == 0 || (ctx->tail_mode < 0 && ctx->variant_override >= 0)) return nullptr;
+    const int P = S0.grid[0];
+    const int nb = S0.nb;
+    const int nb1 = (nb / P) * P;
+    if (nb <= P || nb1 == nb) return nullptr;  // one wave, or whole waves only
+    const long long m2 = J.m - (long long)nb1 * S0.BH;
+    const long long n = std::max<long long>(J.n, 1);
+    const Variant &V0 = *S0.V;
+    const int vidx0 = (int)(&V0 - &variant_for(0));
+    if (ctx->tail_mode > 0) {
+        const Variant &Vt = variant_for(ctx->tail_mode - 1);
+        if (!packed_qualifies(ctx, J, Vt) || Vt.alpha * 32 * Vt.nw >= S0.BH) return nullptr;
+        *nb1_out = nb1;
+        return &Vt;
+    }
+    double cps0 = 0;
+    for (int c = 0; c < NCANDS; c++)
+        if (kCands[c].variant == vidx0 && kCands[c].packed) cps0 = kCands[c].cps_full;
+    if (cps0 <= 0) return nullptr;
+    const long long lag0 = (2ll * V0.nw + 2) * V0.w;
+    const double t_no = model_fill_time(nb, P, n, lag0, cps0);
+    double best = 0.97 * t_no;
+    const Variant *pick = nullptr;
+    for (const Candidate &C : kTailCands) {
+        const Variant &Vt = variant_for(C.variant);
+        const long long bh = (long long)Vt.alpha * 32 * Vt.nw;
+        if (bh >= S0.BH || !packed_qualifies(ctx, J, Vt)) continue;
+        const long long nb2 = (m2 + bh - 1) / bh;
+        if (nb2 > ctx->num_sms) continue;  // the tail must fit in one wave of one CTA per SM
+        const long long lagt = (2ll * Vt.nw + 2) * Vt.w;
+        const double t = model_fill_time(nb1, P, n, lag0, cps0) + ((double)n + (double)(nb2 - 1) * lagt) / C.cps_solo;
+        if (t < best) {
+            best = t;
+            pick = &Vt;
+        }
+    }
+    if (pick) *nb1_out = nb1;
+    return pick;
+}
+
 static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
 {
     const auto h0 = std::chrono::steady_clock::now();
     if (J.local) ctx->s1.valid = false;
-    double hck[6] = {0, 0, 0, 0, 0, 0};
     auto hnow = [&]() { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - h0).count(); };
-    bool use16 = false;
-    const Variant &V = choose_variant(ctx, J, &use16);
-    hck[0] = hnow();
+    // band-cyclic multi-GPU Stage 1: entry d runs bands d, d + P, ...
+    // or column stripes, one per entry (mstr), with the (t, E) border column
+    // stored into the next entry's receive area
+    const bool multi = J.local && !J.rank_mode && J.nv == 1 && ctx->ndev > 1;
+    const bool cyc = multi && ctx->cyclic;
+    const bool mstr = multi && !ctx->cyclic;
+    const int P = multi ? ctx->ndev : 1;
+    const bool cross = multi && distinct_devices(ctx);
+    const int NS = (J.rank_mode || multi) ? 1 : J.nv;  // column stripes of one launch
+    const int NU = multi ? P : NS;                     // units: (entry, stripe) buffer sets
+    Seg seg[2];
+    int nseg = 1;
+    seg[0].V = &choose_variant(ctx, J, &seg[0].use16, cyc ? P : 1);
+    const Variant &V = *seg[0].V;
     const int W = V.w;
-    const int BH = V.alpha * 32 * V.nw;
     const int m = (int)J.m, n = (int)J.n;
-    const int nb = (m + BH - 1) / BH;
-    const long long wa = (J.m + 15) / 16 + 2, wb = (J.n + 15) / 16 + 2;
-    const int NS = J.rank_mode ? 1 : J.nv;
+    seg[0].BH = V.alpha * 32 * V.nw;
+    seg[0].nb = (m + seg[0].BH - 1) / seg[0].BH;
     int rc;
-
-    // stripe geometry
-    long long col0[MAX_STRIPES], wid[MAX_STRIPES];
-    if (J.rank_mode) {
-        col0[0] = J.c_lo;
-        wid[0] = J.c_hi - J.c_lo;
-    } else {
-        for (int s = 0; s < NS; s++) {
-            col0[s] = (long long)n * s / NS;
-            wid[s] = (long long)n * (s + 1) / NS - col0[s];
+    if ((rc = setup_seg(ctx, J, seg[0], P, NS, false))) return rc;
+    // the last partial wave of a multi-wave fill as a second launch with a
+    // smaller band height
+    if (!cyc && NS == 1 && !J.rank_mode && J.local && seg[0].use16) {
+        int nb1 = 0;
+        const Variant *Vt = choose_tail(ctx, J, seg[0], &nb1);
+        if (Vt) {
+            seg[1].V = Vt;
+            seg[1].use16 = true;
+            seg[1].row_base = nb1 * seg[0].BH;
+            seg[1].band_base = nb1;
+            seg[1].BH = Vt->alpha * 32 * Vt->nw;
+            seg[1].nb = (m - seg[1].row_base + seg[1].BH - 1) / seg[1].BH;
+            seg[0].nb = nb1;
+            if ((rc = setup_seg(ctx, J, seg[0], P, NS, false))) return rc;
+            if ((rc = setup_seg(ctx, J, seg[1], P, NS, true))) return rc;
+            nseg = 2;
         }
     }
-    for (int s = 0; s < NS; s++)
-        if (wid[s] <= 0) {
-            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe %d is empty (n=%d, stripes=%d)", s, n, NS);
+    const int nb_total = seg[0].nb + (nseg > 1 ? seg[1].nb : 0);
+    const double h_choose = hnow();
+    const long long wa = (J.m + 15) / 16 + 2, wb = (J.n + 15) / 16 + 2;
+
+    // stripe geometry (units of the band-cyclic mode all span [0, n))
+    long long col0[MAX_STRIPES], wid[MAX_STRIPES];
+    int udev[MAX_STRIPES];  // device entry of each unit
+    for (int u = 0; u < NU; u++) {
+        udev[u] = multi ? u : 0;
+        if (J.rank_mode) { col0[u] = J.c_lo; wid[u] = J.c_hi - J.c_lo; }
+        else if (cyc) { col0[u] = 0; wid[u] = n; }
+        else { col0[u] = (long long)n * u / NU; wid[u] = (long long)n * (u + 1) / NU - col0[u]; }
+        if (wid[u] <= 0) {
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe %d is empty (n=%d, stripes=%d)", u, n, NS);
             return SW_EINVAL;
         }
-
-    if ((rc = grow(ctx, ctx->a2, wa * 4))) return rc;
-    if ((rc = grow(ctx, ctx->b2, wb * 4))) return rc;
-    if ((rc = grow(ctx, ctx->misc, 256))) return rc;
-    if (J.match && (rc = grow(ctx, ctx->capbuf, ((size_t)nb * BH + 2) * sizeof(int2)))) return rc;
-    const size_t border_rows = (size_t)nb * BH + 2;
-    const size_t border_flags = (size_t)nb * V.nw + 1;
-    for (int s = 0; s < NS; s++) {
-        const int npad = (int)((wid[s] + W - 1) / W) * W;
-        const int NT = npad / W + (use16 ? 1 : V.skew_tiles);
-        if ((rc = grow(ctx, ctx->rowb[s], (size_t)(NT * W + 2 * W) * sizeof(int2)))) return rc;
-        if ((rc = grow(ctx, ctx->progress[s], (size_t)(nb + 1) * sizeof(int)))) return rc;
-        if (!J.rank_mode && s > 0)
-            if ((rc = grow_recv(ctx, ctx->vrecv[s], border_rows, border_flags))) return rc;
     }
+    auto devof = [&](int d) { return d == 0 ? ctx->device : ctx->peer[d - 1].device; };
+    auto setdev = [&](int d) { return cudaSetDevice(devof(d)); };
+
+    // ---- per-entry buffers: codes (entry 0 encodes; peers on other GPUs get a copy), misc, slots
+    int grid_sum[MAX_DEV] = {};
+    for (int d = 0; d < P; d++)
+        for (int g = 0; g < nseg; g++) grid_sum[d] += seg[g].grid[d];
+    for (int d = 0; d < P; d++) {
+        DevView D = dview(ctx, d);
+        CK(setdev(d));
+        const bool own_codes = d == 0 || devof(d) != ctx->device;
+        if (own_codes) {
+            if ((rc = grow(ctx, *D.a2, wa * 4))) return rc;
+            if ((rc = grow(ctx, *D.b2, wb * 4))) return rc;
+        }
+        if ((rc = grow(ctx, *D.misc, 256))) return rc;
+        if ((rc = grow(ctx, *D.slots, (size_t)grid_sum[d] * sizeof(int4)))) return rc;
+    }
+    CK(setdev(0));
+    if (J.match && (rc = grow(ctx, ctx->capbuf, ((size_t)nb_total * seg[0].BH + 2) * sizeof(int2)))) return rc;
+    const size_t border_rows = (size_t)seg[0].nb * seg[0].BH + 2;
+    const size_t border_flags = (size_t)seg[0].nb * V.nw + 1;
+    int NT[MAX_STRIPES];
+    for (int u = 0; u < NU; u++) {
+        CK(setdev(udev[u]));
+        if (ctx->unit_dev[u] != devof(udev[u])) {
+            // the unit moved to another device (multi-device vs single-device calls)
+            for (DevBuf *b : {&ctx->rowb[u], &ctx->progress[u], &ctx->sp[u]}) {
+                if (b->p) cudaFree(b->p);
+                *b = DevBuf{};
+            }
+            if (ctx->vrecv[u].base) cudaFree(ctx->vrecv[u].base);
+            ctx->vrecv[u] = RecvArea{};
+            ctx->unit_dev[u] = devof(udev[u]);
+        }
+        const int npad = (int)((wid[u] + W - 1) / W) * W;
+        NT[u] = npad / W + (seg[0].use16 ? 1 : V.skew_tiles);
+        if ((rc = grow(ctx, ctx->rowb[u], (size_t)(NT[u] * W + 2 * W) * sizeof(int2)))) return rc;
+        const size_t pbytes = (size_t)(nb_total + 2) * sizeof(unsigned long long);
+        if (ctx->progress[u].cap < pbytes || !ctx->progress[u].p) {
+            if ((rc = grow(ctx, ctx->progress[u], pbytes))) return rc;
+            CK(cudaMemset(ctx->progress[u].p, 0, ctx->progress[u].cap));  // tags of earlier calls are 0 here
+        }
+        if (!J.rank_mode && !cyc && u > 0)
+            if ((rc = grow_recv(ctx, ctx->vrecv[u], border_rows, border_flags))) return rc;
+    }
+    CK(setdev(0));
     if (J.rank_mode) {
         if (J.c_lo > 0 && (!ctx->recv.base || ctx->recv.rows < border_rows || ctx->recv.flags < border_flags)) {
             snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe receive area missing or too small (sw_stripe_export)");
@@ -820,97 +1163,108 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             return SW_EINVAL;
         }
     }
-    const void *fill_fn = use16 ? (J.local ? V.packed_fn : V.packed_global_fn) : (J.local ? V.local_fn : V.global_fn);
-    const size_t fill_smem = use16 ? V.smem16 : V.smem;
-    bool patched = false;
-    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, use16 ? (J.local ? 0 : 3) : J.local ? 1 : 2)) {
-        fill_fn = pf;
-        patched = true;
-    }
-    const int block = V.nw * 32 + (use16 ? V.io_warps : 1) * 32;
-    int blocks_per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, fill_fn, block, fill_smem);
-    if (blocks_per_sm < 1) blocks_per_sm = 1;
-    // every CTA of every stripe must be co-resident (stripes wait on each other)
-    int per_stripe = std::max(1, std::min(nb, blocks_per_sm * ctx->num_sms / NS));
-    if (const char *g = getenv("SWB_GRID")) per_stripe = std::max(1, std::min(per_stripe, atoi(g) / NS));
-    if (ctx->grid_cap > 0) per_stripe = std::max(1, std::min(per_stripe, ctx->grid_cap / NS));
-    const int grid = per_stripe * NS;
-    hck[1] = hnow();
-    if ((rc = grow(ctx, ctx->slots, (size_t)grid * sizeof(int4)))) return rc;
 
-    // special rows: all of them stay resident on the device (180 GB HBM) and
-    // are streamed to the host as bands complete.
+    // ---- special rows (a6): a ring of R slots per unit in HBM, streamed to the
+    // host as bands complete; R = every row when they fit the device budget,
+    // else as many as fit (at least one band's rows), with back-pressure
+    // (sp_admit) and a host store for Stage 2 (the paper's SRA).
     const long long nsp = (J.local && J.k > 0) ? J.m / J.k : 0;
     int ld[MAX_STRIPES];
     long long stride[MAX_STRIPES];
-    size_t row_ints = 0;
-    for (int s = 0; s < NS; s++) {
-        ld[s] = (int)((wid[s] + 31) / 32) * 32;
-        stride[s] = 2ll * ld[s];
-        row_ints += (size_t)stride[s];
+    size_t slot_bytes = 0;  // bytes of one ring slot on the busiest device
+    for (int u = 0; u < NU; u++) {
+        ld[u] = (int)((wid[u] + 31) / 32) * 32;
+        stride[u] = 2ll * ld[u];
+        if (multi) slot_bytes = std::max(slot_bytes, (size_t)stride[u] * sizeof(int));
+        else slot_bytes += (size_t)stride[u] * sizeof(int);
     }
+    long long R = nsp;
+    bool store = false;
     if (nsp > 0) {
-        size_t have = 0;
+        long long rpb = 1;  // most special rows one band can hold
+        for (int g = 0; g < nseg; g++) rpb = std::max<long long>(rpb, (seg[g].BH + J.k - 1) / J.k + 1);
+        const long long R_min = std::min<long long>(nsp, rpb);
         bool grows = false;
-        for (int s = 0; s < NS; s++) {
-            have += ctx->sp[s].cap;
-            grows |= ctx->sp[s].cap < (size_t)nsp * stride[s] * sizeof(int);
+        size_t have = 0;
+        for (int u = 0; u < NU; u++) {
+            have += ctx->sp[u].cap;
+            grows |= ctx->sp[u].cap < (size_t)nsp * stride[u] * sizeof(int);
         }
-        const size_t need = (size_t)nsp * row_ints * sizeof(int);
-        if (grows) {
+        if (ctx->sp_budget > 0 || grows) {
             // only when the buffers must grow: cudaMemGetInfo can take
             // milliseconds (it stalled repeated calls by up to 19 ms)
             size_t freeb = 0, totb = 0;
-            cudaMemGetInfo(&freeb, &totb);
-            if (need > (size_t)(0.8 * (double)(freeb + have))) {
-                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special rows need %zu bytes on the device", need);
-                return SW_ENOMEM;
+            if (grows) cudaMemGetInfo(&freeb, &totb);
+            const double avail = (double)freeb + (double)(multi ? have / std::max(1, P) : have);
+            double budget = grows ? 0.8 * avail : 1e30;
+            if (ctx->sp_budget > 0) budget = std::min(budget, (double)ctx->sp_budget);
+            if ((double)nsp * slot_bytes > budget) {
+                R = std::max<long long>(R_min, (long long)(budget / (double)slot_bytes));
+                if (grows && (double)R * slot_bytes > 0.95 * avail) {
+                    snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special-row ring of %lld rows needs %zu bytes on the device",
+                             R, (size_t)R * slot_bytes);
+                    return SW_ENOMEM;
+                }
             }
+        } else if (ctx->sp_budget == 0) {
+            R = nsp;
         }
-        hck[2] = hnow();
-        for (int s = 0; s < NS; s++) {
-            if ((rc = grow(ctx, ctx->sp[s], (size_t)nsp * stride[s] * sizeof(int)))) return rc;
-            if ((rc = grow_host(ctx, ctx->flags[s], nsp * sizeof(unsigned int), true))) return rc;
-            memset(ctx->flags[s].p, 0, nsp * sizeof(unsigned int));
+        store = (R < nsp || multi) && NS == 1 && !J.rank_mode;
+        for (int u = 0; u < NU; u++) {
+            CK(setdev(udev[u]));
+            if ((rc = grow(ctx, ctx->sp[u], (size_t)R * stride[u] * sizeof(int)))) return rc;
+            if ((rc = grow_host(ctx, ctx->flags[u], nsp * sizeof(unsigned int), true))) return rc;
+            memset(ctx->flags[u].p, 0, nsp * sizeof(unsigned int));
+            if ((rc = grow_host(ctx, ctx->colp[u], (size_t)nb_total * sizeof(unsigned int), true))) return rc;
+            memset(ctx->colp[u].p, 0, (size_t)nb_total * sizeof(unsigned int));
         }
-        for (int s = 0; s < NS; s++) {
-            if ((rc = grow_host(ctx, ctx->colp[s], (size_t)nb * sizeof(unsigned int), true))) return rc;
-            memset(ctx->colp[s].p, 0, (size_t)nb * sizeof(unsigned int));
-        }
+        CK(setdev(0));
         // staging window: every special row when they fit in ~1 GiB of pinned
         // memory (a one-wave matrix completes all its rows together), else as
         // many as fit (at least 2)
         const size_t row_bytes = (size_t)2 * (n + 64) * sizeof(int32_t);
         ctx->nstage = (int)std::max<size_t>(2, std::min<size_t>((size_t)nsp, ((size_t)1 << 30) / row_bytes));
         if ((rc = grow_host(ctx, ctx->stage, row_bytes * ctx->nstage, false))) return rc;
-        while ((int)ctx->ev_row.size() < ctx->nstage) {
-            cudaEvent_t ev;
-            CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-            ctx->ev_row.push_back(ev);
+        for (int d = 0; d < P; d++) {
+            DevView D = dview(ctx, d);
+            CK(setdev(d));
+            while ((int)D.ev_row->size() < ctx->nstage) {
+                cudaEvent_t ev;
+                CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+                D.ev_row->push_back(ev);
+            }
+        }
+        CK(setdev(0));
+        if (store) {
+            ctx->host_rows.resize((size_t)nsp);
+            for (auto &r : ctx->host_rows) r.clear();
         }
     }
+    *(volatile unsigned long long *)ctx->released.p = 0ull;
+    unsigned long long *d_released = nullptr;
 
-    // With a caller stream, every kernel of the call is launched on it (so the
-    // caller's CUDA events bracket them); otherwise on the library stream.
+    // ---- launches.  With a caller stream, every kernel of entry 0 is launched
+    // on it (so the caller's CUDA events bracket them); otherwise on the
+    // library stream.  The tail segment runs on the aux stream, the main
+    // stream waits for it.
+    const double h_alloc = hnow();
     cudaStream_t st = user_stream ? user_stream : ctx->stream;
-    char *misc = (char *)ctx->misc.p;
-    int *d_err = (int *)(misc + 0);
-    int *d_gbest = (int *)(misc + 8);
-    int *d_hit_band = (int *)(misc + 12);
-    unsigned long long *d_hit_key = (unsigned long long *)(misc + 16);
-    unsigned long long *d_replays = (unsigned long long *)(misc + 24);
-    int4 *d_res = (int4 *)(misc + 32);
-    int *d_tickets = (int *)(misc + 64);  // MAX_STRIPES
-
-    hck[3] = hnow();
+    char *misc0 = (char *)ctx->misc.p;
+    int *d_err = (int *)(misc0 + 0);
+    const int pepoch = ++ctx->pepoch;
     CK(cudaEventRecord(ctx->ev[0], st));
-    CK(cudaMemsetAsync(misc, 0, 16, st));
-    CK(cudaMemsetAsync(d_hit_band, 0x7f, 4, st));
-    CK(cudaMemsetAsync(d_hit_key, 0xff, 8, st));
-    CK(cudaMemsetAsync(d_replays, 0, 8, st));
-    CK(cudaMemsetAsync(d_tickets, 0, MAX_STRIPES * sizeof(int), st));
-    for (int s = 0; s < NS; s++) CK(cudaMemsetAsync(ctx->progress[s].p, 0, (size_t)(nb + 1) * sizeof(int), st));
+    for (int d = 0; d < P; d++) {
+        DevView D = dview(ctx, d);
+        cudaStream_t sd = d == 0 ? st : D.stream;
+        CK(setdev(d));
+        char *misc = (char *)D.misc->p;
+        CK(cudaMemsetAsync(misc, 0, 16, sd));
+        CK(cudaMemsetAsync(misc + 12, 0x7f, 4, sd));  // hit_band
+        CK(cudaMemsetAsync(misc + 16, 0xff, 8, sd));  // hit_key
+        CK(cudaMemsetAsync(misc + 24, 0, 8, sd));     // replays
+        CK(cudaMemsetAsync(misc + 64, 0, 2 * MAX_STRIPES * sizeof(int), sd));  // tickets (2 segments)
+    }
+    CK(setdev(0));
     {
         const long long words = wa + wb;
         const int tpb = 256;
@@ -919,215 +1273,341 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         CK(cudaGetLastError());
     }
     CK(cudaEventRecord(ctx->ev[1], st));
-    hck[4] = hnow();
+    const double h_encode = hnow();
 
-    FillArgs a{};
-    a.m = m;
-    a.n = n;
-    a.nb = nb;
-    a.go = J.go;
-    a.ge = J.ge;
-    a.gf = J.go + J.ge;
-    a.one = 1;
-    for (int x = 0; x < 4; x++) {
-        uint32_t w = 0;
-        for (int y = 0; y < 4; y++) {
-            const int v = (x == y ? J.ma : J.mi) + a.gf;
-            w |= (uint32_t)(uint8_t)(int8_t)v << (8 * y);
+    auto fill_args = [&](int d, const Seg &G) -> FillArgs {
+        DevView D = dview(ctx, d);
+        char *misc = (char *)D.misc->p;
+        const bool own_codes = d == 0 || devof(d) != ctx->device;
+        FillArgs a{};
+        a.m = m;
+        a.n = n;
+        a.nb = G.nb;
+        a.row_base = G.row_base;
+        a.band_base = G.band_base;
+        a.cyc_p = P;
+        a.cyc_g = d;
+        a.cross = cross ? 1 : 0;
+        a.go = J.go;
+        a.ge = J.ge;
+        a.gf = J.go + J.ge;
+        a.one = 1;
+        for (int x = 0; x < 4; x++) {
+            uint32_t w = 0;
+            for (int y = 0; y < 4; y++) {
+                const int v = (x == y ? J.ma : J.mi) + a.gf;
+                w |= (uint32_t)(uint8_t)(int8_t)v << (8 * y);
+            }
+            a.prof[x] = w;
         }
-        a.prof[x] = w;
-    }
-    a.A2 = (const uint32_t *)ctx->a2.p;
-    a.B2 = (const uint32_t *)ctx->b2.p;
-    a.err = d_err;
-    a.k = (int)(nsp > 0 ? J.k : 0);
-    a.gbest = d_gbest;
-    a.slots = (int4 *)ctx->slots.p;
-    a.goal = J.goal;
-    a.hit_w = J.hit_w;
-    a.anchor_gap = J.anchor_gap ? 1 : 0;
-    a.match = J.match ? 1 : 0;
-    a.mjc = (int)J.mjc;
-    a.mH = J.mH;
-    a.mF = J.mF;
-    a.hit_key = d_hit_key;
-    a.hit_band = d_hit_band;
-    a.replays = d_replays;
-    a.epoch = J.epoch;
-    a.timeout_ns = ctx->timeout_ns;
-    a.nstripes = NS;
-    a.force_slow = 0;
-    a.dbg = nullptr;
-    if (getenv("SWB_DEBUG_TIMES")) {
-        if ((rc = grow(ctx, ctx->dbg, (size_t)nb * 80 * sizeof(unsigned long long)))) return rc;
-        CK(cudaMemsetAsync(ctx->dbg.p, 0, (size_t)nb * 80 * sizeof(unsigned long long), st));
-        a.dbg = (unsigned long long *)ctx->dbg.p;
-        ctx->dbg_n = nb;
-    }
-    for (int s = 0; s < NS; s++) {
-        StripeArgs &S = a.st[s];
-        S.col0 = (int)col0[s];
-        S.w = (int)wid[s];
-        S.ncols_pad = (int)((wid[s] + W - 1) / W) * W;
-        S.NT = S.ncols_pad / W + (use16 ? 1 : V.skew_tiles);
-        S.rowb = (int2 *)ctx->rowb[s].p;
-        S.progress = (int *)ctx->progress[s].p;
-        S.ticket = d_tickets + s;
-        S.sp = nsp > 0 ? (int *)ctx->sp[s].p : nullptr;
-        S.sp_stride = stride[s];
-        S.sp_ld = ld[s];
-        unsigned int *fd = nullptr;
-        if (nsp > 0) CK(cudaHostGetDevicePointer((void **)&fd, ctx->flags[s].p, 0));
-        S.row_done = fd;
-        unsigned int *cp = nullptr;
-        if (nsp > 0) CK(cudaHostGetDevicePointer((void **)&cp, ctx->colp[s].p, 0));
-        S.colp = cp;
-        if (J.rank_mode) {
-            S.lb = J.c_lo > 0 ? ctx->recv.lb() : nullptr;
-            S.lready = J.c_lo > 0 ? ctx->recv.lready() : nullptr;
-            RecvArea right;
-            right.base = ctx->right_base;
-            right.rows = ctx->right_rows;
-            S.rb = J.c_hi < n ? right.lb() : nullptr;
-            S.rready = J.c_hi < n ? right.lready() : nullptr;
-        } else {
-            S.lb = s > 0 ? ctx->vrecv[s].lb() : nullptr;
-            S.lready = s > 0 ? ctx->vrecv[s].lready() : nullptr;
-            S.rb = s + 1 < NS ? ctx->vrecv[s + 1].lb() : nullptr;
-            S.rready = s + 1 < NS ? ctx->vrecv[s + 1].lready() : nullptr;
-            if (J.match) {  // Stage 2: capture the last column for the band-end matching
-                S.rb = (int2 *)ctx->capbuf.p;
-                S.rready = nullptr;
+        a.A2 = (const uint32_t *)(own_codes ? D.a2->p : ctx->a2.p);
+        a.B2 = (const uint32_t *)(own_codes ? D.b2->p : ctx->b2.p);
+        a.err = d_err;  // entry 0's: an alphabet error stops every entry
+        a.k = (int)(nsp > 0 ? J.k : 0);
+        a.sp_slots = (int)std::max<long long>(1, R);
+        a.sp_released = (R < nsp) ? d_released : nullptr;
+        a.gbest = (int *)(misc + 8);
+        a.goal = J.goal;
+        a.hit_w = J.hit_w;
+        a.anchor_gap = J.anchor_gap ? 1 : 0;
+        a.match = J.match ? 1 : 0;
+        a.mjc = (int)J.mjc;
+        a.mH = J.mH;
+        a.mF = J.mF;
+        a.hit_key = (unsigned long long *)(misc + 16);
+        a.hit_band = (int *)(misc + 12);
+        a.replays = (unsigned long long *)(misc + 24);
+        a.epoch = J.epoch;
+        a.pepoch = pepoch;
+        a.timeout_ns = ctx->timeout_ns;
+        a.nstripes = NS;
+        a.force_slow = 0;
+        a.dbg = nullptr;
+        return a;
+    };
+    auto fill_stripes = [&](FillArgs &a, int d, int segi) -> int {
+        const Seg &G = seg[segi];
+        for (int s = 0; s < NS; s++) {
+            const int u = multi ? d : s;
+            StripeArgs &S = a.st[s];
+            S.col0 = (int)col0[u];
+            S.w = (int)wid[u];
+            S.ncols_pad = (int)((wid[u] + W - 1) / W) * W;
+            S.NT = NT[u];
+            const int un = cyc ? (u + 1) % P : u;  // the unit that runs the next band
+            S.rowb_in = (const int2 *)ctx->rowb[u].p;
+            S.rowb_out = (int2 *)ctx->rowb[un].p;
+            S.prog_in = (const unsigned long long *)ctx->progress[u].p;
+            S.prog_out = (unsigned long long *)ctx->progress[un].p;
+            S.ticket = (int *)((char *)dview(ctx, d).misc->p + 64) + segi * MAX_STRIPES + s;
+            S.sp = nsp > 0 ? (int *)ctx->sp[u].p : nullptr;
+            S.sp_stride = stride[u];
+            S.sp_ld = ld[u];
+            unsigned int *fd = nullptr, *cp = nullptr;
+            if (nsp > 0) {
+                CK(cudaHostGetDevicePointer((void **)&fd, ctx->flags[u].p, 0));
+                CK(cudaHostGetDevicePointer((void **)&cp, ctx->colp[u].p, 0));
+            }
+            S.row_done = fd;
+            S.colp = cp;
+            S.lb = nullptr; S.lready = nullptr; S.rb = nullptr; S.rready = nullptr;
+            if (mstr) {
+                S.lb = u > 0 ? ctx->vrecv[u].lb() : nullptr;
+                S.lready = u > 0 ? ctx->vrecv[u].lready() : nullptr;
+                S.rb = u + 1 < P ? ctx->vrecv[u + 1].lb() : nullptr;
+                S.rready = u + 1 < P ? ctx->vrecv[u + 1].lready() : nullptr;
+            } else if (J.rank_mode) {
+                S.lb = J.c_lo > 0 ? ctx->recv.lb() : nullptr;
+                S.lready = J.c_lo > 0 ? ctx->recv.lready() : nullptr;
+                RecvArea right;
+                right.base = ctx->right_base;
+                right.rows = ctx->right_rows;
+                S.rb = J.c_hi < n ? right.lb() : nullptr;
+                S.rready = J.c_hi < n ? right.lready() : nullptr;
+            } else if (!cyc) {
+                S.lb = s > 0 ? ctx->vrecv[s].lb() : nullptr;
+                S.lready = s > 0 ? ctx->vrecv[s].lready() : nullptr;
+                S.rb = s + 1 < NS ? ctx->vrecv[s + 1].lb() : nullptr;
+                S.rready = s + 1 < NS ? ctx->vrecv[s + 1].lready() : nullptr;
+                if (J.match) {  // Stage 2: capture the last column for the band-end matching
+                    S.rb = (int2 *)ctx->capbuf.p;
+                    S.rready = nullptr;
+                }
             }
         }
-    }
-    {
+        (void)G;
+        return SW_OK;
+    };
+    auto launch = [&](const Seg &G, int d, FillArgs &a, cudaStream_t sd, int slot_off) -> int {
+        a.slots = (int4 *)dview(ctx, d).slots->p + slot_off;
         void *args[] = {&a};
-        const cudaError_t le = cudaLaunchKernel(fill_fn, dim3(grid), dim3(block), args, fill_smem, st);
+        const cudaError_t le = cudaLaunchKernel(G.fn, dim3(G.grid[d]), dim3(G.block), args, G.smem, sd);
         if (le != cudaSuccess) {
             cudaGetLastError();  // not sticky: do not fail the context's next call
             return cuda_fail(ctx, le, "cudaLaunchKernel(fill)");
         }
+        return SW_OK;
+    };
+    for (int d = 0; d < P; d++) {
+        DevView D = dview(ctx, d);
+        cudaStream_t sd = d == 0 ? st : D.stream;
+        CK(setdev(d));
+        if (nsp > 0 && R < nsp) CK(cudaHostGetDevicePointer((void **)&d_released, ctx->released.p, 0));
+        if (d > 0) {
+            CK(cudaStreamWaitEvent(sd, ctx->ev[1], 0));
+            if (devof(d) != ctx->device) {
+                CK(cudaMemcpyPeerAsync(D.a2->p, devof(d), ctx->a2.p, ctx->device, wa * 4, sd));
+                CK(cudaMemcpyPeerAsync(D.b2->p, devof(d), ctx->b2.p, ctx->device, wb * 4, sd));
+            }
+        }
+        FillArgs a = fill_args(d, seg[0]);
+        if ((rc = fill_stripes(a, d, 0))) return rc;
+        if (d == 0 && getenv("SWB_DEBUG_TIMES")) {
+            if ((rc = grow(ctx, ctx->dbg, (size_t)nb_total * 80 * sizeof(unsigned long long)))) return rc;
+            CK(cudaMemsetAsync(ctx->dbg.p, 0, (size_t)nb_total * 80 * sizeof(unsigned long long), st));
+            a.dbg = (unsigned long long *)ctx->dbg.p;
+            ctx->dbg_n = nb_total;
+        }
+        if ((rc = launch(seg[0], d, a, sd, 0))) return rc;
+        if (nseg > 1) {
+            FillArgs at = fill_args(d, seg[1]);
+            if ((rc = fill_stripes(at, d, 1))) return rc;
+            at.dbg = a.dbg;
+            CK(cudaStreamWaitEvent(ctx->aux, ctx->ev[1], 0));
+            if ((rc = launch(seg[1], d, at, ctx->aux, seg[0].grid[d]))) return rc;
+            CK(cudaEventRecord(ctx->ev_aux[0], ctx->aux));
+            CK(cudaStreamWaitEvent(st, ctx->ev_aux[0], 0));
+        }
+        if (d > 0) CK(cudaEventRecord(D.ev[2], sd));
     }
+    CK(setdev(0));
+    for (int d = 1; d < P; d++) CK(cudaStreamWaitEvent(st, dview(ctx, d).ev[2], 0));
     CK(cudaEventRecord(ctx->ev[2], st));
-    sw_reduce_kernel<<<1, 256, 0, st>>>((const int4 *)ctx->slots.p, grid, J.local ? 1 : 0, d_hit_key, J.goal, d_res);
-    CK(cudaGetLastError());
-    CK(cudaMemcpyAsync(ctx->res_h, d_res, sizeof(int4), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(ctx->res_h + 1, d_err, sizeof(int), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(ctx->res_h + 2, d_replays, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    for (int d = 0; d < P; d++) {
+        DevView D = dview(ctx, d);
+        cudaStream_t sd = d == 0 ? st : D.stream;
+        CK(setdev(d));
+        char *misc = (char *)D.misc->p;
+        sw_reduce_kernel<<<1, 256, 0, sd>>>((const int4 *)D.slots->p, grid_sum[d], J.local ? 1 : 0,
+                                            (const unsigned long long *)(misc + 16), J.goal, (int4 *)(misc + 32));
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(D.res_h, misc + 32, sizeof(int4), cudaMemcpyDeviceToHost, sd));
+        CK(cudaMemcpyAsync(D.res_h + 1, d_err, sizeof(int), cudaMemcpyDeviceToHost, sd));
+        CK(cudaMemcpyAsync(D.res_h + 2, misc + 24, sizeof(unsigned long long), cudaMemcpyDeviceToHost, sd));
+        if (d > 0) CK(cudaEventRecord(D.ev[3], sd));
+    }
+    CK(setdev(0));
     CK(cudaEventRecord(ctx->ev[3], st));
 
-    // Stream special rows to the sink in ascending order while the fill runs.
-    // A staged row is copied in column chunks as its band publishes final
-    // columns (colp), and completed once every stripe has published the row
-    // (row_done); the sink then runs on it in row order.
+    // ---- stream special rows to the sink (and the host store) in ascending
+    // order while the fill runs.  A staged row is copied in column chunks as
+    // its band publishes final columns (colp), and completed once every unit
+    // holding a slice of it has published the row (row_done); the sink then
+    // runs on it in row order, and its ring slot is released.
     int sink_rc = 0;
     long long bytes = 0;
     const int64_t nrow_out = J.rank_mode ? wid[0] : n;
-    const int64_t sld = (NS == 1) ? ld[0] : nrow_out + 32;  // H at [0, sld), F at [sld, 2 sld)
+    const int64_t sld = (NU == 1 || cyc) ? ld[0] : nrow_out + 32;  // H at [0, sld), F at [sld, 2 sld)
     const int nstage = nsp > 0 ? ctx->nstage : 0;
     const int64_t CHUNK = 65536;  // columns per partial copy (512 KiB of H + F)
-    std::vector<int64_t> copied((size_t)nstage * NS, 0);
+    std::vector<int64_t> copied((size_t)nstage * NU, 0);
     std::vector<char> sealed(nstage, 0);
-    // SWB_DEBUG_HOST: host-side timeline of the special-row loop (stderr)
+    std::vector<int> sealdev(nstage, 0);
     const bool dbg_host = nsp > 0 && getenv("SWB_DEBUG_HOST") != nullptr;
-    auto hms = [&]() { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - h0).count(); };
-    const double h_launch = hms();
     double h_fill = -1, h_sink_max = 0;
     long long n_copies = 0;
+    // global band of DP row `row` (1-based) and the unit that ran it
+    auto band_of = [&](long long row) -> int {
+        const long long r0 = row - 1;
+        if (nseg > 1 && r0 >= seg[1].row_base) return seg[1].band_base + (int)((r0 - seg[1].row_base) / seg[1].BH);
+        return (int)(r0 / seg[0].BH);
+    };
+    auto unit_lo = [&](long long q) { return cyc ? band_of((q + 1) * J.k) % P : 0; };
+    auto unit_hi = [&](long long q) { return cyc ? unit_lo(q) + 1 : NU; };
     auto row_ready = [&](long long q) -> bool {
-        for (int s = 0; s < NS; s++)
-            if (((volatile unsigned int *)ctx->flags[s].p)[q] == 0) return false;
+        for (int u = unit_lo(q); u < unit_hi(q); u++)
+            if (((volatile unsigned int *)ctx->flags[u].p)[q] == 0) return false;
         return true;
     };
-    // copy what is final of staged row q; true when the row has been sealed
+    auto release_all = [&]() { *(volatile unsigned long long *)ctx->released.p = ~0ull >> 1; };
+    auto fill_running = [&]() -> cudaError_t {
+        for (int d = P - 1; d >= 0; d--) {
+            const cudaError_t e = cudaEventQuery(dview(ctx, d).ev[d == 0 ? 2 : 2]);
+            if (e != cudaSuccess) return e;
+        }
+        return cudaSuccess;
+    };
+    // copy what is final of staged row q
     auto pump = [&](long long q, bool &moved) -> int {
         const int slot = (int)(q % nstage);
         if (sealed[slot]) return SW_OK;
         const bool ready = row_ready(q);
-        const int band = (int)(((q + 1) * J.k - 1) / BH);
+        const int band = band_of((q + 1) * J.k);
         bool all = true;
         int32_t *dst = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
-        for (int s = 0; s < NS; s++) {
-            int64_t &c = copied[(size_t)slot * NS + s];
-            int64_t avail = wid[s];
-            if (!ready) avail = std::min<int64_t>(avail, ((volatile unsigned int *)ctx->colp[s].p)[band]);
+        for (int u = unit_lo(q); u < unit_hi(q); u++) {
+            int64_t &c = copied[(size_t)slot * NU + u];
+            int64_t avail = wid[u];
+            if (!ready) avail = std::min<int64_t>(avail, ((volatile unsigned int *)ctx->colp[u].p)[band]);
             if (avail > c && (ready || avail - c >= CHUNK)) {
-                const int32_t *src = (const int32_t *)ctx->sp[s].p + q * stride[s] + c;
-                const int64_t off = (NS == 1 || J.rank_mode) ? 0 : col0[s];
-                CK(cudaMemcpy2DAsync(dst + off + c, (size_t)sld * 4, src, (size_t)ld[s] * 4, (size_t)(avail - c) * 4, 2,
-                                     cudaMemcpyDeviceToHost, ctx->side));
+                const int32_t *src = (const int32_t *)ctx->sp[u].p + (q % R) * stride[u] + c;
+                const int64_t off = (NU == 1 || J.rank_mode || cyc) ? 0 : col0[u];
+                DevView D = dview(ctx, udev[u]);
+                CK(setdev(udev[u]));
+                CK(cudaMemcpy2DAsync(dst + off + c, (size_t)sld * 4, src, (size_t)ld[u] * 4, (size_t)(avail - c) * 4, 2,
+                                     cudaMemcpyDeviceToHost, D.side));
                 n_copies++;
                 c = avail;
                 moved = true;
             }
-            if (c < wid[s]) all = false;
+            if (c < wid[u]) all = false;
         }
         if (ready && all) {
-            CK(cudaEventRecord(ctx->ev_row[slot], ctx->side));
+            const int d = udev[unit_lo(q)];
+            DevView D = dview(ctx, d);
+            CK(setdev(d));
+            CK(cudaEventRecord((*D.ev_row)[slot], D.side));
             sealed[slot] = 1;
+            sealdev[slot] = d;
             moved = true;
         }
         return SW_OK;
     };
-    long long done = J.sink ? 0 : nsp;  // no sink (sw_align): the rows stay in HBM only
+    // on an error in this loop the kernels may wait on the ring: release it
+    // and let them finish before returning
+    auto bail = [&](int code) -> int {
+        release_all();
+        for (int d = 0; d < P; d++) {
+            setdev(d);
+            cudaStreamSynchronize(d == 0 ? st : dview(ctx, d).stream);
+            cudaStreamSynchronize(dview(ctx, d).side);
+        }
+        setdev(0);
+        return code;
+    };
+    long long done = (J.sink || store) ? 0 : nsp;  // no sink and resident rows (sw_align): nothing to copy
     while (done < nsp) {
         bool progress = false;
-        if (dbg_host && h_fill < 0 && cudaEventQuery(ctx->ev[2]) == cudaSuccess) h_fill = hms();
-        if (!sink_rc) {
-            const long long hi = std::min<long long>(nsp, done + nstage);
-            for (long long q = done; q < hi; q++)
-                if ((rc = pump(q, progress))) return rc;
-        }
+        if (dbg_host && h_fill < 0 && fill_running() == cudaSuccess) h_fill = hnow();
+        const long long hi = std::min<long long>(nsp, done + nstage);
+        for (long long q = done; q < hi; q++)
+            if ((rc = pump(q, progress))) return bail(rc);
         const int slot = (int)(done % nstage);
-        if (sink_rc || sealed[slot]) {
-            const cudaError_t qe = sink_rc ? cudaSuccess : cudaEventQuery(ctx->ev_row[slot]);
+        if (sealed[slot]) {
+            setdev(sealdev[slot]);
+            const cudaError_t qe = cudaEventQuery((*dview(ctx, sealdev[slot]).ev_row)[slot]);
             if (qe == cudaSuccess) {
-                if (!sink_rc) {
-                    bytes += 8ll * nrow_out;
-                    int32_t *row = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
-                    const double t0 = dbg_host ? hms() : 0;
-                    if (J.sink && J.sink(J.user, (done + 1) * J.k, row, row + sld, nrow_out)) sink_rc = SW_EABORTED;
-                    if (dbg_host) h_sink_max = std::max(h_sink_max, hms() - t0);
+                bytes += 8ll * nrow_out;
+                int32_t *row = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
+                if (store) {
+                    std::vector<int32_t> &hr = ctx->host_rows[(size_t)done];
+                    try {
+                        hr.resize((size_t)2 * n);
+                        memcpy(hr.data(), row, (size_t)n * 4);
+                        memcpy(hr.data() + n, row + sld, (size_t)n * 4);
+                    } catch (...) {
+                        store = false;  // no host memory for the SRA: Stage 2 will refuse
+                        ctx->host_rows.clear();
+                    }
                 }
+                const double t0 = dbg_host ? hnow() : 0;
+                if (J.sink && J.sink(J.user, (done + 1) * J.k, row, row + sld, nrow_out)) sink_rc = SW_EABORTED;
+                if (dbg_host) h_sink_max = std::max(h_sink_max, hnow() - t0);
                 sealed[slot] = 0;
-                for (int s = 0; s < NS; s++) copied[(size_t)slot * NS + s] = 0;
+                for (int u = 0; u < NU; u++) copied[(size_t)slot * NU + u] = 0;
                 done++;
+                // the row's device slot is free: the ring's back-pressure counter
+                *(volatile unsigned long long *)ctx->released.p = (unsigned long long)done;
                 progress = true;
+                if (sink_rc) break;
             } else if (qe != cudaErrorNotReady) {
-                return cuda_fail(ctx, qe, "special-row copy");
+                return bail(cuda_fail(ctx, qe, "special-row copy"));
             }
         }
         if (!progress) {
             // nothing ready: make sure the fill is still running
-            const cudaError_t fe = cudaEventQuery(ctx->ev[2]);
+            const cudaError_t fe = fill_running();
             if (fe == cudaSuccess && !sealed[slot] && !row_ready(done)) {
-                CK(cudaStreamSynchronize(st));
+                bail(0);
                 if (ctx->res_h[1].x == 1) return SW_EALPHABET;
                 snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", done,
                          ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
                 return SW_ECUDA;
             } else if (fe != cudaSuccess && fe != cudaErrorNotReady) {
-                return cuda_fail(ctx, fe, "fill kernel");
+                return bail(cuda_fail(ctx, fe, "fill kernel"));
             }
             std::this_thread::yield();
         }
     }
     if (dbg_host)
-        fprintf(stderr, "[swb host] rows %lld copies %lld launched %.2f ms fill_seen %.2f ms loop_end %.2f ms max_sink %.3f ms nstage %d\n",
-                nsp, n_copies, h_launch, h_fill, hms(), h_sink_max, nstage);
-    if (sink_rc) CK(cudaStreamSynchronize(ctx->side));  // no copy may land in a reused staging slot later
-    CK(cudaStreamSynchronize(st));
+        fprintf(stderr, "[swb host] rows %lld copies %lld ring %lld fill_seen %.2f ms loop_end %.2f ms max_sink %.3f ms nstage %d\n",
+                nsp, n_copies, R, h_fill, hnow(), h_sink_max, nstage);
+    if (sink_rc) {
+        bail(0);  // the kernels finish writing into released slots; no copy may land in a reused staging slot later
+        return sink_rc;
+    }
+    for (int d = P - 1; d >= 0; d--) {
+        CK(setdev(d));
+        CK(cudaStreamSynchronize(d == 0 ? st : dview(ctx, d).stream));
+    }
+    CK(setdev(0));
     if (dbg_host)
-        fprintf(stderr, "[swb host] synced %.2f ms; pre-launch: variant %.2f grid %.2f meminfo %.2f staging %.2f encode %.2f\n", hms(),
-                hck[0], hck[1], hck[2], hck[3], hck[4]);
+        fprintf(stderr, "[swb host] synced %.2f ms; pre-launch: choose %.2f alloc %.2f encode %.2f\n", hnow(), h_choose,
+                h_alloc, h_encode);
     if (ctx->res_h[1].x == 1) return SW_EALPHABET;
     if (ctx->res_h[1].x == 2) {
-        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "fill kernel: border wait timeout (a neighbour stripe did not progress)");
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "fill kernel: wait timeout (a neighbour stripe, entry or the special-row ring did not progress)");
         return SW_ECUDA;
     }
-    if (sink_rc) return sink_rc;
-    *res = ctx->res_h[0];
+    // combine the entries' bests under the total order (reading S4)
+    int4 r = ctx->res_h[0];
+    long long reps = (long long)*(unsigned long long *)(ctx->res_h + 2);
+    for (int d = 1; d < P; d++) {
+        const int4 v = dview(ctx, d).res_h[0];
+        reps += (long long)*(unsigned long long *)(dview(ctx, d).res_h + 2);
+        if (J.local && v.x > 0 && (v.x > r.x || (v.x == r.x && (v.y < r.y || (v.y == r.y && v.z < r.z))))) r = v;
+    }
+    *res = r;
 
     float t01 = 0, t12 = 0, t23 = 0;
     cudaEventElapsedTime(&t01, ctx->ev[0], ctx->ev[1]);
@@ -1136,22 +1616,30 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     ctx->stats.encode_ms += t01;
     ctx->stats.fill_ms += t12;
     ctx->stats.reduce_ms += t23;
-    ctx->stats.kernel_launches += 3;
-    ctx->stats.replays += (long long)*(unsigned long long *)(ctx->res_h + 2);
+    ctx->stats.kernel_launches += 1 + (long long)P * (nseg + 1);
+    ctx->stats.replays += reps;
     ctx->stats.special_rows += nsp;
     ctx->stats.special_bytes_d2h += bytes;
-    ctx->stats.alpha = use16 ? -V.alpha : V.alpha;  // negative: packed 16x2 kernel
-    ctx->stats.patched = patched ? 1 : 0;
+    ctx->stats.alpha = seg[0].use16 ? -V.alpha : V.alpha;  // negative: packed 16x2 kernel
+    ctx->stats.patched = seg[0].patched ? 1 : 0;
     ctx->stats.warps = V.nw;
     ctx->stats.width = W;
-    ctx->stats.grid = grid;
+    ctx->stats.grid = seg[0].grid[0];
+    ctx->stats.devices = P;
+    ctx->stats.sp_slots = (int32_t)R;
+    ctx->stats.tail_alpha = nseg > 1 ? -seg[1].V->alpha : 0;
+    ctx->stats.tail_warps = nseg > 1 ? seg[1].V->nw : 0;
+    ctx->stats.tail_grid = nseg > 1 ? seg[1].grid[0] : 0;
+    ctx->stats.tail_rows = nseg > 1 ? m - seg[1].row_base : 0;
     if (J.local) {
-        // Stage 2 can match against these rows while they stay resident
-        S1Rows &R = ctx->s1;
-        R.valid = NS == 1 && !J.rank_mode;
-        R.m = J.m; R.n = J.n; R.k = J.k;
-        R.ma = J.ma; R.mi = J.mi; R.go = J.go; R.ge = J.ge;
-        R.ld = ld[0]; R.stride = stride[0];
+        // Stage 2 matches against these rows: resident in the ring, or in the host store
+        S1Rows &S1 = ctx->s1;
+        S1.resident = R >= nsp && !multi;
+        S1.stored = store && !S1.resident;
+        S1.valid = NS == 1 && !J.rank_mode && (S1.resident || S1.stored || nsp == 0);
+        S1.m = J.m; S1.n = J.n; S1.k = J.k;
+        S1.ma = J.ma; S1.mi = J.mi; S1.go = J.go; S1.ge = J.ge;
+        S1.ld = ld[0]; S1.stride = stride[0];
     }
     return SW_OK;
 }
@@ -1304,6 +1792,26 @@ extern "C" int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t 
     return SW_OK;
 }
 
+extern "C" int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t mismatch, int32_t gap_open,
+                       int32_t gap_ext, int64_t special_row_interval, int32_t *alpha, int32_t *warps)
+{
+    if (!ctx || !alpha || !warps || m < 0 || n < 0 || special_row_interval < 0) return SW_EINVAL;
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    Job J{};
+    J.m = m; J.n = n;
+    J.ma = match; J.mi = mismatch; J.go = gap_open; J.ge = gap_ext;
+    J.k = special_row_interval;
+    J.local = true;
+    J.rank_mode = true;
+    bool use16 = false;
+    const Variant &V = choose_variant(ctx, J, &use16);
+    *alpha = use16 ? -V.alpha : V.alpha;
+    *warps = V.nw;
+    return SW_OK;
+}
+
 extern "C" int sw_align_stage1_stripe(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
                                       int64_t c_lo, int64_t c_hi, int32_t epoch, int32_t match, int32_t mismatch,
                                       int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
@@ -1311,6 +1819,12 @@ extern "C" int sw_align_stage1_stripe(sw_ctx *ctx, const char *dseqA, int64_t m,
 {
     if (!valid_common(ctx, m, n, special_row_interval, sink, out)) return SW_EINVAL;
     if (!dseqA || !dseqB || m <= 0 || c_lo < 0 || c_hi > n || c_hi <= c_lo || epoch <= 0) return SW_EINVAL;
+    if (epoch <= ctx->stripe_epoch) {
+        // the receive area's flags may hold any epoch up to stripe_epoch (equality test):
+        // a repeated epoch would read stale borders (sw_stripe_epoch)
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe epoch %d not above this context's %d", epoch, ctx->stripe_epoch);
+        return SW_EINVAL;
+    }
     int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
     if (rc) return rc;
     if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
@@ -1325,6 +1839,7 @@ extern "C" int sw_align_stage1_stripe(sw_ctx *ctx, const char *dseqA, int64_t m,
     J.c_lo = c_lo;
     J.c_hi = c_hi;
     J.epoch = epoch;
+    ctx->stripe_epoch = epoch;
     int4 r;
     rc = run_job(ctx, J, (cudaStream_t)stream, &r);
     if (rc) return rc;
@@ -1461,11 +1976,19 @@ static int stage2_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const 
     }
     cudaStream_t st = us ? us : ctx->stream;
     const int32_t *sp = (const int32_t *)ctx->sp[0].p;
-    // H, F of special row r at column j (row 0 and column 0: H = 0, F = -inf)
+    // H, F of special row r at column j (row 0 and column 0: H = 0, F = -inf):
+    // from the device ring when every row stayed resident, else from the host
+    // store (the SRA)
     auto fetch = [&](int64_t r, int64_t j, long long *h, long long *f) -> int {
         *h = 0;
         *f = NEG;
         if (r == 0 || j == 0) return SW_OK;
+        if (!R.resident) {
+            const std::vector<int32_t> &hr = ctx->host_rows[(size_t)(r / k - 1)];
+            *h = hr[(size_t)(j - 1)];
+            *f = hr[(size_t)(n + j - 1)];
+            return SW_OK;
+        }
         const int32_t *row = sp + (r / k - 1) * R.stride;
         CK(cudaMemcpyAsync(ctx->res_h + 3, row + j - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
         CK(cudaMemcpyAsync((int32_t *)(ctx->res_h + 3) + 1, row + R.ld + j - 1, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
@@ -1506,8 +2029,17 @@ static int stage2_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const 
             J.anchor_gap = C.type == 2;
             J.match = true;
             J.mjc = C.j;
-            J.mH = r > 0 ? sp + (r / k - 1) * R.stride : nullptr;
-            J.mF = r > 0 ? J.mH + R.ld : nullptr;
+            if (r > 0 && R.resident) {
+                J.mH = sp + (r / k - 1) * R.stride;
+                J.mF = J.mH + R.ld;
+            } else if (r > 0) {
+                // special row r from the host store into HBM for the matching
+                if ((rc = grow(ctx, ctx->s2row, (size_t)2 * n * sizeof(int32_t)))) return rc;
+                CK(cudaMemcpyAsync(ctx->s2row.p, ctx->host_rows[(size_t)(r / k - 1)].data(), (size_t)2 * n * sizeof(int32_t),
+                                   cudaMemcpyHostToDevice, st));
+                J.mH = (const int *)ctx->s2row.p;
+                J.mF = J.mH + n;
+            }
             int4 res;
             const auto tj = std::chrono::steady_clock::now();
             const double f0 = ctx->stats.fill_ms;

@@ -46,20 +46,34 @@ constexpr int MAX_STRIPES = 8;
 
 // One column stripe [col0, col0 + w) of the matrix.  A launch
 // runs nstripes stripes (CTA -> stripe = blockIdx.x % nstripes): 1 per GPU in
-// the multi-GPU pipeline, several "virtual" stripes on one GPU for testing.
+// the multi-GPU column-stripe pipeline, several "virtual" stripes on one GPU
+// for testing.
+//
+// Band addressing: a launch runs the bands b = t * cyc_p +
+// cyc_g (t = 0, 1, ... its ticket) of one SEGMENT of rows: b < nb, first DP
+// row row_base + b * BH (0-based), global band number G = band_base + b.
+// Band G reads its top border from rowb_in gated by prog_in[G] and drains its
+// bottom row into rowb_out, publishing prog_out[G + 1].  One GPU, one
+// segment: rowb_in == rowb_out (in place) and prog_in == prog_out.  Band-cyclic
+// multi-GPU: rowb_out / prog_out are the NEXT GPU's rowb_in / prog_in (peer
+// memory over NVLink).  A tail segment (a second launch with a smaller band
+// height for the last partial wave) continues the same arrays.  Progress words
+// are epoch-tagged, (epoch << 32) | columns, so they never need re-zeroing.
 struct StripeArgs {
     int col0;            // first global 0-based column
     int w;               // real columns of the stripe
     int ncols_pad;       // w rounded up to a multiple of W
     int NT;              // tiles each warp runs per band = ncols_pad / W + ceil(lane skew / W)
-    int2 *rowb;          // row border: (t, F) per local column, >= NT*W + W entries
-    int *progress;       // per band: number of leading columns of its bottom row published
+    const int2 *rowb_in; // row border read by this launch's bands: (t, F) per local column, >= NT*W + W entries
+    int2 *rowb_out;      // row border written by the drain (== rowb_in on one GPU)
+    const unsigned long long *prog_in;  // [G]: columns of band G-1's bottom row published (epoch-tagged)
+    unsigned long long *prog_out;       // [G + 1] written by band G
     int *ticket;         // band ticket of this stripe
-    int *sp;             // special rows (this stripe's slice): slot q at sp + q*sp_stride: H, then F at + sp_ld
+    int *sp;             // special-row ring (this stripe's slice): row q at slot q % sp_slots: H, then F at + sp_ld
     long long sp_stride;
     int sp_ld;
     unsigned int *row_done;  // mapped host flags, one per special row
-    unsigned int *colp;  // mapped host words, one per band: leading columns of the band's special rows that are final
+    unsigned int *colp;  // mapped host words, one per global band: leading columns of the band's special rows that are final
     const int2 *lb;      // left border (t, E) per DP row 0..m at column col0 - 1 (null: column-0 boundary)
     const int *lready;   // per (band, warp) epoch flags guarding lb
     int2 *rb;            // right neighbour's lb (null: last stripe); a peer-GPU pointer across GPUs
@@ -69,7 +83,13 @@ struct StripeArgs {
 struct FillArgs {
     int m;               // rows of S0
     int n;               // columns of S1 (all stripes)
-    int nb;              // number of bands
+    int nb;              // bands of this launch's segment (band b covers rows row_base + b BH + 1 ..)
+    int row_base;        // 0-based first row of the segment (0 unless a tail segment)
+    int band_base;       // global band number of the segment's band 0
+    int cyc_p, cyc_g;    // band-cyclic multi-GPU: this GPU runs bands b = t * cyc_p + cyc_g (1, 0 on one GPU)
+    int cross;           // 1: the row border / progress go to another GPU (system-scope release)
+    int sp_slots;        // special-row ring slots R (>= the rows of one band)
+    const unsigned long long *sp_released;  // mapped host counter: rows 0 .. value-1 have left the ring
     int go, ge, gf;      // G_open, G_ext, G_first = go + ge
     int one;             // always 1 (see imad())
     uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
@@ -88,7 +108,8 @@ struct FillArgs {
     unsigned long long *hit_key;  // min over hits of (i' << 32 | j')
     int *hit_band;       // min band containing a hit
     unsigned long long *replays;
-    int epoch;           // value written to the border flags by this call
+    int epoch;           // value written to the column-stripe border flags by this call
+    int pepoch;          // tag of this call's band-progress words (strictly increasing per progress array)
     long long timeout_ns;  // spin-wait watchdog
     int nstripes;
     int force_slow;      // unused
@@ -102,6 +123,8 @@ struct StepInfo {
     int col0;            // global column of local column 0
     int sp_ld;
     long long sp_stride;
+    int *sp_end;         // end of the special-row ring: the slot after the last wraps to the first
+    long long sp_span;   // sp_slots * sp_stride
     int jcap;            // local column whose (t, E) goes to the right neighbour
     int2 *rbrow;         // right-border destination for this lane's first row
     int hw;              // columns eligible for tracking (w, or the Stage-2 start-check width)
@@ -207,11 +230,62 @@ __device__ __forceinline__ void st_release_sys(unsigned int *p, unsigned int v)
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// True when DP rows b*BH+1 .. min((b+1)*BH, m) hold a special row (k > 0).
-__device__ __forceinline__ bool band_has_special(int b, int BH, int m, int k)
+// Epoch-tagged band progress: a word from an earlier call is
+// smaller than every tag of this call, so the arrays are never re-zeroed.
+__device__ __forceinline__ unsigned long long ptag(int epoch, int cols)
+{
+    return ((unsigned long long)(unsigned)epoch << 32) | (unsigned)cols;
+}
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p, int sys)
+{
+    unsigned long long v;
+    if (sys) asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    else asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned long long v, int sys)
+{
+    if (sys) asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+    else asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// Publish `cols` leading columns of band G's bottom row (after its stores are fenced).
+__device__ __forceinline__ void publish_progress(const FillArgs &a, const StripeArgs &S, int G, int cols)
+{
+    if (a.cross) __threadfence_system();
+    st_release_u64(S.prog_out + G + 1, ptag(a.pepoch, cols), a.cross);
+}
+// Ring slot of special row q (0-based: DP row (q + 1) k).
+__device__ __forceinline__ int *sp_row(const FillArgs &a, const StripeArgs &S, long long q)
+{
+    return S.sp + (q % a.sp_slots) * S.sp_stride;
+}
+// Back-pressure of the special-row ring (P:178's bounded SRA): before a band
+// with rows [lo, hi] starts, the rows that used its slots before must have left
+// the device: released >= q_hi - R + 1 (deadlock-free: R >= the rows of one
+// band, and the rows waited for belong to earlier bands).  Thread 0 only.
+__device__ __forceinline__ void sp_admit(const FillArgs &a, long long rowtop, int BH)
+{
+    if (a.k <= 0 || a.sp_released == nullptr) return;
+    const long long hi = min(rowtop + BH, (long long)a.m);
+    const long long q_hi = hi / a.k - 1;
+    if (q_hi < 0 || (q_hi + 1) * a.k <= rowtop) return;  // no special row in the band
+    const unsigned long long need = (unsigned long long)max(0ll, q_hi - a.sp_slots + 1);
+    if (need == 0) return;
+    const unsigned long long t0 = gtimer();
+    while (true) {
+        unsigned long long v;
+        asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(a.sp_released) : "memory");
+        if (v >= need) break;
+        if (gtimer() - t0 > 4ull * (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); break; }
+        __nanosleep(256);
+    }
+}
+
+// True when DP rows rowtop+1 .. min(rowtop+BH, m) hold a special row (k > 0).
+__device__ __forceinline__ bool band_has_special(long long rowtop, int BH, int m, int k)
 {
     if (k <= 0) return false;
-    const long long lo = (long long)b * BH + 1, hi = min((long long)(b + 1) * BH, (long long)m);
+    const long long lo = rowtop + 1, hi = min(rowtop + BH, (long long)m);
     return ((lo + k - 1) / k) * k <= hi;
 }
 
@@ -342,6 +416,7 @@ struct Fill {
                         if (j0 < X.w) { spp[j0] = hA; spp[X.sp_ld + j0] = fuA; }
                         if (j0 + 1 < X.w) { spp[j0 + 1] = hB; spp[X.sp_ld + j0 + 1] = fuB; }
                         spp += X.sp_stride;
+                        if (spp >= X.sp_end) spp -= X.sp_span;
                     }
                 }
                 if (TRACK) {
@@ -404,6 +479,7 @@ struct Fill {
                     if (j0 < X.w) { spp[j0] = hA; spp[X.sp_ld + j0] = fuA; }
                     if (j0 + 1 < X.w) { spp[j0 + 1] = hB; spp[X.sp_ld + j0 + 1] = fuB; }
                     spp += X.sp_stride;
+                        if (spp >= X.sp_end) spp -= X.sp_span;
                 }
             }
             if (CAP) {  // the stripe's last column: hand (t, E) to the right neighbour
@@ -560,21 +636,26 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
     // tiles in which a lane meets the capture column jcap (lane l at step jcap/2 + l)
     const int cap_t0 = (X.jcap >> 1) / STEPS, cap_t1 = ((X.jcap >> 1) + 31) / STEPS;
 
+    X.sp_end = S.sp != nullptr ? S.sp + (long long)a.sp_slots * S.sp_stride : nullptr;
+    X.sp_span = (long long)a.sp_slots * S.sp_stride;
     for (;;) {
         if (threadIdx.x == 0) {
-            int b = atomicAdd(S.ticket, 1);
+            int b = atomicAdd(S.ticket, 1) * a.cyc_p + a.cyc_g;
             if (!LOCAL && b > ld_relaxed(a.hit_band)) b = a.nb;
             if (ld_relaxed(a.err)) b = a.nb;
+            if (b < a.nb) sp_admit(a, a.row_base + (long long)b * BH, BH);
             s_band = b;
             s_abort = 0;
         }
         __syncthreads();
         const int b = s_band;
         if (b >= a.nb) break;
-        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b] = gtimer();
+        const int G = a.band_base + b;         // global band number (progress, colp)
+        const int rowtop = a.row_base + b * BH;  // 0-based first row of the band
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * G] = gtimer();
 
         typename F::Lane L;
-        const int row0 = b * BH + (warp * 32 + lane) * ALPHA;  // 0-based first row of the strip
+        const int row0 = rowtop + (warp * 32 + lane) * ALPHA;  // 0-based first row of the strip
         int *sp_ptr = nullptr;
         uint32_t smask = 0;
         bool warp_sp = false;
@@ -595,14 +676,14 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             if (LOCAL && a.k > 0) {
                 // special rows among DP rows row0+1 .. row0+ALPHA (<= m); the band's
                 // bottom row is written by the I/O warp from its coalesced drain
-                const int bottom = (b + 1) * BH;
+                const int bottom = rowtop + BH;
                 for (int r = 0; r < ALPHA; r++) {
                     const int row = row0 + r + 1;
                     if (row <= a.m && row % a.k == 0 && row != bottom) smask |= 1u << r;
                 }
                 if (smask) {
                     const int first = __ffs(smask) - 1;
-                    sp_ptr = S.sp + (long long)((row0 + first + 1) / a.k - 1) * S.sp_stride;
+                    sp_ptr = sp_row(a, S, (row0 + first + 1) / a.k - 1);
                 }
             }
             warp_sp = __any_sync(0xffffffffu, smask != 0);
@@ -611,20 +692,21 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
 
         auto io_load = [&](int c) {
             const int need = min((c + 1) * W, NT * W - SKEW);
-            if (b > 0) {
+            if (rowtop > 0) {
                 if (lane == 0) {
                     const unsigned long long t0 = gtimer();
                     unsigned long long spins = 0;
-                    while (ld_acquire(S.progress + b - 1) < need) {
+                    const unsigned long long want = ptag(a.pepoch, need);
+                    while (ld_acquire_u64(S.prog_in + G, a.cross) < want) {
                         if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
                         if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                         __nanosleep(64);
                         spins++;
                     }
                     if (a.dbg && S.col0 == 0 && spins) {  // debug: total wait ns, spin loops, waits
-                        a.dbg[80 * b + 5] += gtimer() - t0;
-                        a.dbg[80 * b + 6] += spins;
-                        a.dbg[80 * b + 7] += 1;
+                        a.dbg[80 * G + 5] += gtimer() - t0;
+                        a.dbg[80 * G + 6] += spins;
+                        a.dbg[80 * G + 7] += 1;
                     }
                 }
                 __syncwarp();
@@ -633,7 +715,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = c * W + x;
-                int2 v = (b == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb + col);
+                int2 v = (rowtop == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb_in + col);
                 ring0[col & (RING - 1)] = v;
                 uint32_t code = 4u;
                 if (col < S.w) {
@@ -646,10 +728,10 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
         // special row that is this band's bottom row: written here, coalesced
         int *io_sp = nullptr;
         if (LOCAL && a.k > 0) {
-            const int bottom = (b + 1) * BH;
-            if (bottom <= a.m && bottom % a.k == 0) io_sp = S.sp + (long long)(bottom / a.k - 1) * S.sp_stride;
+            const int bottom = rowtop + BH;
+            if (bottom <= a.m && bottom % a.k == 0) io_sp = sp_row(a, S, bottom / a.k - 1);
         }
-        unsigned int *const colp = (LOCAL && band_has_special(b, BH, a.m, a.k)) ? S.colp : nullptr;
+        unsigned int *const colp = (LOCAL && band_has_special(rowtop, BH, a.m, a.k)) ? S.colp : nullptr;
         auto io_drain = [&](int cd) {
             const int2 *ringN = rings + NW * RING;
 #pragma unroll
@@ -657,7 +739,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                 const int col = cd * W - SKEW + x;
                 if (col >= 0) {
                     const int2 v = ringN[col & (RING - 1)];
-                    __stcg(S.rowb + col, v);
+                    __stcg(S.rowb_out + col, v);
                     if (io_sp != nullptr && col < S.w) {
                         __stcg(io_sp + col, v.x + a.gf);  // H = t + G_first
                         __stcg(io_sp + S.sp_ld + col, v.y);
@@ -667,8 +749,8 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             __threadfence();
             __syncwarp();
             if (lane == 0) {
-                st_release(S.progress + b, cd * W + W - SKEW);
-                publish_cols(colp, b, cd, cd * W + W - SKEW);
+                publish_progress(a, S, G, cd * W + W - SKEW);
+                publish_cols(colp, G, cd, cd * W + W - SKEW);
             }
         };
         // left border of this warp's rows (stripes after the first): wait for the
@@ -695,12 +777,12 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
 
         if (warp == NW) io_load(0);
         __syncthreads();
-        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 1] = gtimer();
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * G + 1] = gtimer();
         const int S_END = NT + LAG * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s <= S_END; ++s) {
             if (a.dbg && threadIdx.x == 0 && S.col0 == 0 && (s == NT / 4 || s == NT / 2 || s == 3 * NT / 4))
-                a.dbg[80 * b + 2 + (s == NT / 2) + 2 * (s == 3 * NT / 4)] = gtimer();
+                a.dbg[80 * G + 2 + (s == NT / 2) + 2 * (s == 3 * NT / 4)] = gtimer();
             if (warp < NW) {
                 const int c = s - LAG * warp;
                 if (c >= 0 && c < NT) {
@@ -754,7 +836,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             __syncthreads();
             if (s_abort) break;
         }
-        if (warp == NW && lane == 0 && !s_abort) st_release(S.progress + b, INT_MAX);
+        if (warp == NW && lane == 0 && !s_abort) publish_progress(a, S, G, INT_MAX);
         if (!LOCAL && a.match && !s_abort) {
             // Stage-2 goal-based matching: the
             // capture tiles left (t, E) of the special row's DP column for
@@ -764,8 +846,8 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
             // tiles stalled each warp on dependent global loads).
             __syncthreads();
             unsigned long long key = ~0ull;
-            const int hi = min((b + 1) * BH, a.m);
-            for (int row = b * BH + 1 + (int)threadIdx.x; row <= hi; row += (int)blockDim.x) {
+            const int hi = min(rowtop + BH, a.m);
+            for (int row = rowtop + 1 + (int)threadIdx.x; row <= hi; row += (int)blockDim.x) {
                 const int2 v = __ldcg(S.rb + row);
                 const int j = a.mjc - row;
                 const long long hs = (a.mH != nullptr && j > 0) ? (long long)__ldg(a.mH + j - 1) : 0ll;
@@ -781,13 +863,13 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                 atomicMin(a.hit_band, b);
             }
         }
-        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 15] = gtimer();
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * G + 15] = gtimer();
         if (LOCAL && a.k > 0) {
             // publish this band's special rows (this stripe's slice) to the host
             __threadfence();
             __syncthreads();
             if (threadIdx.x == 0) {
-                const long long lo = (long long)b * BH + 1, hi = min((long long)(b + 1) * BH, (long long)a.m);
+                const long long lo = (long long)rowtop + 1, hi = min((long long)rowtop + BH, (long long)a.m);
                 long long q = (lo + a.k - 1) / a.k;
                 if (q * a.k <= hi) {
                     __threadfence_system();

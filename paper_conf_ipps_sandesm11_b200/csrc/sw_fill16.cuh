@@ -545,19 +545,22 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
 
     for (;;) {
         if (threadIdx.x == 0) {
-            int b = atomicAdd(S.ticket, 1);
+            int b = atomicAdd(S.ticket, 1) * a.cyc_p + a.cyc_g;
             if (!LOCAL && b > ld_relaxed(a.hit_band)) b = a.nb;
             if (ld_relaxed(a.err)) b = a.nb;
+            if (b < a.nb) sp_admit(a, a.row_base + (long long)b * BH, BH);
             s_band = b;
             s_abort = 0;
         }
         __syncthreads();
         const int b = s_band;
         if (b >= a.nb) break;
-        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b] = gtimer();  // debug: band start
+        const int G = a.band_base + b;           // global band number (progress, colp)
+        const int rowtop = a.row_base + b * BH;  // 0-based first row of the band
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * G] = gtimer();  // debug: band start
 
         typename F::Lane L;
-        const int row0 = b * BH + (warp * 32 + lane) * ALPHA;
+        const int row0 = rowtop + (warp * 32 + lane) * ALPHA;
         int *sp_ptr = nullptr;
         bool warp_sp = false;
         X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
@@ -622,33 +625,34 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             if (a.k > 0) {
                 // special rows are strip-bottom rows (k a multiple of ALPHA): row0 + ALPHA
                 const int row = row0 + ALPHA;
-                if (row <= a.m && row % a.k == 0 && row != (b + 1) * BH)  // band bottom: the I/O warp's drain
-                    sp_ptr = S.sp + (long long)(row / a.k - 1) * S.sp_stride;
+                if (row <= a.m && row % a.k == 0 && row != rowtop + BH)  // band bottom: the I/O warp's drain
+                    sp_ptr = sp_row(a, S, row / a.k - 1);
             }
             warp_sp = __any_sync(0xffffffffu, sp_ptr != nullptr);
         }
 
         auto io_load = [&](int c) {
             const int need = min((c + 1) * W, NT * W - SKEW);
-            if (b > 0) {
+            if (rowtop > 0) {
                 if (lane == 0) {
                     const unsigned long long t0 = gtimer();
                     unsigned long long spins = 0;
-                    while (ld_acquire(S.progress + b - 1) < need) {
+                    const unsigned long long want = ptag(a.pepoch, need);
+                    while (ld_acquire_u64(S.prog_in + G, a.cross) < want) {
                         if (!LOCAL && ld_relaxed(a.hit_band) < b) { s_abort = 1; break; }
                         if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                         __nanosleep(64);
                         spins++;
                     }
                     if (a.dbg && S.col0 == 0 && spins) {  // debug: total wait ns, spin loops, waits
-                        a.dbg[80 * b + 5] += gtimer() - t0;
-                        a.dbg[80 * b + 6] += spins;
-                        a.dbg[80 * b + 7] += 1;
+                        a.dbg[80 * G + 5] += gtimer() - t0;
+                        a.dbg[80 * G + 6] += spins;
+                        a.dbg[80 * G + 7] += 1;
                     }
                     if (a.dbg && S.col0 == 0 && c == 0) {  // debug: tile 0's border wait
-                        a.dbg[80 * b + 2] = gtimer();
-                        a.dbg[80 * b + 3] = (unsigned long long)ld_acquire(S.progress + b - 1);
-                        a.dbg[80 * b + 4] = spins;
+                        a.dbg[80 * G + 2] = gtimer();
+                        a.dbg[80 * G + 3] = ld_acquire_u64(S.prog_in + G, a.cross) & 0xffffffffull;
+                        a.dbg[80 * G + 4] = spins;
                     }
                 }
                 __syncwarp();
@@ -656,17 +660,17 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
 #pragma unroll
             for (int x = lane; x < W; x += 32) {
                 const int col = c * W + x;
-                rings[F::ridx(col)] = (b == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb + col);
+                rings[F::ridx(col)] = (rowtop == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb_in + col);
                 // pad columns: code 0 (harmless, see header)
                 F::put_sel(selr, col, code_at(col), code_at(col - 1));
             }
         };
         int *io_sp = nullptr;
         if (a.k > 0) {
-            const int bottom = (b + 1) * BH;
-            if (bottom <= a.m && bottom % a.k == 0) io_sp = S.sp + (long long)(bottom / a.k - 1) * S.sp_stride;
+            const int bottom = rowtop + BH;
+            if (bottom <= a.m && bottom % a.k == 0) io_sp = sp_row(a, S, bottom / a.k - 1);
         }
-        unsigned int *const colp = band_has_special(b, BH, a.m, a.k) ? S.colp : nullptr;
+        unsigned int *const colp = band_has_special(rowtop, BH, a.m, a.k) ? S.colp : nullptr;
         auto io_drain = [&](int cd) {
             const int2 *ringN = rings + NW * F::RS;
 #pragma unroll
@@ -674,7 +678,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 const int col = cd * W - SKEW + x;
                 if (col >= 0) {
                     const int2 v = ringN[F::ridx(col)];
-                    __stcg(S.rowb + col, v);
+                    __stcg(S.rowb_out + col, v);
                     if (io_sp != nullptr && col < S.w) {
                         __stcg(io_sp + col, v.x + a.gf);  // H = t + G_first
                         __stcg(io_sp + S.sp_ld + col, v.y);
@@ -684,8 +688,8 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             __threadfence();
             __syncwarp();
             if (lane == 0) {
-                st_release(S.progress + b, cd * W + W - SKEW);
-                publish_cols(colp, b, cd, cd * W + W - SKEW);
+                publish_progress(a, S, G, cd * W + W - SKEW);
+                publish_cols(colp, G, cd, cd * W + W - SKEW);
             }
         };
         auto wait_left = [&]() {
@@ -705,9 +709,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         static_assert(!COOP || (W % NW == 0 && W / NW <= 32), "W must split over the warps");
         auto coop_wait = [&](int c) {
             const int need = min((c + 1) * W, NT * W - SKEW);
-            if (b > 0 && lane == 0) {
+            if (rowtop > 0 && lane == 0) {
                 const unsigned long long t0 = gtimer();
-                while (ld_acquire(S.progress + b - 1) < need) {
+                const unsigned long long want = ptag(a.pepoch, need);
+                while (ld_acquire_u64(S.prog_in + G, a.cross) < want) {
                     if (gtimer() - t0 > (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); s_abort = 1; break; }
                     __nanosleep(64);
                 }
@@ -716,7 +721,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         };
         auto coop_fetch = [&](int c, int2 &v, uint32_t &code) {  // issue the loads (results used after compute)
             const int col = c * W + warp * CPW + lane;
-            v = (b == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb + col);
+            v = (rowtop == 0) ? top_boundary<LOCAL>(a, S.col0 + col) : __ldcg(S.rowb_in + col);
             code = code_at(col) | (code_at(col - 1) << 2);
         };
         auto coop_put = [&](int c, int2 v, uint32_t code) {
@@ -728,7 +733,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             const int col = cd * W - SKEW + warp * CPW + lane;
             if (col >= 0) {
                 const int2 v = rings[NW * F::RS + F::ridx(col)];
-                __stcg(S.rowb + col, v);
+                __stcg(S.rowb_out + col, v);
                 if (io_sp != nullptr && col < S.w) {
                     __stcg(io_sp + col, v.x + a.gf);
                     __stcg(io_sp + S.sp_ld + col, v.y);
@@ -827,14 +832,14 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             if constexpr (COOP) {
                 // every warp's drain of tile cdc is stored and fenced: publish it
                 if (threadIdx.x == 0 && cdc >= 0 && !s_abort) {
-                    st_release(S.progress + b, cdc * W + W - SKEW);
-                    publish_cols(colp, b, cdc, cdc * W + W - SKEW);
+                    publish_progress(a, S, G, cdc * W + W - SKEW);
+                    publish_cols(colp, G, cdc, cdc * W + W - SKEW);
                 }
             }
             if (s_abort) break;
         }
-        if (threadIdx.x == (COOP ? 0 : NW * 32) && !s_abort) st_release(S.progress + b, INT_MAX);
-        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * b + 15] = gtimer();  // debug: band end
+        if (threadIdx.x == (COOP ? 0 : NW * 32) && !s_abort) publish_progress(a, S, G, INT_MAX);
+        if (a.dbg && threadIdx.x == 0 && S.col0 == 0) a.dbg[80 * G + 15] = gtimer();  // debug: band end
         if constexpr (!LOCAL) {
             if (a.match && !s_abort) {
                 // Stage-2 goal-based matching, as in the
@@ -844,8 +849,8 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 // E the reverse F.  Once per band, coalesced.
                 __syncthreads();
                 unsigned long long key = ~0ull;
-                const int hi = min((b + 1) * BH, a.m);
-                for (int row = b * BH + 1 + (int)threadIdx.x; row <= hi; row += (int)blockDim.x) {
+                const int hi = min(rowtop + BH, a.m);
+                for (int row = rowtop + 1 + (int)threadIdx.x; row <= hi; row += (int)blockDim.x) {
                     const int2 v = __ldcg(S.rb + row);
                     const int j = a.mjc - row;
                     const long long hs = (a.mH != nullptr && j > 0) ? (long long)__ldg(a.mH + j - 1) : 0ll;
@@ -865,7 +870,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             __threadfence();
             __syncthreads();
             if (threadIdx.x == 0) {
-                const long long lo = (long long)b * BH + 1, hi = min((long long)(b + 1) * BH, (long long)a.m);
+                const long long lo = (long long)rowtop + 1, hi = min((long long)rowtop + BH, (long long)a.m);
                 long long q = (lo + a.k - 1) / a.k;
                 if (q * a.k <= hi) {
                     __threadfence_system();

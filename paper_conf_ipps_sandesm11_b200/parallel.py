@@ -30,16 +30,12 @@ def stripe_bounds(n: int, world: int, rank: int) -> Tuple[int, int]:
 
 
 def combine_best(results: Iterable[Sequence[int]]) -> Tuple[int, int, int]:
-    """Best (score, i, j) under: higher score, then smaller i, then smaller j;
-    (0, 0, 0) when every score is 0 (reading S4)."""
-    best = (0, 0, 0)
-    for s, i, j in results:
-        s, i, j = int(s), int(i), int(j)
-        if s <= 0:
-            continue
-        if s > best[0] or (s == best[0] and (i < best[1] or (i == best[1] and j < best[2]))):
-            best = (s, i, j)
-    return best
+    """Best (score, i, j) under the library's total order (sw_combine_best:
+    higher score, then smaller i, then smaller j; (0, 0, 0) when every score
+    is 0, reading S4).  Marshalling only."""
+    from . import combine_best as _lib_combine
+
+    return _lib_combine(results)
 
 
 def exchange_handles(my_handle: Optional[bytes], rank: int, world: int, group=None) -> Optional[bytes]:
@@ -60,24 +56,34 @@ class StripeGroup:
 
         self.ctx, self.rank, self.world, self.group = ctx, rank, world, group
         self.max_rows = max_rows
-        self.epoch = 0
         my = ctx.stripe_export(max_rows) if rank > 0 else None
         right = exchange_handles(my, rank, world, group)
         ctx.stripe_connect(right, max_rows)
         dist.barrier(group=group)
 
+    def _agree(self, value):
+        import torch.distributed as dist
+
+        vals = [None] * self.world
+        dist.all_gather_object(vals, value, group=self.group)
+        return vals
+
     def align_stage1(self, dA_ptr: int, m: int, dB_ptr: int, n: int, scoring=(1, -3, 3, 2), k: int = 0,
                      sink=None, stream: int = 0):
         """Run this rank's stripe; returns (global best, local best, (c_lo, c_hi)).
         `sink(row, H_slice, F_slice)` receives this stripe's slice of each special row."""
-        import torch.distributed as dist
-
         if m > self.max_rows:
             raise ValueError("m exceeds the receive area")
         c_lo, c_hi = stripe_bounds(n, self.world, self.rank)
-        self.epoch += 1
-        local, _ = self.ctx.align_stage1_stripe(dA_ptr, m, dB_ptr, n, c_lo, c_hi, self.epoch, *scoring, k=k,
+        # the epoch: above every epoch any rank's receive area has seen (the flags
+        # are compared for equality), the same on all ranks
+        plan = self.ctx.plan(m, n, *scoring, k=k)
+        info = self._agree((self.ctx.stripe_epoch(), plan))
+        if len({p for _, p in info}) != 1:
+            raise RuntimeError(f"ranks chose different kernel geometries {[p for _, p in info]}: the band "
+                               f"height must agree (same library build, GPU and overrides)")
+        epoch = 1 + max(e for e, _ in info)
+        local, _ = self.ctx.align_stage1_stripe(dA_ptr, m, dB_ptr, n, c_lo, c_hi, epoch, *scoring, k=k,
                                                 sink=sink, stream=stream)
-        allres = [None] * self.world
-        dist.all_gather_object(allres, local.astuple(), group=self.group)
+        allres = self._agree(local.astuple())
         return combine_best(allres), local.astuple(), (c_lo, c_hi)

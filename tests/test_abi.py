@@ -58,9 +58,31 @@ def test_null_and_bad_args(lib):
 
     h = ctypes.c_void_p()
     assert lib.sw_init(None, 1, ctypes.byref(h)) == SW_EINVAL
-    ids = (ctypes.c_int * 2)(0, 1)
-    assert lib.sw_init(ids, 2, ctypes.byref(h)) == SW_EINVAL  # round 1: one device per context
+    ids = (ctypes.c_int * 8)(0, 0, 0, 0, 0, 0, 0, 0)
+    for bad in (0, 3, 5, 6, 7, 9):  # n_devices in {1, 2, 4, 8}
+        assert lib.sw_init(ids, bad, ctypes.byref(h)) == SW_EINVAL
+    neg = (ctypes.c_int * 2)(0, -1)
+    assert lib.sw_init(neg, 2, ctypes.byref(h)) in (SW_EINVAL, -5)  # -5: no GPU here at all
     lib.sw_shutdown(None)  # no-op
+    assert lib.sw_set_grid(None, 1) == SW_EINVAL
+    assert lib.sw_set_tail(None, 0) == SW_EINVAL
+    assert lib.sw_set_row_budget(None, 0) == SW_EINVAL
+    assert lib.sw_set_multi_gpu(None, 1) == SW_EINVAL
+    assert lib.sw_device_count(None) == 0
+
+
+def test_combine_best_total_order(lib):
+    """sw_combine_best is the (max score, min i, min j) order of reading S4,
+    checked against a brute-force sort of random triples (no GPU needed)."""
+    import random
+
+    from paper_conf_ipps_sandesm11_b200 import combine_best
+
+    rng = random.Random(5)
+    for _ in range(300):
+        res = [(rng.randint(0, 4), rng.randint(0, 6), rng.randint(0, 6)) for _ in range(rng.randint(0, 9))]
+        pos = sorted((r for r in res if r[0] > 0), key=lambda x: (-x[0], x[1], x[2]))
+        assert combine_best(res) == (pos[0] if pos else (0, 0, 0))
 
 
 def test_init_without_gpu_fails_loudly(lib):

@@ -107,6 +107,11 @@ def _rank_main(rank, world, port, A, B, k, q):
         for _ in range(2):  # two alignments: epochs 1 and 2 reuse the border areas
             best, local, bounds = grp.align_stage1(dA.data_ptr(), len(A), dB.data_ptr(), len(B), PAPER, k=k, sink=sink)
             res.append(best)
+        # a second group on the same context: its receive area still
+        # holds the first group's flags; the agreed epoch must be above them
+        grp2 = StripeGroup(ctx, rank, world, max_rows=len(A))
+        best, local, bounds = grp2.align_stage1(dA.data_ptr(), len(A), dB.data_ptr(), len(B), PAPER, k=k, sink=sink)
+        res.append(best)
         q.put((rank, res, bounds, rows))
         ctx.close()
     except Exception as e:  # report instead of hanging the parent
@@ -139,7 +144,7 @@ def test_two_ranks_ipc_one_gpu():
         assert not isinstance(got[r][0], str), got[r][0]
     want, orows = oracle.stage1(_s(A), _s(B), *PAPER, k=k)
     for r in range(world):
-        assert got[r][0] == [want, want]
+        assert got[r][0] == [want, want, want]
     for row, oh, of in orows:
         h = np.concatenate([got[r][2][row][0] for r in range(world)])
         f = np.concatenate([got[r][2][row][1] for r in range(world)])
