@@ -8,12 +8,14 @@ pass to the start cell (a8).  GCUPS = m n / (t 10^9).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl ours|reference]
 
-N > 1 (torchrun, one process per GPU): the column-stripe pipeline (a7): rank g
-owns columns [g n / N, (g+1) n / N) and hands each band's right-edge column to
-rank g+1 by peer stores over NVLink (CUDA IPC); strong scaling (the same
-matrix on N GPUs).  Special-row slices stay with their rank's sink; the
-reverse pass (tiny for C2) runs on rank 0.  SWB_SAME_DEVICE=1 maps every rank
-to cuda:0 with gloo (a functional check of the N > 1 path on one GPU).
+N > 1 (torchrun, one process per GPU): the band-cyclic pipeline (a7, DESIGN.md
+8): rank r runs bands r, r + N, ... and stores each band's bottom row and
+progress into rank (r + 1) mod N's area by peer stores over NVLink (CUDA IPC);
+strong scaling (the same matrix on N GPUs).  Each rank's sink gets the whole
+special rows of its bands; the reverse pass runs on rank 0.  SWB_MULTI=stripes
+selects the column-stripe pipeline instead (rank g owns columns
+[g n / N, (g+1) n / N)).  SWB_SAME_DEVICE=1 maps every rank to cuda:0 with gloo
+(a functional check of the N > 1 path on one GPU).
 
 --impl reference: the CPU oracle (oracle/, single-threaded plain C) timed on a
 bounded row-band sample of the same workload on the host cores.
@@ -265,10 +267,12 @@ def main():
     ctx = Context(dev_index)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     grp = None
+    multi = os.environ.get("SWB_MULTI", "cyclic")
     if world > 1:
-        from paper_conf_ipps_sandesm11_b200.parallel import StripeGroup
+        from paper_conf_ipps_sandesm11_b200.parallel import CyclicGroup, StripeGroup
 
-        grp = StripeGroup(ctx, rank, world, max_rows=m)
+        grp = StripeGroup(ctx, rank, world, max_rows=m) if multi == "stripes" else \
+            CyclicGroup(ctx, rank, world, max_rows=m, max_cols=n)
 
     sink_rows = [0]
 
@@ -282,7 +286,7 @@ def main():
             r, _ = ctx.align_stage1_dev(dA.data_ptr(), m, dB.data_ptr(), n, *SCORING, k=k, sink=sink, stream=sptr)
             best = r.astuple()
         else:
-            best, _, _ = grp.align_stage1(dA.data_ptr(), m, dB.data_ptr(), n, SCORING, k=k, sink=sink, stream=sptr)
+            best = grp.align_stage1(dA.data_ptr(), m, dB.data_ptr(), n, SCORING, k=k, sink=sink, stream=sptr)[0]
         s1 = ctx.stats()
         launches = s1["kernel_launches"]
         start = None
@@ -348,7 +352,7 @@ def main():
             # multi-GPU: copy this step's inputs host -> device, then the stripe call
             dA.copy_(hA, non_blocking=True)
             dB.copy_(hB, non_blocking=True)
-            b, _, _ = grp.align_stage1(dA.data_ptr(), m, dB.data_ptr(), n, SCORING, k=k, sink=sink, stream=sptr)
+            b = grp.align_stage1(dA.data_ptr(), m, dB.data_ptr(), n, SCORING, k=k, sink=sink, stream=sptr)[0]
             st = None
             if rank == 0 and b[0] > 0:
                 st = ctx.reverse_goal(host_view(hA, m), b[1], host_view(hB, n), b[2], b[0], *SCORING).astuple()
@@ -438,7 +442,9 @@ def main():
         "config": {"workload": cfg.name, "m": m, "n": n, "k": k, "scoring": list(SCORING),
                    "step": "encode + Stage-1 fill + special rows to host sink + reverse goal pass",
                    "l2": "flushed between timed steps (256 MiB write)",
-                   "parallelism": "single" if world == 1 else f"column stripes x{world} (NVLink border hand-off)"
+                   "parallelism": "single" if world == 1 else (
+                       f"column stripes x{world} (NVLink border hand-off)" if multi == "stripes" else
+                       f"band-cyclic x{world} (rank r runs bands r, r+{world}, ...; bottom rows over NVLink)")
                    + (" [same device, functional check]" if same_dev else ""),
                    "kernel": {"alpha": abs(s1["alpha"]), "packed16x2": s1["alpha"] < 0, "warps": s1["warps"],
                               "width": s1["width"], "grid": s1["grid"]},

@@ -235,10 +235,10 @@ int64_t sw_band_height(const sw_ctx *ctx);
 /* Kernel selection (testing / tuning).  variant = -1: automatic choice per
  * call; 0..7: a fixed geometry (alpha, warps, tile width) of
  * the int32 kernel (DESIGN.md 4.1 lists them), or of the packed 16x2 kernel when packed = 1 and the call
- * qualifies (local mode, k % alpha == 0, small value window); 8..13: packed-only
- * geometries (alpha 32, or alpha 30 for 13) that fall back to the default int32
+ * qualifies (local mode, k % alpha == 0, small value window); 8..17: packed-only
+ * geometries (alpha 32; 30 for 13; 34, 36, 38, 40 x 8 warps for 14..17) that fall back to the default int32
  * geometry when the call does not qualify.  packed = 0 never uses the packed
- * kernel.  Results are identical for every choice.  SW_EINVAL outside -1..13. */
+ * kernel.  Results are identical for every choice.  SW_EINVAL outside -1..17. */
 int sw_set_kernel(sw_ctx *ctx, int variant, int packed);
 
 /* Immediate patching of the packed kernel (testing / tuning; default on).
@@ -263,7 +263,7 @@ int sw_set_grid(sw_ctx *ctx, int ctas);
  * shorter band height, if the band-pipeline model says it is faster; 0: never;
  * v + 1 (v a packed geometry of sw_set_kernel with a shorter band): always
  * that geometry when the fill has a partial last wave.  Results are identical.
- * SW_EINVAL outside -1 .. 14. */
+ * SW_EINVAL outside -1 .. 18. */
 int sw_set_tail(sw_ctx *ctx, int mode);
 
 /* Device-memory budget of the special-row ring in bytes (testing / tuning;
@@ -299,12 +299,13 @@ int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t max_rows);
  * seen. */
 int32_t sw_stripe_epoch(const sw_ctx *ctx);
 
-/* The kernel geometry the next stripe call with these arguments would run
- * (alpha < 0: the packed kernel; warps per CTA): ranks of one group must agree
- * on it (the per-(band, warp) border flags), which the caller checks before
- * the call. */
+/* The kernel geometry the next rank call with these arguments would run
+ * (alpha < 0: the packed kernel; warps per CTA): world = 0 for a column-stripe
+ * rank (sw_align_stage1_stripe), else the band-cyclic group size
+ * (sw_align_stage1_cyclic).  Ranks of one group must agree on it (band height
+ * and border flags), which the caller checks before the call. */
 int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
-            int64_t special_row_interval, int32_t *alpha, int32_t *warps);
+            int64_t special_row_interval, int32_t world, int32_t *alpha, int32_t *warps);
 
 /* Stage 1 on this rank's stripe: global columns [c_lo, c_hi) of S1 (0-based),
  * all m rows.  dseqA / dseqB are the WHOLE sequences in this device's memory.
@@ -315,6 +316,28 @@ int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t mismatch, 
  * ranks under the same order (score, then smallest i, then smallest j). */
 int sw_align_stage1_stripe(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
                            int64_t c_lo, int64_t c_hi, int32_t epoch,
+                           int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
+                           int64_t special_row_interval, sw_row_sink sink, void *user, void *stream,
+                           sw_result *out);
+
+/* ---- Band-cyclic ranks (one process per GPU) ----
+ * Rank r of `world` runs bands r, r + world, ... of every row; band b reads its
+ * top border (the row border and band b-1's progress) from this rank's
+ * incoming area and stores its bottom row and progress into the next rank's
+ * ((r + 1) mod world) area by peer stores over NVLink.  Each rank's sink gets
+ * the WHOLE special rows of its own bands (ascending); `out` is the rank's
+ * best (score, i, j) -- combine the ranks' with sw_combine_best.
+ *
+ * sw_cyclic_export allocates this rank's incoming area for up to max_rows x
+ * max_cols and writes its 64-byte CUDA IPC handle; sw_cyclic_connect maps the
+ * next rank's.  `epoch` must be the same on every rank of one call and above
+ * sw_cyclic_epoch() of every rank (the areas' progress words are tagged with
+ * it and never re-zeroed), else SW_EINVAL. */
+int sw_cyclic_export(sw_ctx *ctx, int64_t max_rows, int64_t max_cols, void *handle_out);
+int sw_cyclic_connect(sw_ctx *ctx, const void *next_handle, int64_t max_rows, int64_t max_cols);
+int32_t sw_cyclic_epoch(const sw_ctx *ctx);
+int sw_align_stage1_cyclic(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                           int32_t rank, int32_t world, int32_t epoch,
                            int32_t match, int32_t mismatch, int32_t gap_open, int32_t gap_ext,
                            int64_t special_row_interval, sw_row_sink sink, void *user, void *stream,
                            sw_result *out);

@@ -53,6 +53,10 @@ EXPORTED = [
     "sw_combine_best",
     "sw_stripe_epoch",
     "sw_plan",
+    "sw_cyclic_export",
+    "sw_cyclic_connect",
+    "sw_cyclic_epoch",
+    "sw_align_stage1_cyclic",
     "sw_stripe_export",
     "sw_stripe_connect",
     "sw_align_stage1_stripe",
@@ -181,8 +185,16 @@ def load_library(path: str = LIB_PATH):
     lib.sw_combine_best.restype = ctypes.c_int
     lib.sw_stripe_epoch.argtypes = [vp]
     lib.sw_stripe_epoch.restype = i32
-    lib.sw_plan.argtypes = [vp, i64, i64, i32, i32, i32, i32, i64, ctypes.POINTER(i32), ctypes.POINTER(i32)]
+    lib.sw_plan.argtypes = [vp, i64, i64, i32, i32, i32, i32, i64, i32, ctypes.POINTER(i32), ctypes.POINTER(i32)]
     lib.sw_plan.restype = ctypes.c_int
+    lib.sw_cyclic_export.argtypes = [vp, i64, i64, vp]
+    lib.sw_cyclic_export.restype = ctypes.c_int
+    lib.sw_cyclic_connect.argtypes = [vp, vp, i64, i64]
+    lib.sw_cyclic_connect.restype = ctypes.c_int
+    lib.sw_cyclic_epoch.argtypes = [vp]
+    lib.sw_cyclic_epoch.restype = i32
+    lib.sw_align_stage1_cyclic.argtypes = [vp, vp, i64, vp, i64, i32, i32, i32, i32, i32, i32, i32, i64, SINK, vp, vp, R]
+    lib.sw_align_stage1_cyclic.restype = ctypes.c_int
     lib.sw_stripe_export.argtypes = [vp, i64, vp]
     lib.sw_stripe_export.restype = ctypes.c_int
     lib.sw_stripe_connect.argtypes = [vp, vp, i64]
@@ -427,12 +439,38 @@ class Context:
         """Highest epoch this context ran a stripe call with (sw_stripe_epoch)."""
         return int(self._lib.sw_stripe_epoch(self._h))
 
-    def plan(self, m, n, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0):
-        """(alpha, warps) of the geometry the next stripe call would run (alpha < 0: packed)."""
+    def plan(self, m, n, match=1, mismatch=-3, gap_open=3, gap_ext=2, k=0, world=0):
+        """(alpha, warps) of the geometry the next rank call would run (alpha < 0:
+        packed); world 0: a column-stripe rank, else a band-cyclic group of `world`."""
         a, w = ctypes.c_int32(0), ctypes.c_int32(0)
-        self._check(self._lib.sw_plan(self._h, m, n, match, mismatch, gap_open, gap_ext, k, ctypes.byref(a),
+        self._check(self._lib.sw_plan(self._h, m, n, match, mismatch, gap_open, gap_ext, k, world, ctypes.byref(a),
                                       ctypes.byref(w)), "sw_plan")
         return (a.value, w.value)
+
+    def cyclic_epoch(self) -> int:
+        return int(self._lib.sw_cyclic_epoch(self._h))
+
+    def cyclic_export(self, max_rows: int, max_cols: int) -> bytes:
+        """Allocate this rank's incoming band-cyclic area; returns its 64-byte CUDA IPC handle."""
+        buf = ctypes.create_string_buffer(64)
+        self._check(self._lib.sw_cyclic_export(self._h, max_rows, max_cols, buf), "sw_cyclic_export")
+        return buf.raw
+
+    def cyclic_connect(self, next_handle, max_rows: int, max_cols: int):
+        """Map the next rank's band-cyclic area."""
+        h = ctypes.create_string_buffer(bytes(next_handle), 64)
+        self._check(self._lib.sw_cyclic_connect(self._h, h, max_rows, max_cols), "sw_cyclic_connect")
+
+    def align_stage1_cyclic(self, dA_ptr, m, dB_ptr, n, rank, world, epoch, match=1, mismatch=-3, gap_open=3,
+                            gap_ext=2, k=0, sink=None, keep_rows=False, stream: int = 0):
+        """This rank's bands (rank, rank + world, ...) of Stage 1 (device sequences)."""
+        rows = []
+        cb = self._make_sink(sink, keep_rows, rows) if k > 0 else SINK()
+        out = _Result()
+        rc = self._lib.sw_align_stage1_cyclic(self._h, dA_ptr, m, dB_ptr, n, rank, world, epoch, match, mismatch,
+                                              gap_open, gap_ext, k, cb, None, stream or None, ctypes.byref(out))
+        self._check(rc, "sw_align_stage1_cyclic")
+        return Result(out.score, out.i, out.j), rows
 
     def stripe_export(self, max_rows: int) -> bytes:
         """Allocate this rank's left-border receive area; returns its 64-byte CUDA IPC handle."""

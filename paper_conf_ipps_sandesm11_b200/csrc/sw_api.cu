@@ -135,8 +135,8 @@ static Variant make_variant()
     v.packed_name[0] = 0;
     v.packed_global_fn = nullptr;
     v.packed_global_name[0] = 0;
-    if constexpr (ALPHA == 32 || ALPHA == 30) {
-        // packed kernel only (16 or 15 slots per lane); int32 work falls back to the default geometry
+    if constexpr (ALPHA >= 30) {
+        // packed kernel only (15 to 20 slots per lane); int32 work falls back to the default geometry
         constexpr int NS = ALPHA / 2;
         v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, NS, SPLIT>;
         v.io_warps = COOP ? 0 : 1;
@@ -176,7 +176,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 14;
+static constexpr int NVARIANTS = 18;
 static constexpr int NINT32_VARIANTS = 8;
 // Dynamic shared memory the tail launch requests: more than
 // half an SM's 228 KB, so its CTAs take one SM each as the main launch frees them.
@@ -199,6 +199,12 @@ static const Variant &variant_for(int idx)
         make_variant<32, 16, 64, true>(),
         make_variant<32, 4, 64, false, true>(),  // split F chain (latency-bound one-wave fills)
         make_variant<30, 4, 64>(),  // 3840-row bands: one-wave matrices of up to 148 bands (C2: 142)
+        // taller 8-warp bands (8704 .. 10240 rows): fewer, fuller waves when the
+        // band count is just above a multiple of the CTAs (C4 on 1 or 8 GPUs)
+        make_variant<34, 8, 64>(),
+        make_variant<36, 8, 64>(),
+        make_variant<38, 8, 64>(),
+        make_variant<40, 8, 64>(),
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -352,6 +358,12 @@ struct sw_ctx {
     DevBuf s2row;               // Stage 2: one special row uploaded from the host store
     int unit_dev[MAX_STRIPES] = {-1, -1, -1, -1, -1, -1, -1, -1};  // physical device of unit u's rowb / progress / sp / vrecv (-1: none)
     int stripe_epoch = 0;       // highest epoch of a rank-mode stripe call (sw_stripe_epoch)
+    // band-cyclic ranks (sw_cyclic_*): this rank's incoming row border + band
+    // progress (exported over CUDA IPC), and the next rank's (imported)
+    void *cin = nullptr;
+    size_t cin_cols = 0, cin_bands = 0;
+    void *cout = nullptr;
+    size_t cout_cols = 0, cout_bands = 0;
     int vstripes = 1;           // virtual stripes for the single-process calls
     S1Rows s1;                  // special rows resident from the last Stage-1 call
     int packed = 1;             // use the packed 16x2 Stage-1 kernel when its preconditions hold
@@ -585,6 +597,8 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     for (auto &P : ctx->patched)
         if (P.lib) cudaLibraryUnload(P.lib);
     if (ctx->right_base) cudaIpcCloseMemHandle(ctx->right_base);
+    if (ctx->cout) cudaIpcCloseMemHandle(ctx->cout);
+    if (ctx->cin) cudaFree(ctx->cin);
     if (ctx->recv.base) cudaFree(ctx->recv.base);
     if (ctx->stage.p) cudaFreeHost(ctx->stage.p);
     if (ctx->released.p) cudaFreeHost(ctx->released.p);
@@ -757,6 +771,9 @@ struct Job {
     bool rank_mode = false;
     int64_t c_lo = 0, c_hi = 0;
     int epoch = 0;
+    // band-cyclic rank (one process per GPU): this rank runs bands rank, rank + world, ...
+    bool rank_cyc = false;
+    int cyc_world = 1, cyc_rank = 0;
 };
 }  // namespace
 
@@ -781,6 +798,11 @@ static const Candidate kCands[] = {
     {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
     {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
     {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
+    // alpha 34-40 x 8 warps: variant 10's cell rate per SM (36.8 G/s) over the taller band
+    {14, true, 4.49e6 * 32 / 34, 4.49e6 * 32 / 34},
+    {15, true, 4.49e6 * 32 / 36, 4.49e6 * 32 / 36},
+    {16, true, 4.49e6 * 32 / 38, 4.49e6 * 32 / 38},
+    {17, true, 4.49e6 * 32 / 40, 4.49e6 * 32 / 40},
 };
 static constexpr int NCANDS = (int)(sizeof(kCands) / sizeof(kCands[0]));
 // Tail-segment candidates: column speed of one CTA alone on
@@ -968,7 +990,7 @@ static bool distinct_devices(const sw_ctx *ctx)
 }
 
 // Resolve a segment's kernel (patched image when available) and its per-entry grid.
-static int setup_seg(sw_ctx *ctx, const Job &J, Seg &G, int P, int NS, bool tail)
+static int setup_seg(sw_ctx *ctx, const Job &J, Seg &G, int P, int NS, bool tail, int cp, const int *cg)
 {
     const Variant &V = *G.V;
     G.BH = V.alpha * 32 * V.nw;
@@ -989,7 +1011,7 @@ static int setup_seg(sw_ctx *ctx, const Job &J, Seg &G, int P, int NS, bool tail
     for (int d = 0; d < P; d++) {
         // every CTA of every stripe / entry must be co-resident (they wait on each other)
         const int cap = std::max(1, per_sm * ctx->num_sms / (NS * (P > 1 ? ctx->share[d] : 1)));
-        const int bands_d = (G.nb - d + P - 1) / P;  // bands b = t P + d of this entry
+        const int bands_d = (G.nb - cg[d] + cp - 1) / cp;  // bands b = t cp + cg[d] of this entry
         int g = std::max(1, std::min(bands_d, cap));
         if (const char *e = getenv("SWB_GRID")) g = std::max(1, std::min(g, atoi(e) / NS));
         if (ctx->grid_cap > 0) g = std::max(1, std::min(g, ctx->grid_cap / NS));
@@ -1054,26 +1076,31 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     // band-cyclic multi-GPU Stage 1: entry d runs bands d, d + P, ...
     // or column stripes, one per entry (mstr), with the (t, E) border column
     // stored into the next entry's receive area
-    const bool multi = J.local && !J.rank_mode && J.nv == 1 && ctx->ndev > 1;
+    const bool rcyc = J.rank_cyc;
+    const bool multi = J.local && !J.rank_mode && !rcyc && J.nv == 1 && ctx->ndev > 1;
     const bool cyc = multi && ctx->cyclic;
     const bool mstr = multi && !ctx->cyclic;
     const int P = multi ? ctx->ndev : 1;
-    const bool cross = multi && distinct_devices(ctx);
+    const bool cross = (multi && distinct_devices(ctx)) || rcyc;
+    // the band-cyclic step and index of each entry (1, 0: every band)
+    const int cp = cyc ? P : rcyc ? J.cyc_world : 1;
+    int cg[MAX_DEV] = {};
+    for (int d = 0; d < P; d++) cg[d] = cyc ? d : rcyc ? J.cyc_rank : 0;
     const int NS = (J.rank_mode || multi) ? 1 : J.nv;  // column stripes of one launch
     const int NU = multi ? P : NS;                     // units: (entry, stripe) buffer sets
     Seg seg[2];
     int nseg = 1;
-    seg[0].V = &choose_variant(ctx, J, &seg[0].use16, cyc ? P : 1);
+    seg[0].V = &choose_variant(ctx, J, &seg[0].use16, cp);
     const Variant &V = *seg[0].V;
     const int W = V.w;
     const int m = (int)J.m, n = (int)J.n;
     seg[0].BH = V.alpha * 32 * V.nw;
     seg[0].nb = (m + seg[0].BH - 1) / seg[0].BH;
     int rc;
-    if ((rc = setup_seg(ctx, J, seg[0], P, NS, false))) return rc;
+    if ((rc = setup_seg(ctx, J, seg[0], P, NS, false, cp, cg))) return rc;
     // the last partial wave of a multi-wave fill as a second launch with a
     // smaller band height
-    if (!cyc && NS == 1 && !J.rank_mode && J.local && seg[0].use16) {
+    if (cp == 1 && !multi && NS == 1 && !J.rank_mode && J.local && seg[0].use16) {
         int nb1 = 0;
         const Variant *Vt = choose_tail(ctx, J, seg[0], &nb1);
         if (Vt) {
@@ -1084,8 +1111,8 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             seg[1].BH = Vt->alpha * 32 * Vt->nw;
             seg[1].nb = (m - seg[1].row_base + seg[1].BH - 1) / seg[1].BH;
             seg[0].nb = nb1;
-            if ((rc = setup_seg(ctx, J, seg[0], P, NS, false))) return rc;
-            if ((rc = setup_seg(ctx, J, seg[1], P, NS, true))) return rc;
+            if ((rc = setup_seg(ctx, J, seg[0], P, NS, false, cp, cg))) return rc;
+            if ((rc = setup_seg(ctx, J, seg[1], P, NS, true, cp, cg))) return rc;
             nseg = 2;
         }
     }
@@ -1099,7 +1126,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     for (int u = 0; u < NU; u++) {
         udev[u] = multi ? u : 0;
         if (J.rank_mode) { col0[u] = J.c_lo; wid[u] = J.c_hi - J.c_lo; }
-        else if (cyc) { col0[u] = 0; wid[u] = n; }
+        else if (cyc || rcyc) { col0[u] = 0; wid[u] = n; }
         else { col0[u] = (long long)n * u / NU; wid[u] = (long long)n * (u + 1) / NU - col0[u]; }
         if (wid[u] <= 0) {
             snprintf(ctx->errbuf, sizeof(ctx->errbuf), "stripe %d is empty (n=%d, stripes=%d)", u, n, NS);
@@ -1143,6 +1170,16 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         }
         const int npad = (int)((wid[u] + W - 1) / W) * W;
         NT[u] = npad / W + (seg[0].use16 ? 1 : V.skew_tiles);
+        if (rcyc) {
+            // the exported / imported areas hold the row border and the band progress
+            if (!ctx->cin || !ctx->cout || ctx->cin_cols < (size_t)(NT[u] * W + 2 * W) ||
+                ctx->cout_cols < (size_t)(NT[u] * W + 2 * W) || ctx->cin_bands < (size_t)nb_total + 2 ||
+                ctx->cout_bands < (size_t)nb_total + 2) {
+                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "band-cyclic areas missing or too small (sw_cyclic_export / connect)");
+                return SW_EINVAL;
+            }
+            continue;
+        }
         if ((rc = grow(ctx, ctx->rowb[u], (size_t)(NT[u] * W + 2 * W) * sizeof(int2)))) return rc;
         const size_t pbytes = (size_t)(nb_total + 2) * sizeof(unsigned long long);
         if (ctx->progress[u].cap < pbytes || !ctx->progress[u].p) {
@@ -1209,7 +1246,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         } else if (ctx->sp_budget == 0) {
             R = nsp;
         }
-        store = (R < nsp || multi) && NS == 1 && !J.rank_mode;
+        store = (R < nsp || multi) && NS == 1 && !J.rank_mode && !rcyc;
         for (int u = 0; u < NU; u++) {
             CK(setdev(udev[u]));
             if ((rc = grow(ctx, ctx->sp[u], (size_t)R * stride[u] * sizeof(int)))) return rc;
@@ -1251,7 +1288,10 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     cudaStream_t st = user_stream ? user_stream : ctx->stream;
     char *misc0 = (char *)ctx->misc.p;
     int *d_err = (int *)(misc0 + 0);
-    const int pepoch = ++ctx->pepoch;
+    // progress tags: the ranks' agreed epoch (the next rank's area holds tags
+    // of earlier agreed epochs only), else this context's own counter
+    const int pepoch = rcyc ? J.epoch : ++ctx->pepoch;
+    if (rcyc) ctx->pepoch = std::max(ctx->pepoch, J.epoch);
     CK(cudaEventRecord(ctx->ev[0], st));
     for (int d = 0; d < P; d++) {
         DevView D = dview(ctx, d);
@@ -1285,8 +1325,8 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         a.nb = G.nb;
         a.row_base = G.row_base;
         a.band_base = G.band_base;
-        a.cyc_p = P;
-        a.cyc_g = d;
+        a.cyc_p = cp;
+        a.cyc_g = cg[d];
         a.cross = cross ? 1 : 0;
         a.go = J.go;
         a.ge = J.ge;
@@ -1305,7 +1345,8 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         a.err = d_err;  // entry 0's: an alphabet error stops every entry
         a.k = (int)(nsp > 0 ? J.k : 0);
         a.sp_slots = (int)std::max<long long>(1, R);
-        a.sp_released = (R < nsp) ? d_released : nullptr;
+        a.sp_released = (R < nsp && !getenv("SWB_NO_ADMIT")) ? d_released : nullptr;
+        a.admit_ns = getenv("SWB_ADMIT_NS") ? (unsigned)atoi(getenv("SWB_ADMIT_NS")) : 2000u;
         a.gbest = (int *)(misc + 8);
         a.goal = J.goal;
         a.hit_w = J.hit_w;
@@ -1339,6 +1380,12 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
             S.rowb_out = (int2 *)ctx->rowb[un].p;
             S.prog_in = (const unsigned long long *)ctx->progress[u].p;
             S.prog_out = (unsigned long long *)ctx->progress[un].p;
+            if (rcyc) {  // this rank's incoming area, and the next rank's over CUDA IPC / NVLink
+                S.rowb_in = (const int2 *)ctx->cin;
+                S.prog_in = (const unsigned long long *)((const char *)ctx->cin + ctx->cin_cols * sizeof(int2));
+                S.rowb_out = (int2 *)ctx->cout;
+                S.prog_out = (unsigned long long *)((char *)ctx->cout + ctx->cout_cols * sizeof(int2));
+            }
             S.ticket = (int *)((char *)dview(ctx, d).misc->p + 64) + segi * MAX_STRIPES + s;
             S.sp = nsp > 0 ? (int *)ctx->sp[u].p : nullptr;
             S.sp_stride = stride[u];
@@ -1423,21 +1470,29 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
     CK(setdev(0));
     for (int d = 1; d < P; d++) CK(cudaStreamWaitEvent(st, dview(ctx, d).ev[2], 0));
     CK(cudaEventRecord(ctx->ev[2], st));
-    for (int d = 0; d < P; d++) {
-        DevView D = dview(ctx, d);
-        cudaStream_t sd = d == 0 ? st : D.stream;
-        CK(setdev(d));
-        char *misc = (char *)D.misc->p;
-        sw_reduce_kernel<<<1, 256, 0, sd>>>((const int4 *)D.slots->p, grid_sum[d], J.local ? 1 : 0,
-                                            (const unsigned long long *)(misc + 16), J.goal, (int4 *)(misc + 32));
-        CK(cudaGetLastError());
-        CK(cudaMemcpyAsync(D.res_h, misc + 32, sizeof(int4), cudaMemcpyDeviceToHost, sd));
-        CK(cudaMemcpyAsync(D.res_h + 1, d_err, sizeof(int), cudaMemcpyDeviceToHost, sd));
-        CK(cudaMemcpyAsync(D.res_h + 2, misc + 24, sizeof(unsigned long long), cudaMemcpyDeviceToHost, sd));
-        if (d > 0) CK(cudaEventRecord(D.ev[3], sd));
-    }
-    CK(setdev(0));
-    CK(cudaEventRecord(ctx->ev[3], st));
+    auto enqueue_results = [&]() -> int {
+        for (int d = 0; d < P; d++) {
+            DevView D = dview(ctx, d);
+            cudaStream_t sd = d == 0 ? st : D.stream;
+            CK(setdev(d));
+            char *misc = (char *)D.misc->p;
+            sw_reduce_kernel<<<1, 256, 0, sd>>>((const int4 *)D.slots->p, grid_sum[d], J.local ? 1 : 0,
+                                                (const unsigned long long *)(misc + 16), J.goal, (int4 *)(misc + 32));
+            CK(cudaGetLastError());
+            CK(cudaMemcpyAsync(D.res_h, misc + 32, sizeof(int4), cudaMemcpyDeviceToHost, sd));
+            CK(cudaMemcpyAsync(D.res_h + 1, d_err, sizeof(int), cudaMemcpyDeviceToHost, sd));
+            CK(cudaMemcpyAsync(D.res_h + 2, misc + 24, sizeof(unsigned long long), cudaMemcpyDeviceToHost, sd));
+            if (d > 0) CK(cudaEventRecord(D.ev[3], sd));
+        }
+        CK(setdev(0));
+        CK(cudaEventRecord(ctx->ev[3], st));
+        return SW_OK;
+    };
+    // The result copies are enqueued after the special-row loop: a device-to-host
+    // copy queued behind the running fill on its stream held back every other
+    // stream's device-to-host copies until the fill ended (measured: special rows
+    // reached the host only after the fill, and a ring that waits on the host
+    // for its slots never drained; profiles/r02_copy_order.txt).
 
     // ---- stream special rows to the sink (and the host store) in ascending
     // order while the fill runs.  A staged row is copied in column chunks as
@@ -1463,6 +1518,8 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         return (int)(r0 / seg[0].BH);
     };
     auto unit_lo = [&](long long q) { return cyc ? band_of((q + 1) * J.k) % P : 0; };
+    // rows of this process (band-cyclic ranks: only the rows of this rank's bands)
+    auto mine = [&](long long q) { return !rcyc || band_of((q + 1) * J.k) % cp == J.cyc_rank; };
     auto unit_hi = [&](long long q) { return cyc ? unit_lo(q) + 1 : NU; };
     auto row_ready = [&](long long q) -> bool {
         for (int u = unit_lo(q); u < unit_hi(q); u++)
@@ -1477,39 +1534,67 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         }
         return cudaSuccess;
     };
-    // copy what is final of staged row q
-    auto pump = [&](long long q, bool &moved) -> int {
-        const int slot = (int)(q % nstage);
-        if (sealed[slot]) return SW_OK;
-        const bool ready = row_ready(q);
-        const int band = band_of((q + 1) * J.k);
-        bool all = true;
-        int32_t *dst = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
-        for (int u = unit_lo(q); u < unit_hi(q); u++) {
-            int64_t &c = copied[(size_t)slot * NU + u];
-            int64_t avail = wid[u];
-            if (!ready) avail = std::min<int64_t>(avail, ((volatile unsigned int *)ctx->colp[u].p)[band]);
-            if (avail > c && (ready || avail - c >= CHUNK)) {
-                const int32_t *src = (const int32_t *)ctx->sp[u].p + (q % R) * stride[u] + c;
-                const int64_t off = (NU == 1 || J.rank_mode || cyc) ? 0 : col0[u];
-                DevView D = dview(ctx, udev[u]);
-                CK(setdev(udev[u]));
-                CK(cudaMemcpy2DAsync(dst + off + c, (size_t)sld * 4, src, (size_t)ld[u] * 4, (size_t)(avail - c) * 4, 2,
-                                     cudaMemcpyDeviceToHost, D.side));
-                n_copies++;
-                c = avail;
+    // last DP row (1-based, inclusive) of global band G
+    auto band_end = [&](int G) -> long long {
+        long long e = (nseg > 1 && G >= seg[1].band_base)
+                          ? (long long)seg[1].row_base + (long long)(G - seg[1].band_base + 1) * seg[1].BH
+                          : (long long)(G + 1) * seg[0].BH;
+        return std::min<long long>(e, J.m);
+    };
+    // one side stream per row, so that one event seals it: the owning entry's
+    // (band-cyclic), else entry 0's (column slices of other entries are read over the peer mapping)
+    auto copy_dev = [&](long long q) { return cyc ? band_of((q + 1) * J.k) % P : 0; };
+    // copy what is final of the staged rows [q0, q1) of one band (ready: the band has ended)
+    const int copy_mode = getenv("SWB_COPY_MODE") ? atoi(getenv("SWB_COPY_MODE")) : 0;
+    cudaStream_t dbg_stream = nullptr;
+    if (copy_mode == 3) cudaStreamCreateWithFlags(&dbg_stream, cudaStreamNonBlocking);
+    auto pump_band = [&](long long q0, long long q1, int band, bool ready, bool &moved) -> int {
+        const int d = copy_dev(q0);
+        DevView D = dview(ctx, d);
+        if (copy_mode == 2) D.side = ctx->aux;
+        if (copy_mode == 3) D.side = dbg_stream;
+        bool devset = false;
+        int64_t av[MAX_STRIPES];
+        const int ulo = unit_lo(q0), uhi = unit_hi(q0);
+        for (int u = ulo; u < uhi; u++)
+            av[u] = ready ? wid[u] : std::min<int64_t>(wid[u], ((volatile unsigned int *)ctx->colp[u].p)[band]);
+        for (long long q = q0; q < q1; q++) {
+            const int slot = (int)(q % nstage);
+            if (sealed[slot]) continue;
+            bool all = true;
+            int32_t *dst = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
+            for (int u = ulo; u < uhi; u++) {
+                int64_t &c = copied[(size_t)slot * NU + u];
+                if (av[u] > c && (ready || av[u] - c >= CHUNK)) {
+                    if (!devset) {
+                        CK(setdev(d));
+                        devset = true;
+                    }
+                    const int32_t *src = (const int32_t *)ctx->sp[u].p + (q % R) * stride[u] + c;
+                    const int64_t off = (NU == 1 || J.rank_mode || cyc) ? 0 : col0[u];
+                    if (copy_mode == 1) {
+                        CK(cudaMemcpyAsync(dst + off + c, src, (size_t)(av[u] - c) * 4, cudaMemcpyDeviceToHost, D.side));
+                        CK(cudaMemcpyAsync(dst + sld + off + c, src + ld[u], (size_t)(av[u] - c) * 4, cudaMemcpyDeviceToHost, D.side));
+                    } else {
+                        CK(cudaMemcpy2DAsync(dst + off + c, (size_t)sld * 4, src, (size_t)ld[u] * 4, (size_t)(av[u] - c) * 4, 2,
+                                             cudaMemcpyDeviceToHost, D.side));
+                    }
+                    n_copies++;
+                    c = av[u];
+                    moved = true;
+                }
+                if (c < wid[u]) all = false;
+            }
+            if (ready && all) {
+                if (!devset) {
+                    CK(setdev(d));
+                    devset = true;
+                }
+                CK(cudaEventRecord((*D.ev_row)[slot], D.side));
+                sealed[slot] = 1;
+                sealdev[slot] = d;
                 moved = true;
             }
-            if (c < wid[u]) all = false;
-        }
-        if (ready && all) {
-            const int d = udev[unit_lo(q)];
-            DevView D = dview(ctx, d);
-            CK(setdev(d));
-            CK(cudaEventRecord((*D.ev_row)[slot], D.side));
-            sealed[slot] = 1;
-            sealdev[slot] = d;
-            moved = true;
         }
         return SW_OK;
     };
@@ -1525,60 +1610,88 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         setdev(0);
         return code;
     };
+    auto release = [&](long long upto) { *(volatile unsigned long long *)ctx->released.p = (unsigned long long)upto; };
     long long done = (J.sink || store) ? 0 : nsp;  // no sink and resident rows (sw_align): nothing to copy
     while (done < nsp) {
         bool progress = false;
         if (dbg_host && h_fill < 0 && fill_running() == cudaSuccess) h_fill = hnow();
+        // 1) copy what is final of the staged window, one band at a time (two
+        //    mapped-flag reads per band, not per row)
         const long long hi = std::min<long long>(nsp, done + nstage);
-        for (long long q = done; q < hi; q++)
-            if ((rc = pump(q, progress))) return bail(rc);
-        const int slot = (int)(done % nstage);
-        if (sealed[slot]) {
+        for (long long q = done; q < hi;) {
+            const int band = band_of((q + 1) * J.k);
+            const long long q1 = std::min<long long>(hi, std::max<long long>(q + 1, band_end(band) / J.k));
+            if (mine(q) && (rc = pump_band(q, q1, band, row_ready(q), progress))) return bail(rc);
+            q = q1;
+        }
+        // 2) hand every completed row to the sink in order and free its ring slot
+        while (done < nsp) {
+            if (!mine(done)) {  // another rank's row: it never occupies this rank's ring
+                release(++done);
+                progress = true;
+                continue;
+            }
+            const int slot = (int)(done % nstage);
+            if (!sealed[slot]) break;
             setdev(sealdev[slot]);
             const cudaError_t qe = cudaEventQuery((*dview(ctx, sealdev[slot]).ev_row)[slot]);
-            if (qe == cudaSuccess) {
-                bytes += 8ll * nrow_out;
-                int32_t *row = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
-                if (store) {
-                    std::vector<int32_t> &hr = ctx->host_rows[(size_t)done];
-                    try {
-                        hr.resize((size_t)2 * n);
-                        memcpy(hr.data(), row, (size_t)n * 4);
-                        memcpy(hr.data() + n, row + sld, (size_t)n * 4);
-                    } catch (...) {
-                        store = false;  // no host memory for the SRA: Stage 2 will refuse
-                        ctx->host_rows.clear();
-                    }
+            if (qe == cudaErrorNotReady) break;
+            if (qe != cudaSuccess) return bail(cuda_fail(ctx, qe, "special-row copy"));
+            bytes += 8ll * nrow_out;
+            int32_t *row = (int32_t *)ctx->stage.p + (size_t)slot * 2 * sld;
+            if (store) {
+                std::vector<int32_t> &hr = ctx->host_rows[(size_t)done];
+                try {
+                    hr.resize((size_t)2 * n);
+                    memcpy(hr.data(), row, (size_t)n * 4);
+                    memcpy(hr.data() + n, row + sld, (size_t)n * 4);
+                } catch (...) {
+                    store = false;  // no host memory for the SRA: Stage 2 will refuse
+                    ctx->host_rows.clear();
                 }
-                const double t0 = dbg_host ? hnow() : 0;
-                if (J.sink && J.sink(J.user, (done + 1) * J.k, row, row + sld, nrow_out)) sink_rc = SW_EABORTED;
-                if (dbg_host) h_sink_max = std::max(h_sink_max, hnow() - t0);
-                sealed[slot] = 0;
-                for (int u = 0; u < NU; u++) copied[(size_t)slot * NU + u] = 0;
-                done++;
-                // the row's device slot is free: the ring's back-pressure counter
-                *(volatile unsigned long long *)ctx->released.p = (unsigned long long)done;
-                progress = true;
-                if (sink_rc) break;
-            } else if (qe != cudaErrorNotReady) {
-                return bail(cuda_fail(ctx, qe, "special-row copy"));
             }
+            const double t0 = dbg_host ? hnow() : 0;
+            if (dbg_host && (done == 0 || done + 1 == nsp || done % 256 == 0))
+                fprintf(stderr, "[swb host] row %lld to the sink at %.3f ms (fill %s)\n", done, t0,
+                        fill_running() == cudaSuccess ? "done" : "running");
+            if (J.sink && J.sink(J.user, (done + 1) * J.k, row, row + sld, nrow_out)) sink_rc = SW_EABORTED;
+            if (dbg_host) h_sink_max = std::max(h_sink_max, hnow() - t0);
+            sealed[slot] = 0;
+            for (int u = 0; u < NU; u++) copied[(size_t)slot * NU + u] = 0;
+            release(++done);  // the row's ring slot is free: the back-pressure counter
+            progress = true;
+            if (sink_rc) break;
         }
-        if (!progress) {
+        if (sink_rc) break;
+        if (!progress && done < nsp) {
             // nothing ready: make sure the fill is still running
+            const int slot = (int)(done % nstage);
             const cudaError_t fe = fill_running();
             if (fe == cudaSuccess && !sealed[slot] && !row_ready(done)) {
                 bail(0);
                 if (ctx->res_h[1].x == 1) return SW_EALPHABET;
-                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld not published%s", done,
-                         ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
+                snprintf(ctx->errbuf, sizeof(ctx->errbuf), "special row %lld (row %lld) not published%s", done,
+                         (done + 1) * J.k, ctx->res_h[1].x == 2 ? " (kernel wait timeout)" : "");
                 return SW_ECUDA;
             } else if (fe != cudaSuccess && fe != cudaErrorNotReady) {
                 return bail(cuda_fail(ctx, fe, "fill kernel"));
             }
+            if (dbg_host) {
+                static double last = 0;
+                if (hnow() - last > 1000.0) {
+                    last = hnow();
+                    fprintf(stderr, "[swb host] %.0f ms: done %lld/%lld released %llu sealed %d ready %d band %d colp %u copies %lld "
+                            "evq %d sideq %d stq %d fill %d err %d\n", last, done,
+                            nsp, *(volatile unsigned long long *)ctx->released.p, (int)sealed[slot], (int)row_ready(done),
+                            band_of((done + 1) * J.k), ((volatile unsigned int *)ctx->colp[unit_lo(done)].p)[band_of((done + 1) * J.k)],
+                            n_copies, (int)cudaEventQuery((*dview(ctx, sealdev[slot]).ev_row)[slot]), (int)cudaStreamQuery(ctx->side),
+                            (int)cudaStreamQuery(st), (int)fe, (int)cudaPeekAtLastError());
+                }
+            }
             std::this_thread::yield();
         }
     }
+    if ((rc = enqueue_results())) return bail(rc);
     if (dbg_host)
         fprintf(stderr, "[swb host] rows %lld copies %lld ring %lld fill_seen %.2f ms loop_end %.2f ms max_sink %.3f ms nstage %d\n",
                 nsp, n_copies, R, h_fill, hnow(), h_sink_max, nstage);
@@ -1636,7 +1749,7 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         S1Rows &S1 = ctx->s1;
         S1.resident = R >= nsp && !multi;
         S1.stored = store && !S1.resident;
-        S1.valid = NS == 1 && !J.rank_mode && (S1.resident || S1.stored || nsp == 0);
+        S1.valid = NS == 1 && !J.rank_mode && !rcyc && (S1.resident || S1.stored || nsp == 0);
         S1.m = J.m; S1.n = J.n; S1.k = J.k;
         S1.ma = J.ma; S1.mi = J.mi; S1.go = J.go; S1.ge = J.ge;
         S1.ld = ld[0]; S1.stride = stride[0];
@@ -1792,10 +1905,93 @@ extern "C" int sw_stripe_connect(sw_ctx *ctx, const void *right_handle, int64_t 
     return SW_OK;
 }
 
-extern "C" int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t mismatch, int32_t gap_open,
-                       int32_t gap_ext, int64_t special_row_interval, int32_t *alpha, int32_t *warps)
+// ---------------------------------------------------------------- band-cyclic ranks (one process per GPU)
+
+static size_t cyc_cols(int64_t max_cols) { return (size_t)(((max_cols + 63) / 64) * 64 + 5 * 64); }
+static size_t cyc_bands(int64_t max_rows) { return (size_t)((max_rows + 2047) / 2048 + 4); }  // shortest band: 2048 rows
+
+extern "C" int sw_cyclic_export(sw_ctx *ctx, int64_t max_rows, int64_t max_cols, void *handle_out)
 {
-    if (!ctx || !alpha || !warps || m < 0 || n < 0 || special_row_interval < 0) return SW_EINVAL;
+    if (!ctx || max_rows < 0 || max_cols < 0 || !handle_out) return SW_EINVAL;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const size_t cols = cyc_cols(max_cols), bands = cyc_bands(max_rows);
+    if (!ctx->cin || ctx->cin_cols != cols || ctx->cin_bands != bands) {
+        if (ctx->cin) cudaFree(ctx->cin);
+        ctx->cin = nullptr;
+        const size_t bytes = cols * sizeof(int2) + bands * sizeof(unsigned long long);
+        if (cudaMalloc(&ctx->cin, bytes) != cudaSuccess) {
+            cudaGetLastError();
+            snprintf(ctx->errbuf, sizeof(ctx->errbuf), "cudaMalloc(%zu) for the band-cyclic area failed", bytes);
+            return SW_ENOMEM;
+        }
+        CK(cudaMemset(ctx->cin, 0, bytes));  // progress tags start below every epoch
+        ctx->cin_cols = cols;
+        ctx->cin_bands = bands;
+    }
+    cudaIpcMemHandle_t h;
+    CK(cudaIpcGetMemHandle(&h, ctx->cin));
+    memcpy(handle_out, &h, sizeof(h));
+    return SW_OK;
+}
+
+extern "C" int sw_cyclic_connect(sw_ctx *ctx, const void *next_handle, int64_t max_rows, int64_t max_cols)
+{
+    if (!ctx || !next_handle || max_rows < 0 || max_cols < 0) return SW_EINVAL;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    if (ctx->cout) {
+        cudaIpcCloseMemHandle(ctx->cout);
+        ctx->cout = nullptr;
+    }
+    cudaIpcMemHandle_t h;
+    memcpy(&h, next_handle, sizeof(h));
+    CK(cudaIpcOpenMemHandle(&ctx->cout, h, cudaIpcMemLazyEnablePeerAccess));
+    ctx->cout_cols = cyc_cols(max_cols);
+    ctx->cout_bands = cyc_bands(max_rows);
+    return SW_OK;
+}
+
+extern "C" int32_t sw_cyclic_epoch(const sw_ctx *ctx) { return ctx ? ctx->pepoch : 0; }
+
+extern "C" int sw_align_stage1_cyclic(sw_ctx *ctx, const char *dseqA, int64_t m, const char *dseqB, int64_t n,
+                                      int32_t rank, int32_t world, int32_t epoch, int32_t match, int32_t mismatch,
+                                      int32_t gap_open, int32_t gap_ext, int64_t special_row_interval,
+                                      sw_row_sink sink, void *user, void *stream, sw_result *out)
+{
+    if (!valid_common(ctx, m, n, special_row_interval, sink, out)) return SW_EINVAL;
+    if (!dseqA || !dseqB || m <= 0 || n <= 0 || world < 2 || world > 64 || rank < 0 || rank >= world) return SW_EINVAL;
+    if (epoch <= ctx->pepoch) {
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "cyclic epoch %d not above this context's %d (sw_cyclic_epoch)", epoch, ctx->pepoch);
+        return SW_EINVAL;
+    }
+    int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
+    if (rc) return rc;
+    if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
+    const auto t0 = std::chrono::steady_clock::now();
+    begin_stats(ctx);
+    Job J{};
+    J.dA = (const unsigned char *)dseqA; J.m = m; J.dB = (const unsigned char *)dseqB; J.n = n;
+    J.ma = match; J.mi = mismatch; J.go = gap_open; J.ge = gap_ext;
+    J.k = special_row_interval; J.sink = sink; J.user = user;
+    J.local = true;
+    J.nv = 1;
+    J.rank_cyc = true;
+    J.cyc_world = world;
+    J.cyc_rank = rank;
+    J.epoch = epoch;
+    int4 r;
+    rc = run_job(ctx, J, (cudaStream_t)stream, &r);
+    if (rc) return rc;
+    out->score = r.x;
+    out->i = r.y;
+    out->j = r.z;
+    ctx->stats.total_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return SW_OK;
+}
+
+extern "C" int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t mismatch, int32_t gap_open,
+                       int32_t gap_ext, int64_t special_row_interval, int32_t world, int32_t *alpha, int32_t *warps)
+{
+    if (!ctx || !alpha || !warps || m < 0 || n < 0 || special_row_interval < 0 || world < 0) return SW_EINVAL;
     int rc = check_scoring(match, mismatch, gap_open, gap_ext, m, n);
     if (rc) return rc;
     if (cudaSetDevice(ctx->device) != cudaSuccess) return SW_ECUDA;
@@ -1804,9 +2000,11 @@ extern "C" int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t
     J.ma = match; J.mi = mismatch; J.go = gap_open; J.ge = gap_ext;
     J.k = special_row_interval;
     J.local = true;
-    J.rank_mode = true;
+    J.rank_mode = world == 0;  // 0: a column-stripe rank; >= 1: a band-cyclic rank of `world`
+    J.rank_cyc = world >= 1;
+    J.cyc_world = std::max(1, (int)world);
     bool use16 = false;
-    const Variant &V = choose_variant(ctx, J, &use16);
+    const Variant &V = choose_variant(ctx, J, &use16, J.rank_cyc ? J.cyc_world : 1);
     *alpha = use16 ? -V.alpha : V.alpha;
     *warps = V.nw;
     return SW_OK;

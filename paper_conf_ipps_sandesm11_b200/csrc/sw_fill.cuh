@@ -90,6 +90,7 @@ struct FillArgs {
     int cross;           // 1: the row border / progress go to another GPU (system-scope release)
     int sp_slots;        // special-row ring slots R (>= the rows of one band)
     const unsigned long long *sp_released;  // mapped host counter: rows 0 .. value-1 have left the ring
+    unsigned admit_ns;   // poll interval of the ring admission
     int go, ge, gf;      // G_open, G_ext, G_first = go + ge
     int one;             // always 1 (see imad())
     uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
@@ -259,6 +260,9 @@ __device__ __forceinline__ int *sp_row(const FillArgs &a, const StripeArgs &S, l
 {
     return S.sp + (q % a.sp_slots) * S.sp_stride;
 }
+#ifndef SWB_ADMIT_POLL
+#define SWB_ADMIT_POLL 1
+#endif
 // Back-pressure of the special-row ring (P:178's bounded SRA): before a band
 // with rows [lo, hi] starts, the rows that used its slots before must have left
 // the device: released >= q_hi - R + 1 (deadlock-free: R >= the rows of one
@@ -274,11 +278,16 @@ __device__ __forceinline__ void sp_admit(const FillArgs &a, long long rowtop, in
     const unsigned long long t0 = gtimer();
     while (true) {
         unsigned long long v;
+#if SWB_ADMIT_POLL == 0
         asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(a.sp_released) : "memory");
+#else
+        asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(a.sp_released) : "memory");
+#endif
         if (v >= need) break;
         if (gtimer() - t0 > 4ull * (unsigned long long)a.timeout_ns) { atomicExch(a.err, 2); break; }
-        __nanosleep(256);
+        __nanosleep(a.admit_ns);
     }
+    __threadfence_system();
 }
 
 // True when DP rows rowtop+1 .. min(rowtop+BH, m) hold a special row (k > 0).

@@ -77,7 +77,7 @@ class StripeGroup:
         c_lo, c_hi = stripe_bounds(n, self.world, self.rank)
         # the epoch: above every epoch any rank's receive area has seen (the flags
         # are compared for equality), the same on all ranks
-        plan = self.ctx.plan(m, n, *scoring, k=k)
+        plan = self.ctx.plan(m, n, *scoring, k=k, world=0)
         info = self._agree((self.ctx.stripe_epoch(), plan))
         if len({p for _, p in info}) != 1:
             raise RuntimeError(f"ranks chose different kernel geometries {[p for _, p in info]}: the band "
@@ -87,3 +87,46 @@ class StripeGroup:
                                                 sink=sink, stream=stream)
         allres = self._agree(local.astuple())
         return combine_best(allres), local.astuple(), (c_lo, c_hi)
+
+
+class CyclicGroup:
+    """This rank's share of a band-cyclic multi-GPU Stage 1:
+    rank r runs bands r, r + world, ...; each band's bottom row and progress go
+    to rank (r + 1) mod world by peer stores into its CUDA IPC area.  The
+    handles are exchanged here; the epoch and the kernel geometry are agreed
+    before each call; the ranks' bests are combined by the library's order."""
+
+    def __init__(self, ctx, rank: int, world: int, max_rows: int, max_cols: int, group=None):
+        import torch.distributed as dist
+
+        if world < 2:
+            raise ValueError("a band-cyclic group needs at least two ranks")
+        self.ctx, self.rank, self.world, self.group = ctx, rank, world, group
+        self.max_rows, self.max_cols = max_rows, max_cols
+        mine = ctx.cyclic_export(max_rows, max_cols)
+        handles = [None] * world
+        dist.all_gather_object(handles, mine, group=group)
+        ctx.cyclic_connect(handles[(rank + 1) % world], max_rows, max_cols)
+        dist.barrier(group=group)
+
+    def _agree(self, value):
+        import torch.distributed as dist
+
+        vals = [None] * self.world
+        dist.all_gather_object(vals, value, group=self.group)
+        return vals
+
+    def align_stage1(self, dA_ptr: int, m: int, dB_ptr: int, n: int, scoring=(1, -3, 3, 2), k: int = 0,
+                     sink=None, stream: int = 0):
+        """Run this rank's bands; returns (global best, local best).  `sink(row, H, F)`
+        receives the whole special rows of this rank's bands."""
+        if m > self.max_rows or n > self.max_cols:
+            raise ValueError("the matrix exceeds the band-cyclic areas")
+        plan = self.ctx.plan(m, n, *scoring, k=k, world=self.world)
+        info = self._agree((self.ctx.cyclic_epoch(), plan))
+        if len({p for _, p in info}) != 1:
+            raise RuntimeError(f"ranks chose different kernel geometries {[p for _, p in info]}")
+        epoch = 1 + max(e for e, _ in info)
+        local, _ = self.ctx.align_stage1_cyclic(dA_ptr, m, dB_ptr, n, self.rank, self.world, epoch, *scoring, k=k,
+                                                sink=sink, stream=stream)
+        return combine_best(self._agree(local.astuple())), local.astuple()

@@ -149,3 +149,75 @@ def test_two_ranks_ipc_one_gpu():
         h = np.concatenate([got[r][2][row][0] for r in range(world)])
         f = np.concatenate([got[r][2][row][1] for r in range(world)])
         assert np.array_equal(h, oh) and np.array_equal(f, of), row
+
+
+# ---------------------------------------------------------------- band-cyclic ranks, one GPU, CUDA IPC
+
+def _cyc_rank_main(rank, world, port, A, B, k, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_sandesm11_b200 import Context
+    from paper_conf_ipps_sandesm11_b200.parallel import CyclicGroup
+
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        ctx = Context(0)
+        ctx.set_kernel(1, True)  # 4096-row bands: several per rank
+        ctx.set_grid(2)          # the two processes time-share one GPU: keep their CTAs few
+        dA = torch.from_numpy(A).cuda()
+        dB = torch.from_numpy(B).cuda()
+        rows = {}
+
+        def sink(row, H, F):
+            rows[row] = (H.copy(), F.copy())
+
+        res = []
+        for _ in range(2):  # two groups on one context: epochs agreed above the areas' old tags
+            grp = CyclicGroup(ctx, rank, world, max_rows=len(A), max_cols=len(B))
+            best, local = grp.align_stage1(dA.data_ptr(), len(A), dB.data_ptr(), len(B), PAPER, k=k, sink=sink)
+            res.append(best)
+        q.put((rank, res, rows))
+        ctx.close()
+    except Exception as e:  # report instead of hanging the parent
+        q.put((rank, repr(e), None))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_cyclic_ranks_ipc_one_gpu():
+    """Band-cyclic ranks in two processes (CUDA IPC areas): every special row
+    comes from exactly one rank, whole, bit-exact; the combined best is the
+    oracle's."""
+    import torch.multiprocessing as mp
+
+    A, B = synth.random_pair(12, 4 * 4096 + 1234, 1900, plant_len=1500, s=0.04, g=0.01)
+    k = 512
+    world = 2
+    port = 33000 + random.randint(0, 2000)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    os.environ["SWB_TIMEOUT_S"] = "60"
+    procs = [ctx.Process(target=_cyc_rank_main, args=(r, world, port, A, B, k, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = {}
+    for _ in range(world):
+        rank, res, rows = q.get(timeout=300)
+        got[rank] = (res, rows)
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(world):
+        assert not isinstance(got[r][0], str), got[r][0]
+    want, orows = oracle.stage1(_s(A), _s(B), *PAPER, k=k)
+    for r in range(world):
+        assert got[r][0] == [want, want]
+    assert set(got[0][1]).isdisjoint(got[1][1])
+    allrows = {**got[0][1], **got[1][1]}
+    assert sorted(allrows) == [r for r, _, _ in orows]
+    for row, oh, of in orows:
+        h, f = allrows[row]
+        assert np.array_equal(h, oh) and np.array_equal(f, of), row
