@@ -17,8 +17,10 @@
  *   costs gap_open + L*gap_ext, i.e. G_first = gap_open + gap_ext and
  *   G_ext = gap_ext.  The paper's experiments are (+1, -3, 3, 2)
  *   ("first gap -5, extension -2").
- *   Supported range (the kernel packs the substitution profile into int8):
- *   |match + gap_open + gap_ext| <= 127 and |mismatch + gap_open + gap_ext| <= 127.
+ *   Supported range: any scoring inside the SW_ERANGE rule.  Scorings with
+ *   |match + gap_open + gap_ext| <= 127 and |mismatch + gap_open + gap_ext| <= 127
+ *   use the int8 substitution profile (and the packed kernel when its value
+ *   window allows); wider ones run the WIDE int32 kernels.
  *
  * Coordinates (reading S8): 1-based DP cells.  The end cell is the last
  * aligned pair; the start cell is the cell *before* the first aligned pair

@@ -44,7 +44,10 @@ def check_patch_sites(path: str) -> dict:
     (sw_api.cu patch_sites) refuses to patch otherwise."""
     import struct
 
+    from . import patch_check
+
     data = open(path, "rb").read()
+    text = patch_check.text_ranges(data)
     counts = {}
     for name, v in MAGIC.items():
         pat = struct.pack("<I", v)
@@ -52,9 +55,12 @@ def check_patch_sites(path: str) -> dict:
         while i >= 0:
             offs.append(i)
             i = data.find(pat, i + 1)
-        bad = [o for o in offs if o % 16 != 4]
+        # inside a kernel's .text section, at byte 4 of a 16-byte instruction (the
+        # 32-bit immediate field), counted from the section start
+        sec = [next(((lo, hi) for lo, hi in text if lo <= o < hi), None) for o in offs]
+        bad = [o for o, r in zip(offs, sec) if r is None or (o - r[0]) % 16 != 4]
         if bad:
-            raise RuntimeError(f"{path}: magic {name} at non-immediate offsets {bad[:4]}")
+            raise RuntimeError(f"{path}: magic {name} outside an instruction immediate at offsets {bad[:4]}")
         # ptxas must use the constant as written: a negated copy (x - (-K)) could not be patched
         if data.find(struct.pack("<I", (-v) & 0xFFFFFFFF)) >= 0:
             raise RuntimeError(f"{path}: the negation of magic {name} occurs (an unpatchable form)")
@@ -79,8 +85,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if any(p.wait() for p in procs):
         raise RuntimeError("nvcc failed on the patchable cubin")
     check_patch_sites(ptmp)
-    sys.path.insert(0, os.path.join(ROOT, "tools"))
-    import patch_check
+    from . import patch_check
 
     if patch_check.main(ptmp, palt):
         raise RuntimeError("patchable cubin: SASS depends on the magic values (a derived constant)")

@@ -110,6 +110,7 @@ struct Variant {
     char packed_name[96];   // mangled name of the packed kernel in the patchable cubin ("" : none)
     const void *packed_global_fn;  // packed kernel in global (reverse-pass) mode, alpha 32 x 8 warps only
     char packed_global_name[96];
+    const void *local_wide_fn, *global_wide_fn;  // int32 kernels for scorings outside the int8 profile (default geometry)
 };
 
 template <int NW, int W, bool COOP, int NS>
@@ -135,6 +136,7 @@ static Variant make_variant()
     v.packed_name[0] = 0;
     v.packed_global_fn = nullptr;
     v.packed_global_name[0] = 0;
+    v.local_wide_fn = v.global_wide_fn = nullptr;
     if constexpr (ALPHA >= 30) {
         // packed kernel only (15 to 20 slots per lane); int32 work falls back to the default geometry
         constexpr int NS = ALPHA / 2;
@@ -152,6 +154,10 @@ static Variant make_variant()
     } else {
         v.local_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true>;
         v.global_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, false>;
+        if constexpr (ALPHA == 16 && NW == 8 && W == 64) {
+            v.local_wide_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, true, true>;
+            v.global_wide_fn = (const void *)&sw_fill_kernel<ALPHA, NW, W, false, true>;
+        }
         v.smem = Fill<ALPHA, NW, W, true>::smem_bytes();
         v.skew_tiles = (Fill<ALPHA, NW, W, true>::SKEW + W - 1) / W;
     }
@@ -476,6 +482,8 @@ static void set_kernel_attrs()
     for (int i = 0; i < NVARIANTS; i++) {
         const Variant &v = variant_for(i);
         if (v.local_fn) cudaFuncSetAttribute(v.local_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+        if (v.local_wide_fn) cudaFuncSetAttribute(v.local_wide_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
+        if (v.global_wide_fn) cudaFuncSetAttribute(v.global_wide_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
         if (v.global_fn) cudaFuncSetAttribute(v.global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem);
         if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, TAIL_SMEM);
         if (v.packed_global_fn)
@@ -736,7 +744,6 @@ static int check_scoring(int32_t ma, int32_t mi, int32_t go, int32_t ge, int64_t
 {
     if (go < 0 || ge < 0) return SW_EINVAL;
     const long long gf = (long long)go + ge;
-    if (llabs(ma + gf) > 127 || llabs(mi + gf) > 127) return SW_EINVAL;  // int8 profile
     const long long lim = 1ll << 30;
     const long long mn = std::min(m, n);
     if (mn * (long long)std::max(std::abs(ma), std::abs(mi)) >= lim) return SW_ERANGE;
@@ -771,6 +778,8 @@ struct Job {
     bool rank_mode = false;
     int64_t c_lo = 0, c_hi = 0;
     int epoch = 0;
+    // scoring outside the int8 profile window (|p + G_first| > 127): the WIDE int32 kernels
+    bool wide = false;
     // band-cyclic rank (one process per GPU): this rank runs bands rank, rank + world, ...
     bool rank_cyc = false;
     int cyc_world = 1, cyc_rank = 0;
@@ -895,21 +904,25 @@ static bool packed_qualifies(const sw_ctx *ctx, const Job &J, const Variant &V)
 {
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
     const long long span = 32ll * V.alpha + 140;
-    return ctx->packed && J.local && V.packed_fn && (J.k == 0 || J.k % V.alpha == 0) &&
+    // k >= alpha: at most one special row per lane; rows that are not strip
+    // bottoms take the generic special-row tiles (SPM 2, sw_fill16.cuh), except in
+    // the split-F geometry (variant 12: strip bottoms only, k % alpha == 0)
+    const bool split = &V == &variant_for(12);
+    return ctx->packed && J.local && V.packed_fn && (J.k == 0 || (split ? J.k % V.alpha == 0 : J.k >= V.alpha)) &&
            span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
 }
 
 static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16, int gpus = 1)
 {
+    if (J.wide) {  // only the default int32 geometry has the WIDE instantiation
+        *use16 = false;
+        return variant_for(DEFAULT_VARIANT);
+    }
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
     // packed preconditions: local mode, special rows at strip
     // bottoms, and a warp's live values (32 alpha rows x ~130 columns of
     // Manhattan distance, each step <= p_max + G_first apart) inside the 16-bit frame
-    auto packed_ok = [&](const Variant &V) {
-        const long long span = 32ll * V.alpha + 140;
-        return ctx->packed && J.local && V.packed_fn && (J.k == 0 || J.k % V.alpha == 0) &&
-               span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
-    };
+    auto packed_ok = [&](const Variant &V) { return packed_qualifies(ctx, J, V); };
     if (!J.local && J.match && !J.anchor_gap && ctx->variant_override < 0) {
         // Stage-2 partitions: the packed kernel in global mode with the band-end
         // matching, alpha 16 x 8 warps (4096-row bands, the int32 default's
@@ -994,7 +1007,8 @@ static int setup_seg(sw_ctx *ctx, const Job &J, Seg &G, int P, int NS, bool tail
 {
     const Variant &V = *G.V;
     G.BH = V.alpha * 32 * V.nw;
-    G.fn = G.use16 ? (J.local ? V.packed_fn : V.packed_global_fn) : (J.local ? V.local_fn : V.global_fn);
+    G.fn = G.use16 ? (J.local ? V.packed_fn : V.packed_global_fn)
+                   : J.wide ? (J.local ? V.local_wide_fn : V.global_wide_fn) : (J.local ? V.local_fn : V.global_fn);
     G.smem = G.use16 ? V.smem16 : V.smem;
     G.patched = false;
     if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, G.use16 ? (J.local ? 0 : 3) : J.local ? 1 : 2)) {
@@ -1068,8 +1082,10 @@ static const Variant *choose_tail(sw_ctx *ctx, const Job &J, const Seg &S0, int 
     return pick;
 }
 
-static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *res)
+static int run_job(sw_ctx *ctx, const Job &J0, cudaStream_t user_stream, int4 *res)
 {
+    Job J = J0;
+    J.wide = std::abs((long long)J.ma + J.go + J.ge) > 127 || std::abs((long long)J.mi + J.go + J.ge) > 127;
     const auto h0 = std::chrono::steady_clock::now();
     if (J.local) ctx->s1.valid = false;
     auto hnow = [&]() { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - h0).count(); };
@@ -1332,6 +1348,8 @@ static int run_job(sw_ctx *ctx, const Job &J, cudaStream_t user_stream, int4 *re
         a.ge = J.ge;
         a.gf = J.go + J.ge;
         a.one = 1;
+        a.pm_gf = J.ma + a.gf;
+        a.pn_gf = J.mi + a.gf;
         for (int x = 0; x < 4; x++) {
             uint32_t w = 0;
             for (int y = 0; y < 4; y++) {
@@ -2000,6 +2018,7 @@ extern "C" int sw_plan(sw_ctx *ctx, int64_t m, int64_t n, int32_t match, int32_t
     J.ma = match; J.mi = mismatch; J.go = gap_open; J.ge = gap_ext;
     J.k = special_row_interval;
     J.local = true;
+    J.wide = std::abs((long long)match + gap_open + gap_ext) > 127 || std::abs((long long)mismatch + gap_open + gap_ext) > 127;
     J.rank_mode = world == 0;  // 0: a column-stripe rank; >= 1: a band-cyclic rank of `world`
     J.rank_cyc = world >= 1;
     J.cyc_world = std::max(1, (int)world);
@@ -2361,6 +2380,9 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
         for (int y = 0; y < 4; y++) wv |= (uint32_t)(uint8_t)(int8_t)((x == y ? ma : mi) + g.gf) << (8 * y);
         g.prof[x] = wv;
     }
+    g.pm_gf = ma + g.gf;
+    g.pn_gf = mi + g.gf;
+    g.wide = std::abs((long long)ma + g.gf) > 127 || std::abs((long long)mi + g.gf) > 127;
     auto cells = [](const MMPart &p) { return (long long)(p.i_e - p.i_s) * (long long)(p.j_e - p.j_s); };
     const int WPB = 8;  // warps per block
     if ((rc = grow(ctx, ctx->mm_err, sizeof(int)))) return rc;

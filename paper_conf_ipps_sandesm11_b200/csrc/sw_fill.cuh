@@ -94,6 +94,7 @@ struct FillArgs {
     int go, ge, gf;      // G_open, G_ext, G_first = go + ge
     int one;             // always 1 (see imad())
     uint32_t prof[4];    // profile word for row code a: byte x = (a == x ? ma : mi) + gf
+    int pm_gf, pn_gf;    // WIDE kernels: match + gf, mismatch + gf (any scoring within the SW_ERANGE rule)
     const uint32_t *A2;  // S0 codes, 2 bits each, 16 per word
     const uint32_t *B2;  // S1 codes (global columns)
     int *err;            // non-zero: encode found a bad byte -> do nothing; kernel sets 2 on a wait timeout
@@ -252,6 +253,7 @@ __device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned l
 // Publish `cols` leading columns of band G's bottom row (after its stores are fenced).
 __device__ __forceinline__ void publish_progress(const FillArgs &a, const StripeArgs &S, int G, int cols)
 {
+    cols = max(cols, 0);  // the first drained tile of a W = 32 kernel publishes W - SKEW < 0 columns
     if (a.cross) __threadfence_system();
     st_release_u64(S.prog_out + G + 1, ptag(a.pepoch, cols), a.cross);
 }
@@ -327,7 +329,14 @@ struct Smem {
     static constexpr int SRING = SRING_MIN <= 256 ? 256 : SRING_MIN <= 512 ? 512 : SRING_MIN <= 1024 ? 1024 : SRING_MIN <= 2048 ? 2048 : 4096;
 };
 
-template <int ALPHA, int NW, int W, bool LOCAL>
+// WIDE = true: the substitution score p + G_first is selected from the two
+// int32 values (pm_gf, pn_gf) by comparing the row's and the column's 2-bit
+// codes (ISETP + SEL) instead of a PRMT of the int8x4 profile, so any scoring
+// inside the SW_ERANGE rule runs (|p + G_first| > 127 included).  Pad rows and
+// pad columns get codes that never match: their cells are real-looking
+// mismatches, which is harmless -- they lie below / right of every real cell
+// and the exact tracking ignores rows > m and columns > w.
+template <int ALPHA, int NW, int W, bool LOCAL, bool WIDE = false>
 struct Fill {
     static constexpr int BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
@@ -344,6 +353,12 @@ struct Fill {
     static size_t smem_bytes()
     {
         return sizeof(int2) * RING * (NW + 1) + sizeof(uint32_t) * SRING + sizeof(int) * NSAVE * 32 * NW;
+    }
+
+    static __device__ __forceinline__ int subst(const FillArgs &a, uint32_t P, uint32_t sel)
+    {
+        if constexpr (WIDE) return P == sel ? a.pm_gf : a.pn_gf;
+        else return prmt(P, PADPROF, sel);
     }
 
     // ---------------------------------------------------------------- per-lane state
@@ -395,7 +410,7 @@ struct Fill {
             // G_ext <= G_first, so the chain down the rows is one VIADDMNMX per row;
             // the constants are immediates in the patched image.
             const int eA = __viaddmax_s32(L.e[r], NGE(a), L.t[r]);
-            const int pA = prmt(L.P[r], PADPROF, sl.x);
+            const int pA = subst(a, L.P[r], sl.x);
             const int xA = tdA + pA;
             const int dA = LOCAL ? __vimax_s32_relu(eA, xA) : max(eA, xA);
             const int dgA = dA + NGF(a);
@@ -406,7 +421,7 @@ struct Fill {
             tuA = tA;
             // column j0 + 1 (one row behind column j0 in the dependency chain)
             const int eB = __viaddmax_s32(eA, NGE(a), tA);
-            const int pB = prmt(L.P[r], PADPROF, sl.y);
+            const int pB = subst(a, L.P[r], sl.y);
             const int xB = tdB + pB;
             const int dB = LOCAL ? __vimax_s32_relu(eB, xB) : max(eB, xB);
             const int dgB = dB + NGF(a);
@@ -465,7 +480,7 @@ struct Fill {
             // FMA pipe (the adds, as IMAD with a runtime 1): DESIGN.md section 5.
             const int eA = __viaddmax_s32(L.e[r], NGE(a), L.t[r]);
             fuA = max(fuA + NGE(a), tuA);
-            const int pA = prmt(L.P[r], PADPROF, sl.x);
+            const int pA = subst(a, L.P[r], sl.x);
             const int xA = tdA + pA;
             const int hA = LOCAL ? __vimax3_s32_relu(eA, fuA, xA) : __vimax3_s32(eA, fuA, xA);
             tdA = L.t[r];
@@ -474,7 +489,7 @@ struct Fill {
             // column j0 + 1 (one row behind column j0 in the dependency chain)
             const int eB = __viaddmax_s32(eA, NGE(a), tA);
             fuB = max(fuB + NGE(a), tuB);
-            const int pB = prmt(L.P[r], PADPROF, sl.y);
+            const int pB = subst(a, L.P[r], sl.y);
             const int xB = tdB + pB;
             const int hB = LOCAL ? __vimax3_s32_relu(eB, fuB, xB) : __vimax3_s32(eB, fuB, xB);
             tdB = tA;
@@ -615,10 +630,10 @@ __device__ __forceinline__ int2 ld_sys_int2(const int2 *p)
     return v;
 }
 
-template <int ALPHA, int NW, int W, bool LOCAL>
+template <int ALPHA, int NW, int W, bool LOCAL, bool WIDE = false>
 __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_constant__ FillArgs a)
 {
-    using F = Fill<ALPHA, NW, W, LOCAL>;
+    using F = Fill<ALPHA, NW, W, LOCAL, WIDE>;
     constexpr int RING = F::RING, SRING = F::SRING, BH = F::BH, SKEW = F::SKEW, STEPS = F::STEPS, LAG = F::LAG;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int2 *rings = reinterpret_cast<int2 *>(smem_raw);                        // (NW+1) x RING
@@ -675,7 +690,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
 #pragma unroll
             for (int r = 0; r < ALPHA; r++) {
                 const uint32_t code = (w >> (sh + 2 * r)) & 3u;
-                L.P[r] = (row0 + r < a.m) ? a.prof[code] : PADPROF;
+                L.P[r] = (row0 + r < a.m) ? (WIDE ? code : a.prof[code]) : (WIDE ? 5u : PADPROF);
                 L.e[r] = NEG;
                 // H(i,0) - G_first; -inf when the anchor is a gap crosspoint (S20)
                 L.t[r] = LOCAL ? -a.gf : a.anchor_gap ? NEG : -(a.go + (row0 + r + 1) * a.ge) - a.gf;
@@ -731,7 +746,7 @@ __global__ void __launch_bounds__((NW + 1) * 32) sw_fill_kernel(const __grid_con
                     const int gc = S.col0 + col;
                     code = (__ldg(a.B2 + (gc >> 4)) >> ((gc & 15) * 2)) & 3u;
                 }
-                selr[col & (SRING - 1)] = col_sel(code);
+                selr[col & (SRING - 1)] = WIDE ? (code == 4u ? 6u : code) : col_sel(code);
             }
         };
         // special row that is this band's bottom row: written here, coalesced

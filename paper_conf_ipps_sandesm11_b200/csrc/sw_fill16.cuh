@@ -185,12 +185,21 @@ struct Fill16 {
     // Offset from the tile maximum a non-replay tile returns to H (mode 2: t).
     static __device__ __forceinline__ int tmax_off(const FillArgs &a) { return SWB_FMODE == 2 && !SPLIT ? a.gf : 0; }
 
-    template <bool GUARD, bool TRACK, bool SP1, bool CAP>
+    // SPM: 0 no special row in the warp; 1 special rows are strip bottoms (the
+    // high half of the last slot); 2 one special row per lane anywhere in the
+    // strip (k >= alpha, host rule): strip row sp_r (< NS: slot sp_r's low half,
+    // else slot sp_r - NS's high half, one column behind), -1 none -- a tail
+    // segment whose first row is not a multiple of alpha, or k not a multiple of
+    // alpha.  The slot loop only selects that slot's (t, F) (two SELs per slot);
+    // one store pair after the loop.
+    template <bool GUARD, bool TRACK, int SPM, bool CAP>
     static __device__ __forceinline__ uint32_t step(const FillArgs &a, const StepInfo &X, Lane &L, int k, int lane,
                                                     uint32_t cr_a, uint32_t ro_a, uint32_t sel_a, uint32_t pt_sel,
                                                     int one, uint32_t tmax, int row1, int &bs, int &bi, int &bj,
-                                                    int *sp_ptr)
+                                                    int *sp_ptr, int sp_r)
     {
+        const int sp_s = sp_r < NS ? sp_r : sp_r - NS;  // the slot of the lane's special row (SPM 2)
+        uint32_t sp_t = 0u, sp_f = 0u;
         const uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[NS - 1], 1);
         const uint32_t up_f = __shfl_up_sync(0xffffffffu, L.fn, 1);
         const int jl = k - 2 * lane;
@@ -284,9 +293,11 @@ struct Fill16 {
                 td = L.t[s];
                 uint32_t h0, t0;
                 if (s == NS - 1) f15 = fu;  // odd NS: the last slot is unpaired
+                const uint32_t fin0 = fu;   // F of slot s's rows (SPM 2)
                 cell_hf<TRACK>(d0, fu, h0, t0, one, nge2, ngf2, nge16, ngf16);
                 L.e[s] = e0;
                 L.t[s] = t0;
+                if (SPM == 2 && !TRACK && s == sp_s) { sp_t = t0; sp_f = fin0; }
                 if (s + 1 == NS) {
                     tmax = __vmaxu2(tmax, h0);
                     if (CAP) {
@@ -301,9 +312,11 @@ struct Fill16 {
                 const uint32_t d1 = __viaddmax_u16x2(td, p1, e1);
                 td = L.t[s + 1];
                 uint32_t h1, t1;
+                const uint32_t fin1 = fu;
                 cell_hf<TRACK>(d1, fu, h1, t1, one, nge2, ngf2, nge16, ngf16);
                 L.e[s + 1] = e1;
                 L.t[s + 1] = t1;
+                if (SPM == 2 && !TRACK && s + 1 == sp_s) { sp_t = t1; sp_f = fin1; }
                 tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
                 if (CAP) {
                     if (jl == X.jcap) {
@@ -392,7 +405,14 @@ struct Fill16 {
             return 0;
         }
         const int jo = jl - 1;  // row 2NS-1's column (high half of the last slot)
-        if (SP1 && sp_ptr != nullptr && jo >= 0 && jo < X.w) {
+        if (SPM == 2 && !SPLIT && sp_ptr != nullptr) {
+            const int hi = sp_r >= NS ? 1 : 0, col = jl - hi;
+            if (col >= 0 && col < X.w) {
+                sp_ptr[col] = toabs(L, hi ? hi16(sp_t) : lo16(sp_t)) + a.gf;  // H = t + G_first
+                sp_ptr[X.sp_ld + col] = toabs(L, hi ? hi16(sp_f) : lo16(sp_f));
+            }
+        }
+        if (SPM == 1 && sp_ptr != nullptr && jo >= 0 && jo < X.w) {
             sp_ptr[jo] = toabs(L, hi16(L.t[NS - 1])) + a.gf;  // H = t + G_first
             sp_ptr[X.sp_ld + jo] = toabs(L, hi16(f15));
         }
@@ -418,10 +438,10 @@ struct Fill16 {
         __syncwarp();
     }
 
-    template <bool GUARD, bool TRACK, bool SP1, bool CAP>
+    template <bool GUARD, bool TRACK, int SPM, bool CAP>
     static __device__ __forceinline__ uint32_t tile(const FillArgs &a, const StepInfo &X, Lane &L, int c, int lane,
                                                     uint32_t cring, uint32_t ring_out, uint32_t selr, int row1,
-                                                    int &bs, int &bi, int &bj, int *sp_ptr)
+                                                    int &bs, int &bi, int &bj, int *sp_ptr, int sp_r)
     {
         uint32_t tmax = 0;
         const int k0 = c * STEPS;
@@ -434,18 +454,18 @@ struct Fill16 {
         if (GUARD || TRACK || CAP) {
 #pragma unroll 1
             for (int kk = 0; kk < STEPS; kk++)
-                tmax = step<GUARD, TRACK, SP1, CAP>(a, X, L, k0 + kk, lane, cring + 4u * kk, ro0 + 8u * kk,
+                tmax = step<GUARD, TRACK, SPM, CAP>(a, X, L, k0 + kk, lane, cring + 4u * kk, ro0 + 8u * kk,
                                                     sel0 + 4u * ((kk >> 1) + (kk & 1) * HALF), pt_sel, one, tmax,
-                                                    row1, bs, bi, bj, sp_ptr);
+                                                    row1, bs, bi, bj, sp_ptr, sp_r);
         } else {
 #pragma unroll 1
             for (int kq = 0; kq < STEPS; kq += UNR) {
                 const uint32_t sq = sel0 + 2u * kq, cq = cring + 4u * kq, oq = ro0 + 8u * kq;
 #pragma unroll
                 for (int u = 0; u < UNR; u++)
-                    tmax = step<false, false, SP1, false>(a, X, L, k0 + kq + u, lane, cq + 4u * u, oq + 8u * u,
+                    tmax = step<false, false, SPM, false>(a, X, L, k0 + kq + u, lane, cq + 4u * u, oq + 8u * u,
                                                           sq + 4u * ((u >> 1) + (u & 1) * HALF), pt_sel, one, tmax,
-                                                          row1, bs, bi, bj, sp_ptr);
+                                                          row1, bs, bi, bj, sp_ptr, sp_r);
             }
         }
         return tmax;
@@ -540,6 +560,8 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
     X.sp_stride = S.sp_stride;
     X.jcap = S.w - 1;
     X.rbrow = nullptr;
+    X.sp_end = S.sp != nullptr ? S.sp + (long long)a.sp_slots * S.sp_stride : nullptr;
+    X.sp_span = (long long)a.sp_slots * S.sp_stride;
     // steps at which a lane meets the capture column: low half at k = jcap + 2 lane, high at +1
     const int cap_t0 = X.jcap / STEPS, cap_t1 = (X.jcap + 63) / STEPS;
 
@@ -562,7 +584,8 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         typename F::Lane L;
         const int row0 = rowtop + (warp * 32 + lane) * ALPHA;
         int *sp_ptr = nullptr;
-        bool warp_sp = false;
+        int sp_r = -1;  // this lane's special row within its strip (-1: none)
+        bool warp_sp = false, warp_sp2 = false;
         X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
         auto init_state = [&](bool from_left) {
             // state at the column left of the stripe: the column-0 boundary or the left border
@@ -623,12 +646,16 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             }
             init_state(false);
             if (a.k > 0) {
-                // special rows are strip-bottom rows (k a multiple of ALPHA): row0 + ALPHA
-                const int row = row0 + ALPHA;
-                if (row <= a.m && row % a.k == 0 && row != rowtop + BH)  // band bottom: the I/O warp's drain
+                // this lane's special row among rows row0 + 1 .. row0 + ALPHA (k >= ALPHA:
+                // at most one; the band's bottom row is the I/O warp's drain)
+                const int row = ((row0 + a.k) / a.k) * a.k;  // the first multiple of k above row0
+                if (row <= row0 + ALPHA && row <= a.m && row != rowtop + BH) {
+                    sp_r = row - row0 - 1;
                     sp_ptr = sp_row(a, S, row / a.k - 1);
+                }
             }
-            warp_sp = __any_sync(0xffffffffu, sp_ptr != nullptr);
+            warp_sp = __any_sync(0xffffffffu, sp_r >= 0);
+            warp_sp2 = !SPLIT && __any_sync(0xffffffffu, sp_r >= 0 && sp_r != ALPHA - 1);
         }
 
         auto io_load = [&](int c) {
@@ -785,27 +812,31 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     uint32_t tm;
                     const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
                     if (cap) {
-                        tm = warp_sp ? F::template tile<true, false, true, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr)
-                                     : F::template tile<true, false, false, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr);
+                        tm = warp_sp2 ? F::template tile<true, false, 2, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                           : warp_sp ? F::template tile<true, false, 1, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                                     : F::template tile<true, false, 0, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                         if (c == cap_t1) {
                             __threadfence_system();
                             __syncwarp();
                             if (lane == 0 && S.rready != nullptr) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
                         }
                     } else if (c == 0) {
-                        tm = warp_sp ? F::template tile<true, false, true, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr)
-                                     : F::template tile<true, false, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr);
+                        tm = warp_sp2 ? F::template tile<true, false, 2, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                           : warp_sp ? F::template tile<true, false, 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                                     : F::template tile<true, false, 0, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
+                    } else if (warp_sp2) {
+                        tm = F::template tile<false, false, 2, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else if (warp_sp) {
-                        tm = F::template tile<false, false, true, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr);
+                        tm = F::template tile<false, false, 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else {
-                        tm = F::template tile<false, false, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
+                        tm = F::template tile<false, false, 0, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr, -1);
                     }
                     const int tmax = F::toabs(L, max(lo16(tm), hi16(tm))) + F::tmax_off(a);
                     const int thr = LOCAL ? max(max(bs0, gbest), 1) : a.goal;
                     if (__any_sync(0xffffffffu, tmax >= thr)) {
                         F::restore(L, sv, lane);
                         const int obs = bs, obi = bi, obj = bj;
-                        F::template tile<true, true, false, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr);
+                        F::template tile<true, true, 0, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, nullptr, -1);
                         if (lane == 0) nrep++;
                         if (LOCAL) {
                             if (bs > obs) atomicMax(a.gbest, bs);

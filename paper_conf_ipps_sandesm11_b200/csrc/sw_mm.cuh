@@ -53,6 +53,8 @@ struct MMArgs {
     const unsigned char *A, *B;  // ASCII S0, S1 (0-based; DP row i pairs A[i - 1])
     int ma, mi, go, ge, gf;
     uint32_t prof[4];    // row code a -> int8x4 word, byte x = (a == x ? ma : mi) + G_first
+    int wide;            // 1: |p + G_first| > 127; p + G_first selected from pm_gf / pn_gf by comparing codes
+    int pm_gf, pn_gf;
     int nparts;
     const MMPart *parts;
     int2 *scratch;
@@ -104,10 +106,10 @@ __device__ __forceinline__ uint32_t mm_code(unsigned char c) { return (c >> 1) &
 //     bit 3 F extends; codes[b * HW + (a - 1) / 8], nibble (a - 1) % 8.
 // wait(need): block until rin holds columns 1..need (CTA pipeline; no-op for
 // one warp); publish(cols): rout holds columns 1..cols.
-template <int MODE, bool CAPC, class Wait, class Publish>
-__device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a0, const int2 *rin, int2 *rout,
-                                         int capR, int2 *cap, unsigned int *codes, int lane, Wait wait,
-                                         Publish publish)
+template <int MODE, bool CAPC, bool WIDE, class Wait, class Publish>
+__device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, int a0, const int2 *rin, int2 *rout,
+                                              int capR, int2 *cap, unsigned int *codes, int lane, Wait wait,
+                                              Publish publish)
 {
     const int h = P.h, w = P.w, kind = P.kind;
     const int HW = (h + 7) / 8;
@@ -118,7 +120,8 @@ __device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a
 #pragma unroll
     for (int r = 0; r < MM_ALPHA; r++) {
         const int a = r0 + r + 1;
-        Pw[r] = a <= h ? g.prof[mm_code(P.rs[(long long)a * P.rstep])] : PADPROF;
+        if constexpr (WIDE) Pw[r] = a <= h ? mm_code(P.rs[(long long)a * P.rstep]) : 5u;  // pad rows: never a match
+        else Pw[r] = a <= h ? g.prof[mm_code(P.rs[(long long)a * P.rstep])] : PADPROF;
         T[r] = mm_col0(g, kind, a) - gf;
         E[r] = NEG;
     }
@@ -138,7 +141,7 @@ __device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a
         if (lane == 0) { tu = rH - gf; fu = rF; }
         const int b = k - lane + 1;
         if (guard && (b < 1 || b > w)) return;
-        const uint32_t sel = col_sel(mm_code(P.cs[(long long)b * P.cstep]));
+        const uint32_t sel = WIDE ? mm_code(P.cs[(long long)b * P.cstep]) : col_sel(mm_code(P.cs[(long long)b * P.cstep]));
         int td = tdiag;
         tdiag = tu;
         unsigned int code = 0;
@@ -147,7 +150,7 @@ __device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a
         for (int r = 0; r < MM_ALPHA; r++) {
             const int e = __viaddmax_s32(E[r], nge, T[r]);   // Eq. 2
             const int f = __viaddmax_s32(fu, nge, tu);       // Eq. 3
-            const int x = td + prmt(Pw[r], PADPROF, sel);    // H_diag + p
+            const int x = td + (WIDE ? (Pw[r] == sel ? g.pm_gf : g.pn_gf) : prmt(Pw[r], PADPROF, sel));  // H_diag + p
             const int hv = __vimax3_s32(e, f, x);            // Eq. 1 (global: no 0 term)
             if (MODE == 1) {
                 const unsigned int src = (x >= e && x >= f) ? 0u : (f >= e ? 1u : 2u);
@@ -184,6 +187,16 @@ __device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a
         }
         publish(min(w, kb + 1));
     }
+}
+
+// The int8-profile or the WIDE cell update (a uniform branch outside the cell loop).
+template <int MODE, bool CAPC, class Wait, class Publish>
+__device__ __forceinline__ void mm_chunk(const MMArgs &g, const DpProb &P, int a0, const int2 *rin, int2 *rout,
+                                         int capR, int2 *cap, unsigned int *codes, int lane, Wait wait,
+                                         Publish publish)
+{
+    if (g.wide) mm_chunk_impl<MODE, CAPC, true>(g, P, a0, rin, rout, capR, cap, codes, lane, wait, publish);
+    else mm_chunk_impl<MODE, CAPC, false>(g, P, a0, rin, rout, capR, cap, codes, lane, wait, publish);
 }
 
 // One warp runs the whole pass (chunks one after the other, row buffer in place).

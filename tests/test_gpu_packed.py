@@ -10,7 +10,7 @@ import synth
 
 pytestmark = pytest.mark.gpu
 PAPER = (1, -3, 3, 2)
-PACKED_VARIANTS = [0, 3, 5, 6, 8, 9, 10, 11, 12]
+PACKED_VARIANTS = [0, 1, 3, 5, 6, 8, 9, 10, 11, 12, 13, 14, 15, 16, 17]
 # alpha 16: 4, 12, 15 warps + I/O warp, 16 warps with cooperative I/O;
 # alpha 32 (16 slots per lane): 4 warps + I/O warp, 4 cooperative, 8 + I/O warp, 16 cooperative, 4 + I/O split F chain
 
@@ -68,8 +68,23 @@ def test_packed_scorings(ctx, variant):
 
 def test_packed_falls_back_when_not_applicable(ctx):
     A, B = synth.random_pair(8, 900, 700, plant_len=500)
-    check(ctx, A, B, PAPER, 7, 5, expect_packed=False)            # k not a multiple of 16
     check(ctx, A, B, (100, -20, 20, 5), 16, 5, expect_packed=False)  # value window too wide
+    check(ctx, A, B, PAPER, 7, 12, expect_packed=False)  # the split-F geometry keeps strip-bottom rows only
+
+
+ALPHA = {0: 16, 1: 16, 3: 16, 5: 16, 6: 16, 8: 32, 9: 32, 10: 32, 11: 32, 12: 32, 13: 30, 14: 34, 15: 36,
+         16: 38, 17: 40}
+
+
+@pytest.mark.parametrize("variant", [0, 1, 5, 8, 10, 13, 14, 16, 17])
+@pytest.mark.parametrize("k", [7, 16, 33, 100, 1000, 4097])
+def test_packed_any_special_row_interval(ctx, variant, k):
+    """Special rows that are not strip bottoms (k >= alpha, not a multiple of
+    it): the generic special-row tiles (SPM 2) store the lane's one special row
+    from whichever slot and half holds it; every row against the oracle.  k <
+    alpha (several rows per lane) runs the int32 kernel."""
+    A, B = synth.random_pair(30 + variant + k, 9000, 1300, plant_len=1000, s=0.05, g=0.01)
+    check(ctx, A, B, PAPER, k, variant, expect_packed=k >= ALPHA[variant])
 
 
 def test_packed_ties_and_long_alignment(ctx):
@@ -95,7 +110,8 @@ def test_packed_alpha32(ctx, variant):
     A, B = synth.random_pair(70 + variant, 7000, 2100, plant_len=1500, s=0.04, g=0.01)
     check(ctx, A, B, PAPER, 96, variant)
     check(ctx, A, B, (5, -4, 10, 1), 64, variant)
-    check(ctx, A, B, PAPER, 16, variant, expect_packed=False)
+    check(ctx, A, B, PAPER, 16, variant, expect_packed=False)  # k < alpha: two rows per lane, int32
+    check(ctx, A, B, PAPER, 48, variant, expect_packed=variant != 12)  # k % alpha != 0: generic rows
     X = synth.random_pair(4, 500, 1)[0]
     check(ctx, np.concatenate([X, X, X, X]), X, PAPER, 32, variant)
     check(ctx, A, B, PAPER, 32, variant, stripes=3)

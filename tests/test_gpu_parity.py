@@ -112,7 +112,7 @@ def test_case_insensitive_and_alphabet(ctx):
 def test_bad_parameters(ctx):
     from paper_conf_ipps_sandesm11_b200 import SW_EINVAL, SW_ERANGE, SwError
 
-    for args in [(1, -3, -1, 2), (1, -3, 3, -2), (200, -3, 3, 2)]:
+    for args in [(1, -3, -1, 2), (1, -3, 3, -2)]:  # (200, -3, 3, 2) runs: tests/test_gpu_wide.py
         with pytest.raises(SwError) as e:
             ctx.align_stage1("ACGT", "ACGT", *args)
         assert e.value.code == SW_EINVAL

@@ -107,7 +107,10 @@ def _sampled_induction(ctx, cfg, k, sample, expect_kernel):
 
     got, _ = ctx.align_stage1(A, B, *PAPER, k=k, sink=sink)
     s1 = ctx.stats()
-    assert (s1["alpha"], s1["warps"], s1["patched"]) == expect_kernel, s1
+    if expect_kernel is not None:
+        assert (s1["alpha"], s1["warps"], s1["patched"]) == expect_kernel, s1
+    else:  # the automatic choice (the one bench.py runs): a patched packed geometry, maybe with a tail segment
+        assert s1["alpha"] < 0 and s1["patched"] == 1, s1
     assert s1["special_rows"] == cfg.m // k
     jobs = [(q, q * k, min((q + 1) * k, cfg.m)) for q in sorted(sample) if q * k < cfg.m]
     res = _run_bands(A, B, rows, jobs)
@@ -139,11 +142,11 @@ def test_c3_sampled_band_induction(ctx):
 
 
 def test_c4_sampled_band_induction(ctx):
-    """C4 (10M x 10M, the scaling config) in the geometry bench.py times
-    (alpha 32 x 8 warps, 8192-row bands: 1221 bands on 148 CTAs, 8 full waves
-    and a partial ninth): special rows every 8192 rows; a seeded sample of
-    bands from every wave, the bands around the planted homology (the end
-    cell) and the ragged last band."""
+    """C4 (10M x 10M, the scaling config) in the geometry bench.py times (the
+    automatic choice: several waves of tall bands, plus a tail segment when the
+    last wave is partial): special rows every 8192 rows; a
+    seeded sample of bands from every wave, the bands around the planted
+    homology (the end cell) and the ragged last band."""
     cfg = synth.CONFIGS["C4"]
     k = 8192
     rng = np.random.default_rng(4)
@@ -152,5 +155,5 @@ def test_c4_sampled_band_induction(ctx):
     a0, L = cfg.params["a0"], cfg.params["L"]
     sample.update(range(a0 // k, (a0 + 2 * L) // k + 1))
     sample.add(nbands)  # the ragged last band
-    got = _sampled_induction(ctx, cfg, k, sample, (-32, 8, 1))
+    got = _sampled_induction(ctx, cfg, k, sample, None)
     assert a0 < got.i <= a0 + 2 * L

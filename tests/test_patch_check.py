@@ -1,5 +1,5 @@
 """The two-build check that guards the immediate-patched packed kernels
-(tools/patch_check.py), pinned on tiny kernels compiled here
+(paper_conf_ipps_sandesm11_b200/patch_check.py), pinned on tiny kernels compiled here
 (nvcc cross-compiles without a GPU): a magic constant used verbatim passes; a
 constant derived from it (2*K folded into an immediate) is caught."""
 import os
@@ -10,7 +10,7 @@ import sys
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-sys.path.insert(0, os.path.join(ROOT, "tools"))
+sys.path.insert(0, ROOT)
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 SRC = r"""
@@ -35,7 +35,7 @@ def _cubin(tmp_path, name, *flags):
 
 @pytest.mark.skipif(shutil.which(NVCC) is None and not os.path.exists(NVCC), reason="nvcc not available")
 def test_patch_check_accepts_verbatim_and_catches_derived(tmp_path):
-    import patch_check
+    from paper_conf_ipps_sandesm11_b200 import patch_check
 
     alt = "-DK=0x1d2f3b61u"  # patch_check.MB[0], the alternative of MA[0]
     assert patch_check.main(_cubin(tmp_path, "a"), _cubin(tmp_path, "b", alt)) == 0
