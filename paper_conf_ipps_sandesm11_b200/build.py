@@ -74,16 +74,23 @@ def check_patch_sites(path: str) -> dict:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
-    # the patchable cubin, twice: with the magic set used at run time and with an
-    # alternative set; the SASS must agree up to the magic words (tools/patch_check.py)
+    # in parallel: the patchable cubin twice (the magic set used at run time and
+    # an alternative set; the SASS must agree up to the magic words,
+    # patch_check.py) and the library's object; then the embedding object and the link
     ptmp = PATCH_CUBIN + f".tmp{os.getpid()}"
     palt = PATCH_CUBIN + f".alt{os.getpid()}"
+    obj = LIB[:-3] + f".{os.getpid()}.o"  # nvcc picks the input kind by extension
     cflags = [f for f in FLAGS if f not in ("-Xcompiler", "-fPIC", "-shared")]
     alt = [f"-DSWB_K_{k}={v:#x}u" for k, v in zip(MAGIC, ALT_MAGIC)]
+    ocmd = [NVCC, *cflags, "-Xcompiler", "-fPIC", "-DSWB_PATCH_EXTERN", "-c", "-o", obj, *SOURCES]
+    if verbose:
+        ocmd.insert(1, "-Xptxas=-v")
+        print(" ".join(ocmd))
     procs = [subprocess.Popen([NVCC, *cflags, "-cubin", "-o", ptmp, PATCH_SRC]),
-             subprocess.Popen([NVCC, *cflags, *alt, "-cubin", "-o", palt, PATCH_SRC])]
-    if any(p.wait() for p in procs):
-        raise RuntimeError("nvcc failed on the patchable cubin")
+             subprocess.Popen([NVCC, *cflags, *alt, "-cubin", "-o", palt, PATCH_SRC]),
+             subprocess.Popen(ocmd)]
+    if any([p.wait() for p in procs]):
+        raise RuntimeError("nvcc failed")
     check_patch_sites(ptmp)
     from . import patch_check
 
@@ -91,12 +98,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("patchable cubin: SASS depends on the magic values (a derived constant)")
     os.remove(palt)
     os.replace(ptmp, PATCH_CUBIN)
+    emb_s = LIB[:-3] + f".embed{os.getpid()}.S"
+    emb_o = emb_s[:-2] + ".o"
+    with open(emb_s, "w") as f:
+        f.write(".section .rodata\n.balign 16\n.globl swb_patch_cubin_begin\n.globl swb_patch_cubin_end\n"
+                f"swb_patch_cubin_begin:\n.incbin \"{PATCH_CUBIN}\"\nswb_patch_cubin_end:\n"
+                ".section .note.GNU-stack,\"\",@progbits\n")
+    subprocess.check_call(["gcc", "-c", "-fPIC", "-o", emb_o, emb_s])
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *FLAGS, f'-DSWB_PATCH_CUBIN="{PATCH_CUBIN}"', "-o", tmp, *SOURCES]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
+    subprocess.check_call([NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, obj, emb_o])
+    for f in (obj, emb_s, emb_o):
+        os.remove(f)
     os.replace(tmp, LIB)
     return LIB
 

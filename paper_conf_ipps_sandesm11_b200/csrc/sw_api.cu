@@ -138,7 +138,7 @@ static Variant make_variant()
     v.packed_global_name[0] = 0;
     v.local_wide_fn = v.global_wide_fn = nullptr;
     if constexpr (ALPHA >= 30) {
-        // packed kernel only (15 to 20 slots per lane); int32 work falls back to the default geometry
+        // packed kernel only (15 or 16 slots per lane); int32 work falls back to the default geometry
         constexpr int NS = ALPHA / 2;
         v.packed_fn = (const void *)&sw_fill16_kernel<NW, W, COOP, NS, SPLIT>;
         v.io_warps = COOP ? 0 : 1;
@@ -182,7 +182,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 18;
+static constexpr int NVARIANTS = 14;
 static constexpr int NINT32_VARIANTS = 8;
 // Dynamic shared memory the tail launch requests: more than
 // half an SM's 228 KB, so its CTAs take one SM each as the main launch frees them.
@@ -205,12 +205,6 @@ static const Variant &variant_for(int idx)
         make_variant<32, 16, 64, true>(),
         make_variant<32, 4, 64, false, true>(),  // split F chain (latency-bound one-wave fills)
         make_variant<30, 4, 64>(),  // 3840-row bands: one-wave matrices of up to 148 bands (C2: 142)
-        // taller 8-warp bands (8704 .. 10240 rows): fewer, fuller waves when the
-        // band count is just above a multiple of the CTAs (C4 on 1 or 8 GPUs)
-        make_variant<34, 8, 64>(),
-        make_variant<36, 8, 64>(),
-        make_variant<38, 8, 64>(),
-        make_variant<40, 8, 64>(),
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -273,7 +267,14 @@ struct Peer {
 // instruction) and loads it with cudaLibraryLoadData.  The build checks that
 // every occurrence of the magic words is such a field (build.py).
 
-#if defined(SWB_PATCH_CUBIN) && !defined(__CUDA_ARCH__)
+#if defined(SWB_PATCH_EXTERN) && !defined(__CUDA_ARCH__)
+// the image is embedded by a separate object (build.py: an .incbin of the cubin,
+// assembled and linked next to this one, so both compile in parallel)
+extern "C" const unsigned char swb_patch_cubin_begin[];
+extern "C" const unsigned char swb_patch_cubin_end[];
+static const unsigned char *patch_image() { return swb_patch_cubin_begin; }
+static size_t patch_image_size() { return (size_t)(swb_patch_cubin_end - swb_patch_cubin_begin); }
+#elif defined(SWB_PATCH_CUBIN) && !defined(__CUDA_ARCH__)
 asm(".section .rodata\n"
     ".balign 16\n"
     "swb_patch_cubin_begin:\n"
@@ -807,11 +808,6 @@ static const Candidate kCands[] = {
     {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
     {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
     {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
-    // alpha 34-40 x 8 warps: variant 10's cell rate per SM (36.8 G/s) over the taller band
-    {14, true, 4.49e6 * 32 / 34, 4.49e6 * 32 / 34},
-    {15, true, 4.49e6 * 32 / 36, 4.49e6 * 32 / 36},
-    {16, true, 4.49e6 * 32 / 38, 4.49e6 * 32 / 38},
-    {17, true, 4.49e6 * 32 / 40, 4.49e6 * 32 / 40},
 };
 static constexpr int NCANDS = (int)(sizeof(kCands) / sizeof(kCands[0]));
 // Tail-segment candidates: column speed of one CTA alone on

@@ -25,10 +25,6 @@ template __global__ void sw_fill16_kernel<4, 64, true, 16, false>(const __grid_c
 template __global__ void sw_fill16_kernel<4, 64, false, 15, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<16, 64, true, 16, false>(const __grid_constant__ FillArgs);
-template __global__ void sw_fill16_kernel<8, 64, false, 17, false>(const __grid_constant__ FillArgs);
-template __global__ void sw_fill16_kernel<8, 64, false, 18, false>(const __grid_constant__ FillArgs);
-template __global__ void sw_fill16_kernel<8, 64, false, 19, false>(const __grid_constant__ FillArgs);
-template __global__ void sw_fill16_kernel<8, 64, false, 20, false>(const __grid_constant__ FillArgs);
 // the reverse pass (global mode), variant 10's geometry
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false, false>(const __grid_constant__ FillArgs);
 // Stage-2 partitions (global mode with matching), variant 1's geometry

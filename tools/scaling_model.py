@@ -21,10 +21,6 @@ GEOMS = {  # variant: (band height, CTAs per SM, lag columns, cps_full, cps_solo
     8: (4096, 2, (2 * 4 + 2) * 64, 4.25e6, 7.86e6),
     13: (3840, 2, (2 * 4 + 2) * 64, 4.45e6, 8.17e6),
     10: (8192, 1, (2 * 8 + 2) * 64, 4.49e6, 4.49e6),
-    14: (8704, 1, (2 * 8 + 2) * 64, 4.49e6 * 32 / 34, 4.49e6 * 32 / 34),
-    15: (9216, 1, (2 * 8 + 2) * 64, 4.49e6 * 32 / 36, 4.49e6 * 32 / 36),
-    16: (9728, 1, (2 * 8 + 2) * 64, 4.49e6 * 32 / 38, 4.49e6 * 32 / 38),
-    17: (10240, 1, (2 * 8 + 2) * 64, 4.49e6 * 32 / 40, 4.49e6 * 32 / 40),
 }
 NSM = 148
 CONFIGS = {"C3": (5_000_000, 5_000_000), "C4": (10_000_000, 10_000_000), "C5": (32_799_110, 46_944_323)}
