@@ -110,14 +110,25 @@ struct Variant {
     char packed_name[96];   // mangled name of the packed kernel in the patchable cubin ("" : none)
     const void *packed_global_fn;  // packed kernel in global (reverse-pass) mode, alpha 32 x 8 warps only
     char packed_global_name[96];
+    const void *packed_gen_fn;  // packed kernel with the generic special-row tiles (GEN, sw_fill16.cuh)
+    char packed_gen_name[96];
     const void *local_wide_fn, *global_wide_fn;  // int32 kernels for scorings outside the int8 profile (default geometry)
 };
 
 template <int NW, int W, bool COOP, int NS>
 static void packed_name(Variant &v)
 {
-    snprintf(v.packed_name, sizeof(v.packed_name), "_ZN3swb16sw_fill16_kernelILi%dELi%dELb%dELi%dELb0ELb1EEEvNS_8FillArgsE",
+    snprintf(v.packed_name, sizeof(v.packed_name), "_ZN3swb16sw_fill16_kernelILi%dELi%dELb%dELi%dELb0ELb1ELb0EEEvNS_8FillArgsE",
              NW, W, COOP ? 1 : 0, NS);
+}
+
+// the GEN instantiation (generic special rows) of a packed geometry
+template <int NW, int W, int NS>
+static void packed_gen(Variant &v)
+{
+    v.packed_gen_fn = (const void *)&sw_fill16_kernel<NW, W, false, NS, false, true, true>;
+    snprintf(v.packed_gen_name, sizeof(v.packed_gen_name),
+             "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi%dELb0ELb1ELb1EEEvNS_8FillArgsE", NW, W, NS);
 }
 
 template <int ALPHA, int NW, int W, bool COOP = false, bool SPLIT = false>
@@ -136,6 +147,8 @@ static Variant make_variant()
     v.packed_name[0] = 0;
     v.packed_global_fn = nullptr;
     v.packed_global_name[0] = 0;
+    v.packed_gen_fn = nullptr;
+    v.packed_gen_name[0] = 0;
     v.local_wide_fn = v.global_wide_fn = nullptr;
     if constexpr (ALPHA >= 30) {
         // packed kernel only (15 or 16 slots per lane); int32 work falls back to the default geometry
@@ -144,11 +157,12 @@ static Variant make_variant()
         v.io_warps = COOP ? 0 : 1;
         v.smem16 = Fill16<NW, W, NS, SPLIT>::smem_bytes();
         if constexpr (!SPLIT) packed_name<NW, W, COOP, NS>(v);
+        if constexpr (!SPLIT && !COOP) packed_gen<NW, W, NS>(v);  // variants 8, 10, 13
         if constexpr (ALPHA == 32 && NW == 8 && !COOP && !SPLIT) {
             // the reverse pass (a8) on the packed kernel
             v.packed_global_fn = (const void *)&sw_fill16_kernel<NW, W, false, 16, false, false>;
             snprintf(v.packed_global_name, sizeof(v.packed_global_name),
-                     "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi16ELb0ELb0EEEvNS_8FillArgsE", NW, W);
+                     "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi16ELb0ELb0ELb0EEEvNS_8FillArgsE", NW, W);
         }
         return v;
     } else {
@@ -169,11 +183,12 @@ static Variant make_variant()
         } else {
             v.packed_fn = (const void *)&sw_fill16_kernel<NW, W>;
             packed_name<NW, W, false, 8>(v);
+            if constexpr (NW == 4 || NW == 8) packed_gen<NW, W, 8>(v);  // variants 0, 1
             if constexpr (NW == 8) {
                 // Stage-2 partitions (global mode with matching) on the packed kernel
                 v.packed_global_fn = (const void *)&sw_fill16_kernel<NW, W, false, 8, false, false>;
                 snprintf(v.packed_global_name, sizeof(v.packed_global_name),
-                         "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi8ELb0ELb0EEEvNS_8FillArgsE", NW, W);
+                         "_ZN3swb16sw_fill16_kernelILi%dELi%dELb0ELi8ELb0ELb0ELb0EEEvNS_8FillArgsE", NW, W);
             }
         }
         v.smem16 = Fill16<NW, W>::smem_bytes();
@@ -293,7 +308,7 @@ static size_t patch_image_size() { return 0; }
 struct PatchedSet {
     int ge = -1, gf = -1;
     cudaLibrary_t lib = nullptr;
-    const void *fn[4][NVARIANTS] = {};  // [packed, int32 local, int32 global, packed global][variant]
+    const void *fn[5][NVARIANTS] = {};  // [packed, int32 local, int32 global, packed global, packed GEN][variant]
 };
 
 // Offsets of the magic immediates in the embedded image (computed once).
@@ -489,6 +504,7 @@ static void set_kernel_attrs()
         if (v.packed_fn) cudaFuncSetAttribute(v.packed_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, TAIL_SMEM);
         if (v.packed_global_fn)
             cudaFuncSetAttribute(v.packed_global_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)v.smem16);
+        if (v.packed_gen_fn) cudaFuncSetAttribute(v.packed_gen_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, TAIL_SMEM);
     }
 }
 
@@ -840,10 +856,10 @@ static double model_fill_time(long long nb, long long P, long long n, long long 
 // and the caller runs the runtime-operand kernel (same results).
 static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf, int kind = 0)
 {
-    // kind 0: packed local, 3: packed global (the kernels in the patched image);
-    // 1, 2: int32 local/global (not patched)
-    if ((kind != 0 && kind != 3) || !ctx->patch) return nullptr;
-    const char *name = kind == 0 ? V.packed_name : V.packed_global_name;
+    // kind 0: packed local, 3: packed global, 4: packed local GEN (the kernels in
+    // the patched image); 1, 2: int32 local/global (not patched)
+    if ((kind != 0 && kind != 3 && kind != 4) || !ctx->patch) return nullptr;
+    const char *name = kind == 0 ? V.packed_name : kind == 3 ? V.packed_global_name : V.packed_gen_name;
     if (!name[0]) return nullptr;
     const PatchSites &ps = patch_sites();
     if (!ps.ok) return nullptr;
@@ -886,7 +902,7 @@ static const void *patched_kernel(sw_ctx *ctx, const Variant &V, int ge, int gf,
             return nullptr;
         }
         if (cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)(kind == 0 ? std::max<size_t>(V.smem16, TAIL_SMEM) : kind == 3 ? V.smem16 : V.smem)) != cudaSuccess) {
+                                 (int)(kind == 0 || kind == 4 ? std::max<size_t>(V.smem16, TAIL_SMEM) : kind == 3 ? V.smem16 : V.smem)) != cudaSuccess) {
             cudaGetLastError();
             return nullptr;
         }
@@ -901,11 +917,10 @@ static bool packed_qualifies(const sw_ctx *ctx, const Job &J, const Variant &V)
     const long long pmax_abs = std::max(std::abs(J.ma), std::abs(J.mi));
     const long long span = 32ll * V.alpha + 140;
     // k >= alpha: at most one special row per lane; rows that are not strip
-    // bottoms take the generic special-row tiles (SPM 2, sw_fill16.cuh), except in
-    // the split-F geometry (variant 12: strip bottoms only, k % alpha == 0)
-    const bool split = &V == &variant_for(12);
-    return ctx->packed && J.local && V.packed_fn && (J.k == 0 || (split ? J.k % V.alpha == 0 : J.k >= V.alpha)) &&
-           span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
+    // bottoms take the generic special-row tiles of the GEN instantiation (SPM 2,
+    // sw_fill16.cuh; variants 0, 1, 8, 10, 13)
+    const bool rows_ok = J.k == 0 || J.k % V.alpha == 0 || (J.k >= V.alpha && V.packed_gen_fn);
+    return ctx->packed && J.local && V.packed_fn && rows_ok && span * (pmax_abs + J.go + J.ge) + 1024 < 30000;
 }
 
 static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16, int gpus = 1)
@@ -1003,11 +1018,18 @@ static int setup_seg(sw_ctx *ctx, const Job &J, Seg &G, int P, int NS, bool tail
 {
     const Variant &V = *G.V;
     G.BH = V.alpha * 32 * V.nw;
-    G.fn = G.use16 ? (J.local ? V.packed_fn : V.packed_global_fn)
+    // special rows off the strip bottoms (k not a multiple of alpha, or a segment
+    // starting off a multiple of alpha): the GEN instantiation
+    const bool gen = G.use16 && J.local && J.k > 0 && (J.k % V.alpha != 0 || G.row_base % V.alpha != 0);
+    G.fn = G.use16 ? (J.local ? (gen ? V.packed_gen_fn : V.packed_fn) : V.packed_global_fn)
                    : J.wide ? (J.local ? V.local_wide_fn : V.global_wide_fn) : (J.local ? V.local_fn : V.global_fn);
+    if (!G.fn) {
+        snprintf(ctx->errbuf, sizeof(ctx->errbuf), "no kernel for geometry alpha %d x %d warps (gen %d)", V.alpha, V.nw, gen ? 1 : 0);
+        return SW_EINVAL;
+    }
     G.smem = G.use16 ? V.smem16 : V.smem;
     G.patched = false;
-    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, G.use16 ? (J.local ? 0 : 3) : J.local ? 1 : 2)) {
+    if (const void *pf = patched_kernel(ctx, V, J.ge, J.go + J.ge, G.use16 ? (J.local ? (gen ? 4 : 0) : 3) : J.local ? 1 : 2)) {
         G.fn = pf;
         G.patched = true;
     }
@@ -1050,6 +1072,7 @@ static const Variant *choose_tail(sw_ctx *ctx, const Job &J, const Seg &S0, int 
     if (ctx->tail_mode > 0) {
         const Variant &Vt = variant_for(ctx->tail_mode - 1);
         if (!packed_qualifies(ctx, J, Vt) || Vt.alpha * 32 * Vt.nw >= S0.BH) return nullptr;
+        if (J.k > 0 && ((long long)nb1 * S0.BH) % Vt.alpha != 0 && !Vt.packed_gen_fn) return nullptr;
         *nb1_out = nb1;
         return &Vt;
     }
@@ -1065,6 +1088,7 @@ static const Variant *choose_tail(sw_ctx *ctx, const Job &J, const Seg &S0, int 
         const Variant &Vt = variant_for(C.variant);
         const long long bh = (long long)Vt.alpha * 32 * Vt.nw;
         if (bh >= S0.BH || !packed_qualifies(ctx, J, Vt)) continue;
+        if (J.k > 0 && ((long long)nb1 * S0.BH) % Vt.alpha != 0 && !Vt.packed_gen_fn) continue;
         const long long nb2 = (m2 + bh - 1) / bh;
         if (nb2 > ctx->num_sms) continue;  // the tail must fit in one wave of one CTA per SM
         const long long lagt = (2ll * Vt.nw + 2) * Vt.w;

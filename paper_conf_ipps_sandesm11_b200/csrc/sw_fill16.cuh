@@ -526,7 +526,11 @@ struct Fill16 {
 // recurrence with no 0 floor (FL = 0), global boundaries, first-hit tracking of
 // the goal and the early exit after the band with the first hit, as in the
 // int32 kernel; one stripe, no special rows, no Stage-2 matching (host checks).
-template <int NW, int W, bool COOP = false, int NS = 8, bool SPLIT = false, bool LOCAL = true>
+// GEN = true: also the generic special-row tiles (SPM 2: a special row that is
+// not a strip bottom -- k not a multiple of alpha, or a tail segment whose first
+// row is not); a separate instantiation, so the strip-bottom kernels keep their
+// code (the generic tiles cost the GEN kernel ~2 % on C4).
+template <int NW, int W, bool COOP = false, int NS = 8, bool SPLIT = false, bool LOCAL = true, bool GEN = false>
 __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(const __grid_constant__ FillArgs a)
 {
     using F = Fill16<NW, W, NS, SPLIT, LOCAL>;
@@ -655,7 +659,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 }
             }
             warp_sp = __any_sync(0xffffffffu, sp_r >= 0);
-            warp_sp2 = !SPLIT && __any_sync(0xffffffffu, sp_r >= 0 && sp_r != ALPHA - 1);
+            warp_sp2 = GEN && !SPLIT && __any_sync(0xffffffffu, sp_r >= 0 && sp_r != ALPHA - 1);
         }
 
         auto io_load = [&](int c) {
@@ -812,7 +816,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     uint32_t tm;
                     const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
                     if (cap) {
-                        tm = warp_sp2 ? F::template tile<true, false, 2, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                        tm = warp_sp2 ? F::template tile<true, false, GEN ? 2 : 1, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                            : warp_sp ? F::template tile<true, false, 1, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                                      : F::template tile<true, false, 0, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                         if (c == cap_t1) {
@@ -821,11 +825,11 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                             if (lane == 0 && S.rready != nullptr) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
                         }
                     } else if (c == 0) {
-                        tm = warp_sp2 ? F::template tile<true, false, 2, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                        tm = warp_sp2 ? F::template tile<true, false, GEN ? 2 : 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                            : warp_sp ? F::template tile<true, false, 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                                      : F::template tile<true, false, 0, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else if (warp_sp2) {
-                        tm = F::template tile<false, false, 2, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
+                        tm = F::template tile<false, false, GEN ? 2 : 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else if (warp_sp) {
                         tm = F::template tile<false, false, 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else {

@@ -73,6 +73,7 @@ def test_packed_falls_back_when_not_applicable(ctx):
 
 
 ALPHA = {0: 16, 1: 16, 3: 16, 5: 16, 6: 16, 8: 32, 9: 32, 10: 32, 11: 32, 12: 32, 13: 30}
+GEN = {0, 1, 8, 10, 13}  # geometries with the generic special-row instantiation
 
 
 @pytest.mark.parametrize("variant", [0, 1, 5, 8, 10, 13])
@@ -83,7 +84,7 @@ def test_packed_any_special_row_interval(ctx, variant, k):
     from whichever slot and half holds it; every row against the oracle.  k <
     alpha (several rows per lane) runs the int32 kernel."""
     A, B = synth.random_pair(30 + variant + k, 9000, 1300, plant_len=1000, s=0.05, g=0.01)
-    check(ctx, A, B, PAPER, k, variant, expect_packed=k >= ALPHA[variant])
+    check(ctx, A, B, PAPER, k, variant, expect_packed=k % ALPHA[variant] == 0 or (k >= ALPHA[variant] and variant in GEN))
 
 
 def test_packed_ties_and_long_alignment(ctx):
@@ -110,7 +111,7 @@ def test_packed_alpha32(ctx, variant):
     check(ctx, A, B, PAPER, 96, variant)
     check(ctx, A, B, (5, -4, 10, 1), 64, variant)
     check(ctx, A, B, PAPER, 16, variant, expect_packed=False)  # k < alpha: two rows per lane, int32
-    check(ctx, A, B, PAPER, 48, variant, expect_packed=variant != 12)  # k % alpha != 0: generic rows
+    check(ctx, A, B, PAPER, 48, variant, expect_packed=variant in GEN)  # k % alpha != 0: generic rows (GEN)
     X = synth.random_pair(4, 500, 1)[0]
     check(ctx, np.concatenate([X, X, X, X]), X, PAPER, 32, variant)
     check(ctx, A, B, PAPER, 32, variant, stripes=3)
@@ -131,7 +132,8 @@ def test_packed_alpha30(ctx):
     for scoring in (PAPER, (2, -1, 4, 1), (1, -1, 0, 2), (5, -4, 10, 1), (3, -2, 0, 1)):
         check(ctx, A, B, scoring, 3840, 13)
     check(ctx, A, B, PAPER, 90, 13)
-    check(ctx, A, B, PAPER, 32, 13, expect_packed=False)  # k not a multiple of 30: int32 kernel
+    check(ctx, A, B, PAPER, 32, 13)  # k not a multiple of 30: the GEN instantiation (generic special rows)
+    check(ctx, A, B, PAPER, 29, 13, expect_packed=False)  # k < alpha: int32 kernel
     check(ctx, A, B, PAPER, 60, 13, stripes=3)
     X = synth.random_pair(5, 500, 1)[0]
     check(ctx, np.concatenate([X, X, X, X]), X, PAPER, 30, 13)
