@@ -12,6 +12,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <thread>
+#include <unistd.h>
 #include <vector>
 
 #include "../../include/cudalign_b200.h"
@@ -1283,6 +1284,12 @@ static int run_job(sw_ctx *ctx, const Job &J0, cudaStream_t user_stream, int4 *r
             R = nsp;
         }
         store = (R < nsp || multi) && NS == 1 && !J.rank_mode && !rcyc;
+        if (store) {
+            // the host store (the SRA) may take at most half the physical memory:
+            // a larger one would page the host out (Stage 2 then refuses: SW_EINVAL)
+            const double phys = (double)sysconf(_SC_PHYS_PAGES) * (double)sysconf(_SC_PAGE_SIZE);
+            if ((double)nsp * 8.0 * (double)n > 0.5 * phys) store = false;
+        }
         for (int u = 0; u < NU; u++) {
             CK(setdev(udev[u]));
             if ((rc = grow(ctx, ctx->sp[u], (size_t)R * stride[u] * sizeof(int)))) return rc;
