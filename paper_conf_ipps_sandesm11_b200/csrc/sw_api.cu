@@ -980,10 +980,7 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16, int
         const long long bh = (long long)V.alpha * 32 * V.nw;
         const long long nb = std::max<long long>(1, (J.m + bh - 1) / bh);
         const double cps = nb <= (long long)ctx->num_sms * gpus ? C.cps_solo : C.cps_full;
-        // band lag: warps skewed two intervals, border load one ahead, drain one
-        // behind; the packed I/O-warp kernels with >= 8 warps run 2 tiles per interval
-        const long long ipt = (C.packed && V.io_warps == 1 && V.nw >= 8) ? 2 : 1;
-        double t = model_fill_time(nb, P, std::max<long long>(J.n, 1), (2ll * V.nw + 2) * V.w * ipt, cps);
+        double t = model_fill_time(nb, P, std::max<long long>(J.n, 1), (2ll * V.nw + 2) * V.w, cps);
         // special rows that are not band bottoms are written by the compute
         // warps (SP1 tiles) instead of the I/O warp: measured +7.7 % on C2
         // (variant 8 at k = 3840 vs 4096, profiles/r01_fill_a30.txt)

@@ -57,12 +57,6 @@ constexpr int BIAS16 = 32768;
 #ifndef SWB_UNR
 #define SWB_UNR 0
 #endif
-// Tiles per lockstep interval of the I/O-warp kernels (one __syncthreads per
-// interval; the warp skew is 2 intervals): 2 halves the barriers and evens out
-// the per-interval imbalance between a SMSP's two compute warps.
-#ifndef SWB_IPT
-#define SWB_IPT 2
-#endif
 
 
 __device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(lo & 0xffff) | ((uint32_t)hi << 16); }
@@ -83,12 +77,7 @@ template <int NW, int W, int NS = 8, bool SPLIT = false, bool LOCAL = true>
 struct Fill16 {
     static constexpr int ALPHA = 2 * NS, BH = ALPHA * 32 * NW;
     static constexpr int RING = Smem<W, NW>::RING;
-    // selector ring: spans the warp skew of up to SWB_IPT tiles per interval
-    // (the I/O warp loads the next interval's tiles while the last warp is
-    // 2 (NW - 1) intervals behind), rounded up to a power of two
-    static constexpr int IPT_IO = NW >= 8 ? SWB_IPT : 1;  // one-wave 4-warp fills keep the short band lag
-    static constexpr int SRING_MIN16 = (2 * IPT_IO * (NW - 1) + 2 * IPT_IO) * W + 128;
-    static constexpr int SRING = SRING_MIN16 <= 1024 ? 1024 : SRING_MIN16 <= 2048 ? 2048 : SRING_MIN16 <= 4096 ? 4096 : 8192;
+    static constexpr int SRING = Smem<W, NW>::SRING;
     static constexpr int SKEW = 63;     // lane 31's output column lags lane 0's by 2*31 + 1
     static constexpr int STEPS = W;     // one column per lane step
     static constexpr int UNR = SWB_UNR > 0 ? SWB_UNR : (LOCAL && (NW >= 8 || NS == 15)) ? 8 : 4;
@@ -784,7 +773,6 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             }
         };
 
-        constexpr int IPT = COOP ? 1 : F::IPT_IO;  // tiles per interval (I/O-warp kernels with >= 8 compute warps)
         if constexpr (COOP) {
             coop_wait(0);
             if (lane < CPW) {
@@ -794,11 +782,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 coop_put(0, v, code);
             }
         } else {
-            if (warp == NW)
-                for (int u = 0; u < IPT && u < NT; u++) io_load(u);
+            if (warp == NW) io_load(0);
         }
         __syncthreads();
-        const int S_END = (NT + IPT - 1) / IPT + 2 * (NW - 1);
+        const int S_END = NT + 2 * (NW - 1);
         int *sv = saves + warp * F::NSAVE * 32;
         for (int s = 0; s < S_END + 1; ++s) {
             int2 fv = make_int2(0, 0);
@@ -810,9 +797,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                 }
             }
             if (warp < NW) {
-#pragma unroll 1
-              for (int u = 0; u < IPT; u++) {
-                const int c = IPT * (s - 2 * warp) + u;
+                const int c = s - 2 * warp;
                 if (c >= 0 && c < NT) {
                     const uint32_t rin = pin((uint32_t)__cvta_generic_to_shared(crings + warp * W));
                     const uint32_t rout = pin((uint32_t)__cvta_generic_to_shared(rings + (warp + 1) * F::RS));
@@ -865,16 +850,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                         }
                     }
                 }
-              }
             } else {
-                for (int u = 0; u < IPT; u++) {
-                    const int t = IPT * (s + 1) + u;
-                    if (t < NT) io_load(t);
-                }
-                for (int u = 0; u < IPT; u++) {
-                    const int cd = IPT * (s - 1 - 2 * (NW - 1)) + u;
-                    if (cd >= 0 && cd < NT) io_drain(cd);
-                }
+                if (s + 1 < NT) io_load(s + 1);
+                const int cd = s - 1 - 2 * (NW - 1);
+                if (cd >= 0) io_drain(cd);
                 if (!LOCAL && lane == 0 && ld_relaxed(a.hit_band) < b) s_abort = 1;
             }
             const int cdc = s - 1 - 2 * (NW - 1);
