@@ -237,10 +237,10 @@ int64_t sw_band_height(const sw_ctx *ctx);
 /* Kernel selection (testing / tuning).  variant = -1: automatic choice per
  * call; 0..7: a fixed geometry (alpha, warps, tile width) of
  * the int32 kernel (DESIGN.md 4.1 lists them), or of the packed 16x2 kernel when packed = 1 and the call
- * qualifies (local mode, k % alpha == 0, small value window); 8..13: packed-only
- * geometries (alpha 32, or alpha 30 for 13) that fall back to the default int32
+ * qualifies (local mode, k % alpha == 0, small value window); 8..14: packed-only
+ * geometries (alpha 32; 30 for 13; 34 x 8 warps for 14) that fall back to the default int32
  * geometry when the call does not qualify.  packed = 0 never uses the packed
- * kernel.  Results are identical for every choice.  SW_EINVAL outside -1..13. */
+ * kernel.  Results are identical for every choice.  SW_EINVAL outside -1..14. */
 int sw_set_kernel(sw_ctx *ctx, int variant, int packed);
 
 /* Immediate patching of the packed kernel (testing / tuning; default on).
@@ -265,7 +265,7 @@ int sw_set_grid(sw_ctx *ctx, int ctas);
  * shorter band height, if the band-pipeline model says it is faster; 0: never;
  * v + 1 (v a packed geometry of sw_set_kernel with a shorter band): always
  * that geometry when the fill has a partial last wave.  Results are identical.
- * SW_EINVAL outside -1 .. 14. */
+ * SW_EINVAL outside -1 .. 15. */
 int sw_set_tail(sw_ctx *ctx, int mode);
 
 /* Device-memory budget of the special-row ring in bytes (testing / tuning;

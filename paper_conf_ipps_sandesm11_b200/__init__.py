@@ -401,7 +401,7 @@ class Context:
         return int(self._lib.sw_band_height(self._h))
 
     def set_kernel(self, variant: int = -1, packed: bool = True):
-        """variant -1: automatic; 0..13: fixed geometry (8..13 packed-only); packed: allow the 16x2 kernel."""
+        """variant -1: automatic; 0..14: fixed geometry (8..14 packed-only); packed: allow the 16x2 kernel."""
         self._check(self._lib.sw_set_kernel(self._h, variant, int(bool(packed))), "sw_set_kernel")
 
     def set_patch(self, on: bool = True):

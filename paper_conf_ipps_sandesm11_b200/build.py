@@ -38,7 +38,7 @@ def stale() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS)
 
 
-def check_patch_sites(path: str) -> dict:
+def check_patch_sites(path: str, required=("NGE2", "NGE16", "NGF16")) -> dict:
     """Every occurrence of a magic word in the cubin must be a 32-bit
     instruction immediate (byte 4 of a 16-byte SASS instruction); the loader
     (sw_api.cu patch_sites) refuses to patch otherwise."""
@@ -65,22 +65,32 @@ def check_patch_sites(path: str) -> dict:
         if data.find(struct.pack("<I", (-v) & 0xFFFFFFFF)) >= 0:
             raise RuntimeError(f"{path}: the negation of magic {name} occurs (an unpatchable form)")
         counts[name] = len(offs)
-    for name in ("NGE2", "NGE16", "NGF16"):
+    for name in required:
         if counts[name] == 0:
             raise RuntimeError(f"{path}: magic {name} not found (ptxas folded it?)")
     return counts
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defs: list | None = None, out_dir: str | None = None) -> str:
+    """Build the library.  ``defs`` (extra -D flags) and ``out_dir`` (where the
+    library and its cubin go) serve A/B experiments (tools/build_variant.py);
+    the product build uses neither."""
+    global LIB, PATCH_CUBIN
+    if out_dir:
+        os.makedirs(out_dir, exist_ok=True)
+        LIB = os.path.join(out_dir, "libcudalign_b200.so")
+        PATCH_CUBIN = os.path.join(out_dir, "sw_fill16_patch.cubin")
+        force = True
     if not force and not stale():
         return LIB
+    defs = list(defs or [])
     # in parallel: the patchable cubin twice (the magic set used at run time and
     # an alternative set; the SASS must agree up to the magic words,
     # patch_check.py) and the library's object; then the embedding object and the link
     ptmp = PATCH_CUBIN + f".tmp{os.getpid()}"
     palt = PATCH_CUBIN + f".alt{os.getpid()}"
     obj = LIB[:-3] + f".{os.getpid()}.o"  # nvcc picks the input kind by extension
-    cflags = [f for f in FLAGS if f not in ("-Xcompiler", "-fPIC", "-shared")]
+    cflags = [f for f in FLAGS if f not in ("-Xcompiler", "-fPIC", "-shared")] + defs
     alt = [f"-DSWB_K_{k}={v:#x}u" for k, v in zip(MAGIC, ALT_MAGIC)]
     ocmd = [NVCC, *cflags, "-Xcompiler", "-fPIC", "-DSWB_PATCH_EXTERN", "-c", "-o", obj, *SOURCES]
     if verbose:
@@ -91,7 +101,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
              subprocess.Popen(ocmd)]
     if any([p.wait() for p in procs]):
         raise RuntimeError("nvcc failed")
-    check_patch_sites(ptmp)
+    check_patch_sites(ptmp, ("NGE2", "NGE16", "NGF16") if not defs else ("NGE2",))
     from . import patch_check
 
     if patch_check.main(ptmp, palt):

@@ -158,7 +158,7 @@ static Variant make_variant()
         v.io_warps = COOP ? 0 : 1;
         v.smem16 = Fill16<NW, W, NS, SPLIT>::smem_bytes();
         if constexpr (!SPLIT) packed_name<NW, W, COOP, NS>(v);
-        if constexpr (!SPLIT && !COOP) packed_gen<NW, W, NS>(v);  // variants 8, 10, 13
+        if constexpr (!SPLIT && !COOP) packed_gen<NW, W, NS>(v);  // variants 8, 10, 13, 14
         if constexpr (ALPHA == 32 && NW == 8 && !COOP && !SPLIT) {
             // the reverse pass (a8) on the packed kernel
             v.packed_global_fn = (const void *)&sw_fill16_kernel<NW, W, false, 16, false, false>;
@@ -198,7 +198,7 @@ static Variant make_variant()
 }
 
 static constexpr int DEFAULT_VARIANT = 1;  // (alpha 16, 8 warps, W 64): fastest on C2/C3
-static constexpr int NVARIANTS = 14;
+static constexpr int NVARIANTS = 15;
 static constexpr int NINT32_VARIANTS = 8;
 // Dynamic shared memory the tail launch requests: more than
 // half an SM's 228 KB, so its CTAs take one SM each as the main launch frees them.
@@ -221,6 +221,7 @@ static const Variant &variant_for(int idx)
         make_variant<32, 16, 64, true>(),
         make_variant<32, 4, 64, false, true>(),  // split F chain (latency-bound one-wave fills)
         make_variant<30, 4, 64>(),  // 3840-row bands: one-wave matrices of up to 148 bands (C2: 142)
+        make_variant<34, 8, 64>(),  // 8704-row bands: C4 as one wave of 8 x 148 CTAs (band-cyclic)
     };
     return vs[idx < 0 ? 0 : idx >= NVARIANTS ? NVARIANTS - 1 : idx];
 }
@@ -825,6 +826,7 @@ static const Candidate kCands[] = {
     {10, true, 4.49e6, 4.49e6},                // packed alpha 32, 8 warps + I/O warp
     {5, true, 4.03e6, 4.03e6},                 // packed alpha 16, 15 warps + I/O warp
     {6, true, 3.87e6, 3.87e6},                 // packed alpha 16, 16 warps, cooperative I/O
+    {14, true, 4.49e6 * 32 / 34, 4.49e6 * 32 / 34},  // packed alpha 34, 8 warps + I/O warp
 };
 static constexpr int NCANDS = (int)(sizeof(kCands) / sizeof(kCands[0]));
 // Tail-segment candidates: column speed of one CTA alone on

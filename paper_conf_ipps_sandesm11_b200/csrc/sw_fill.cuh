@@ -130,6 +130,8 @@ struct StepInfo {
     int jcap;            // local column whose (t, E) goes to the right neighbour
     int2 *rbrow;         // right-border destination for this lane's first row
     int hw;              // columns eligible for tracking (w, or the Stage-2 start-check width)
+    int splane;          // packed GEN kernel, SPM 3: the warp's one lane with a special row
+    uint32_t spb;        // ... and the warp's staging buffer (shared, 128 x uint2) for it
 };
 
 __device__ __forceinline__ unsigned long long gtimer()

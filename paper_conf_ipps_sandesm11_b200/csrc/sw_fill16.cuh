@@ -57,6 +57,13 @@ constexpr int BIAS16 = 32768;
 #ifndef SWB_UNR
 #define SWB_UNR 0
 #endif
+// Lane steps per iteration in the special-row tiles (SPM 1 / 2 / 3); 0: as SWB_UNR's
+// rule.  4: the warp with a special row runs a different loop than its CTA's other
+// warps; a shorter body keeps both hot loops in the instruction cache (C4, alpha 34,
+// k = 131072: 21.4 -> 19.9 s; profiles/r02_spm3.txt).
+#ifndef SWB_SPU
+#define SWB_SPU 4
+#endif
 
 
 __device__ __forceinline__ uint32_t pk(int lo, int hi) { return (uint32_t)(lo & 0xffff) | ((uint32_t)hi << 16); }
@@ -82,6 +89,7 @@ struct Fill16 {
     static constexpr int STEPS = W;     // one column per lane step
     static constexpr int UNR = SWB_UNR > 0 ? SWB_UNR : (LOCAL && (NW >= 8 || NS == 15)) ? 8 : 4;
     static constexpr int NSAVE = 2 * NS + 3;
+    static constexpr int SPB = 128;  // SPM 3 staging entries per warp (two tiles of columns)
     static constexpr int HALF = SRING / 2 + 32;  // selector ring: one parity half + a 32-entry mirror
     // Warp-to-warp rings of (t, F): column col lives at ridx(col) in [1, RING]
     // (stride RS = RING + 1), so the 64 columns k0 - 63 .. k0 a lane-31 tile
@@ -96,7 +104,7 @@ struct Fill16 {
     static size_t smem_bytes()
     {
         return sizeof(int2) * RS * (NW + 1) + sizeof(uint32_t) * 2 * HALF + sizeof(uint32_t) * NW * W +
-               sizeof(int) * NSAVE * 32 * NW;
+               sizeof(int) * NSAVE * 32 * NW + sizeof(uint2) * SPB * NW;
     }
 
     struct Lane {
@@ -175,15 +183,21 @@ struct Fill16 {
             if constexpr (SWB_FMODE == 1 || TRACK) {
                 h = __vmaxu2(d, fu);
                 t = (uint32_t)imad((int)h, one, ngf2);
+            } else if constexpr (SWB_FMODE >= 3) {
+                // t = max(F - G_first, D - G_first) as an FMA-pipe add and a
+                // full-rate max (one ALU cycle instead of two)
+                t = __vmaxu2(add_fma(fu, one, ngf2), dg);
+                h = t;
             } else {
                 t = __viaddmax_u16x2(fu, ngf16, dg);
                 h = t;
             }
-            fu = __viaddmax_u16x2(fu, nge16, dg);
+            if constexpr (SWB_FMODE == 4 && !TRACK) fu = __vmaxu2(add_fma(fu, one, nge2), dg);
+            else fu = __viaddmax_u16x2(fu, nge16, dg);
         }
     }
     // Offset from the tile maximum a non-replay tile returns to H (mode 2: t).
-    static __device__ __forceinline__ int tmax_off(const FillArgs &a) { return SWB_FMODE == 2 && !SPLIT ? a.gf : 0; }
+    static __device__ __forceinline__ int tmax_off(const FillArgs &a) { return SWB_FMODE >= 2 && !SPLIT ? a.gf : 0; }
 
     // SPM: 0 no special row in the warp; 1 special rows are strip bottoms (the
     // high half of the last slot); 2 one special row per lane anywhere in the
@@ -192,13 +206,20 @@ struct Fill16 {
     // segment whose first row is not a multiple of alpha, or k not a multiple of
     // alpha.  The slot loop only selects that slot's (t, F) (two SELs per slot);
     // one store pair after the loop.
-    template <bool GUARD, bool TRACK, int SPM, bool CAP>
+    // SPM 3: as SPM 2 for a warp with exactly one such lane (X.splane, k >= 32
+    // alpha): that lane stages the packed (t, F) pair in shared memory (X.spb,
+    // one STS per step) and the warp writes the tile's columns coalesced after
+    // the tile (sw_fill16_kernel sp_flush) instead of two guarded global stores
+    // per step.  SPS >= 0 (SPM 2 / 3): the special row's slot is SPS in every
+    // lane that has one (warp-uniform, known at compile time), so the capture is
+    // two register moves at that slot instead of a compare and two selects per slot.
+    template <bool GUARD, bool TRACK, int SPM, bool CAP, int SPS = -1>
     static __device__ __forceinline__ uint32_t step(const FillArgs &a, const StepInfo &X, Lane &L, int k, int lane,
                                                     uint32_t cr_a, uint32_t ro_a, uint32_t sel_a, uint32_t pt_sel,
                                                     int one, uint32_t tmax, int row1, int &bs, int &bi, int &bj,
                                                     int *sp_ptr, int sp_r)
     {
-        const int sp_s = sp_r < NS ? sp_r : sp_r - NS;  // the slot of the lane's special row (SPM 2)
+        const int sp_s = SPS >= 0 ? SPS : sp_r < NS ? sp_r : sp_r - NS;  // the slot of the lane's special row (SPM 2)
         uint32_t sp_t = 0u, sp_f = 0u;
         const uint32_t up_t = __shfl_up_sync(0xffffffffu, L.t[NS - 1], 1);
         const uint32_t up_f = __shfl_up_sync(0xffffffffu, L.fn, 1);
@@ -297,7 +318,7 @@ struct Fill16 {
                 cell_hf<TRACK>(d0, fu, h0, t0, one, nge2, ngf2, nge16, ngf16);
                 L.e[s] = e0;
                 L.t[s] = t0;
-                if (SPM == 2 && !TRACK && s == sp_s) { sp_t = t0; sp_f = fin0; }
+                if (SPM >= 2 && !TRACK && (SPS >= 0 ? s == SPS : s == sp_s)) { sp_t = t0; sp_f = fin0; }
                 if (s + 1 == NS) {
                     tmax = __vmaxu2(tmax, h0);
                     if (CAP) {
@@ -316,7 +337,7 @@ struct Fill16 {
                 cell_hf<TRACK>(d1, fu, h1, t1, one, nge2, ngf2, nge16, ngf16);
                 L.e[s + 1] = e1;
                 L.t[s + 1] = t1;
-                if (SPM == 2 && !TRACK && s + 1 == sp_s) { sp_t = t1; sp_f = fin1; }
+                if (SPM >= 2 && !TRACK && (SPS >= 0 ? s + 1 == SPS : s + 1 == sp_s)) { sp_t = t1; sp_f = fin1; }
                 tmax = __vimax3_u16x2(tmax, h0, h1);  // TRACK: this step's maximum (reset per step)
                 if (CAP) {
                     if (jl == X.jcap) {
@@ -412,6 +433,9 @@ struct Fill16 {
                 sp_ptr[X.sp_ld + col] = toabs(L, hi ? hi16(sp_f) : lo16(sp_f));
             }
         }
+        if (SPM == 3 && lane == X.splane)
+            asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(X.spb + 8u * ((uint32_t)jl & (SPB - 1))), "r"(sp_t), "r"(sp_f)
+                         : "memory");
         if (SPM == 1 && sp_ptr != nullptr && jo >= 0 && jo < X.w) {
             sp_ptr[jo] = toabs(L, hi16(L.t[NS - 1])) + a.gf;  // H = t + G_first
             sp_ptr[X.sp_ld + jo] = toabs(L, hi16(f15));
@@ -438,7 +462,7 @@ struct Fill16 {
         __syncwarp();
     }
 
-    template <bool GUARD, bool TRACK, int SPM, bool CAP>
+    template <bool GUARD, bool TRACK, int SPM, bool CAP, int SPS = -1>
     static __device__ __forceinline__ uint32_t tile(const FillArgs &a, const StepInfo &X, Lane &L, int c, int lane,
                                                     uint32_t cring, uint32_t ring_out, uint32_t selr, int row1,
                                                     int &bs, int &bi, int &bj, int *sp_ptr, int sp_r)
@@ -458,17 +482,35 @@ struct Fill16 {
                                                     sel0 + 4u * ((kk >> 1) + (kk & 1) * HALF), pt_sel, one, tmax,
                                                     row1, bs, bi, bj, sp_ptr, sp_r);
         } else {
+            // special-row tiles run next to the other warps' SPM-0 loop: a shorter
+            // body keeps both hot loops in the instruction cache (SWB_SPU)
+            constexpr int U = SPM == 0 ? UNR : (SWB_SPU > 0 ? SWB_SPU : UNR);
 #pragma unroll 1
-            for (int kq = 0; kq < STEPS; kq += UNR) {
+            for (int kq = 0; kq < STEPS; kq += U) {
                 const uint32_t sq = sel0 + 2u * kq, cq = cring + 4u * kq, oq = ro0 + 8u * kq;
 #pragma unroll
-                for (int u = 0; u < UNR; u++)
-                    tmax = step<false, false, SPM, false>(a, X, L, k0 + kq + u, lane, cq + 4u * u, oq + 8u * u,
+                for (int u = 0; u < U; u++)
+                    tmax = step<false, false, SPM, false, SPS>(a, X, L, k0 + kq + u, lane, cq + 4u * u, oq + 8u * u,
                                                           sq + 4u * ((u >> 1) + (u & 1) * HALF), pt_sel, one, tmax,
                                                           row1, bs, bi, bj, sp_ptr, sp_r);
             }
         }
         return tmax;
+    }
+
+    // The fast SPM-3 tile with the special row's slot sps as a compile-time
+    // constant: one instantiation per slot.
+    template <int S = 0>
+    static __device__ __forceinline__ uint32_t tile_gen(int sps, const FillArgs &a, const StepInfo &X, Lane &L, int c,
+                                                        int lane, uint32_t cring, uint32_t ring_out, uint32_t selr,
+                                                        int row1, int &bs, int &bi, int &bj, int *sp_ptr, int sp_r)
+    {
+        if constexpr (S < NS) {
+            if (sps == S) return tile<false, false, 3, false, S>(a, X, L, c, lane, cring, ring_out, selr, row1, bs, bi, bj, sp_ptr, sp_r);
+            return tile_gen<S + 1>(sps, a, X, L, c, lane, cring, ring_out, selr, row1, bs, bi, bj, sp_ptr, sp_r);
+        } else {
+            return tile<false, false, 3, false>(a, X, L, c, lane, cring, ring_out, selr, row1, bs, bi, bj, sp_ptr, sp_r);
+        }
     }
 
     // Re-base the frame to lane 0's slot-0 low value (warp-uniform shift).
@@ -541,6 +583,7 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
     uint32_t *selr = reinterpret_cast<uint32_t *>(rings + (NW + 1) * F::RS);
     uint32_t *crings = selr + 2 * F::HALF;
     int *saves = reinterpret_cast<int *>(crings + NW * W);
+    uint2 *spbuf = reinterpret_cast<uint2 *>(saves + F::NSAVE * 32 * NW);  // SPM 3 staging, F::SPB per warp
     __shared__ int s_band, s_abort;
 
     const int warp = threadIdx.x >> 5, lane = lane_id();
@@ -590,6 +633,10 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
         int *sp_ptr = nullptr;
         int sp_r = -1;  // this lane's special row within its strip (-1: none)
         bool warp_sp = false, warp_sp2 = false;
+        // a warp with one special lane (SPM 3): its slot, half (row >= NS) and row pointer
+        int warp_sps = -1, warp_sphi = 0;
+        int band_sps = -1;  // GEN, k >= BH: the slot of the band's one special row (every warp's tile_gen)
+        int *warp_spp = nullptr;
         X.rbrow = has_right ? S.rb + row0 + 1 : nullptr;
         auto init_state = [&](bool from_left) {
             // state at the column left of the stripe: the column-0 boundary or the left border
@@ -660,6 +707,31 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
             }
             warp_sp = __any_sync(0xffffffffu, sp_r >= 0);
             warp_sp2 = GEN && !SPLIT && __any_sync(0xffffffffu, sp_r >= 0 && sp_r != ALPHA - 1);
+            warp_sps = -1;
+            X.splane = -1;
+            band_sps = -1;
+            if (GEN && !SPLIT && a.k >= BH) {
+                // k >= BH: at most one special row inside the band (its bottom row is
+                // the I/O warp's): every warp runs the staged tiles of its slot, so
+                // the SM keeps one hot loop (only the owning lane stores)
+                const long long row = (((long long)rowtop + a.k) / a.k) * a.k;
+                if (row < (long long)rowtop + BH && row <= a.m) {
+                    const int r = (int)(row - rowtop - 1) % ALPHA;
+                    band_sps = r < NS ? r : r - NS;
+                }
+            }
+            if (GEN && warp_sp && !SPLIT) {
+                const unsigned bal = __ballot_sync(0xffffffffu, sp_r >= 0);
+                if (__popc(bal) == 1) {  // k >= 32 alpha: one lane (SPM 3)
+                    const int sl = __ffs(bal) - 1;
+                    const int r = __shfl_sync(0xffffffffu, sp_r, sl);
+                    warp_sps = r < NS ? r : r - NS;
+                    warp_sphi = r < NS ? 0 : 1;
+                    warp_spp = reinterpret_cast<int *>(__shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(sp_ptr), sl));
+                    X.splane = sl;
+                    X.spb = (uint32_t)__cvta_generic_to_shared(spbuf + warp * F::SPB);
+                }
+            }
         }
 
         auto io_load = [&](int c) {
@@ -816,7 +888,8 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                     uint32_t tm;
                     const bool cap = has_right && c >= cap_t0 && c <= cap_t1;
                     if (cap) {
-                        tm = warp_sp2 ? F::template tile<true, false, GEN ? 2 : 1, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                        tm = (GEN && warp_sps >= 0) ? F::template tile<true, false, 3, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                           : warp_sp2 ? F::template tile<true, false, GEN ? 2 : 1, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                            : warp_sp ? F::template tile<true, false, 1, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                                      : F::template tile<true, false, 0, true>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                         if (c == cap_t1) {
@@ -825,9 +898,13 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                             if (lane == 0 && S.rready != nullptr) st_release_sys_s32(S.rready + b * NW + warp, a.epoch);
                         }
                     } else if (c == 0) {
-                        tm = warp_sp2 ? F::template tile<true, false, GEN ? 2 : 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                        tm = (GEN && warp_sps >= 0) ? F::template tile<true, false, 3, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
+                           : warp_sp2 ? F::template tile<true, false, GEN ? 2 : 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                            : warp_sp ? F::template tile<true, false, 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r)
                                      : F::template tile<true, false, 0, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
+                    } else if (GEN && (band_sps >= 0 || warp_sps >= 0)) {
+                        // one special lane: staged (SPM 3), the slot a compile-time constant
+                        tm = F::tile_gen(band_sps >= 0 ? band_sps : warp_sps, a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else if (warp_sp2) {
                         tm = F::template tile<false, false, GEN ? 2 : 1, false>(a, X, L, c, lane, rin, rout, selr_s, row0 + 1, bs, bi, bj, sp_ptr, sp_r);
                     } else if (warp_sp) {
@@ -847,6 +924,20 @@ __global__ void __launch_bounds__((NW + (COOP ? 0 : 1)) * 32) sw_fill16_kernel(c
                         } else if (bi != obi || bj != obj) {
                             atomicMin(a.hit_key, ((unsigned long long)(unsigned)bi << 32) | (unsigned)bj);
                             atomicMin(a.hit_band, b);
+                        }
+                    }
+                    if (GEN && warp_sps >= 0) {
+                        // SPM 3: the special lane's columns of this tile (staged
+                        // in the tile's frame), coalesced
+                        __syncwarp();
+#pragma unroll
+                        for (int x = lane; x < STEPS; x += 32) {
+                            const int jl = c * STEPS + x - 2 * X.splane, col = jl - warp_sphi;
+                            if (col >= 0 && col < X.w) {
+                                const uint2 v = spbuf[warp * F::SPB + (jl & (F::SPB - 1))];
+                                __stcg(warp_spp + col, F::toabs(L, warp_sphi ? hi16(v.x) : lo16(v.x)) + a.gf);  // H = t + G_first
+                                __stcg(warp_spp + X.sp_ld + col, F::toabs(L, warp_sphi ? hi16(v.y) : lo16(v.y)));
+                            }
                         }
                     }
                 }

@@ -25,12 +25,14 @@ template __global__ void sw_fill16_kernel<4, 64, true, 16, false>(const __grid_c
 template __global__ void sw_fill16_kernel<4, 64, false, 15, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<16, 64, true, 16, false>(const __grid_constant__ FillArgs);
-// the GEN instantiations (generic special rows): variants 0, 1, 8, 10, 13
+template __global__ void sw_fill16_kernel<8, 64, false, 17, false>(const __grid_constant__ FillArgs);
+// the GEN instantiations (generic special rows): variants 0, 1, 8, 10, 13, 14
 template __global__ void sw_fill16_kernel<4, 64, false, 8, false, true, true>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<8, 64, false, 8, false, true, true>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<4, 64, false, 16, false, true, true>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false, true, true>(const __grid_constant__ FillArgs);
 template __global__ void sw_fill16_kernel<4, 64, false, 15, false, true, true>(const __grid_constant__ FillArgs);
+template __global__ void sw_fill16_kernel<8, 64, false, 17, false, true, true>(const __grid_constant__ FillArgs);
 // the reverse pass (global mode), variant 10's geometry
 template __global__ void sw_fill16_kernel<8, 64, false, 16, false, false>(const __grid_constant__ FillArgs);
 // Stage-2 partitions (global mode with matching), variant 1's geometry

@@ -21,7 +21,7 @@ PAPER = (1, -3, 3, 2)
 # (variant, alpha, compute warps) of sw_api.cu variant_for
 INT32 = [(0, 16, 4), (1, 16, 8), (2, 8, 8), (3, 16, 12), (4, 16, 14), (5, 16, 15), (6, 16, 16), (7, 16, 8)]
 PACKED = [(0, 16, 4), (1, 16, 8), (3, 16, 12), (5, 16, 15), (6, 16, 16), (8, 32, 4), (9, 32, 4), (10, 32, 8),
-          (11, 32, 16), (12, 32, 4), (13, 30, 4)]
+          (11, 32, 16), (12, 32, 4), (13, 30, 4), (14, 34, 8)]
 
 
 @pytest.fixture(scope="module")

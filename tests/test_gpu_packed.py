@@ -10,7 +10,7 @@ import synth
 
 pytestmark = pytest.mark.gpu
 PAPER = (1, -3, 3, 2)
-PACKED_VARIANTS = [0, 1, 3, 5, 6, 8, 9, 10, 11, 12, 13]
+PACKED_VARIANTS = [0, 1, 3, 5, 6, 8, 9, 10, 11, 12, 13, 14]
 # alpha 16: 4, 12, 15 warps + I/O warp, 16 warps with cooperative I/O;
 # alpha 32 (16 slots per lane): 4 warps + I/O warp, 4 cooperative, 8 + I/O warp, 16 cooperative, 4 + I/O split F chain
 
@@ -55,14 +55,14 @@ def check(ctx, A, B, scoring, k, variant, stripes=1, expect_packed=True):
 @pytest.mark.parametrize("m,n", [(1, 1), (17, 1), (16, 300), (1000, 999), (3000, 64), (5000, 2049)])
 def test_packed_shapes(ctx, variant, m, n):
     A, B = synth.random_pair(m + 3 * n + variant, m, n, plant_len=min(m, n) // 2, s=0.05, g=0.01)
-    check(ctx, A, B, PAPER, 32, variant)
+    check(ctx, A, B, PAPER, 34 if variant == 14 else 32, variant)
 
 
 @pytest.mark.parametrize("variant", PACKED_VARIANTS)
 def test_packed_scorings(ctx, variant):
     A, B = synth.random_pair(5 + variant, 2500, 1700, plant_len=1500, s=0.06, g=0.01)
     for scoring in (PAPER, (2, -1, 4, 1), (1, -1, 0, 2), (5, -4, 10, 1), (3, -2, 0, 1)):
-        check(ctx, A, B, scoring, 32, variant)
+        check(ctx, A, B, scoring, 34 if variant == 14 else 32, variant)
     check(ctx, A, B, PAPER, 0, variant)
 
 
@@ -72,11 +72,11 @@ def test_packed_falls_back_when_not_applicable(ctx):
     check(ctx, A, B, PAPER, 7, 12, expect_packed=False)  # the split-F geometry keeps strip-bottom rows only
 
 
-ALPHA = {0: 16, 1: 16, 3: 16, 5: 16, 6: 16, 8: 32, 9: 32, 10: 32, 11: 32, 12: 32, 13: 30}
-GEN = {0, 1, 8, 10, 13}  # geometries with the generic special-row instantiation
+ALPHA = {0: 16, 1: 16, 3: 16, 5: 16, 6: 16, 8: 32, 9: 32, 10: 32, 11: 32, 12: 32, 13: 30, 14: 34}
+GEN = {0, 1, 8, 10, 13, 14}  # geometries with the generic special-row instantiation
 
 
-@pytest.mark.parametrize("variant", [0, 1, 5, 8, 10, 13])
+@pytest.mark.parametrize("variant", [0, 1, 5, 8, 10, 13, 14])
 @pytest.mark.parametrize("k", [7, 16, 33, 100, 1000, 4097])
 def test_packed_any_special_row_interval(ctx, variant, k):
     """Special rows that are not strip bottoms (k >= alpha, not a multiple of
@@ -85,6 +85,24 @@ def test_packed_any_special_row_interval(ctx, variant, k):
     alpha (several rows per lane) runs the int32 kernel."""
     A, B = synth.random_pair(30 + variant + k, 9000, 1300, plant_len=1000, s=0.05, g=0.01)
     check(ctx, A, B, PAPER, k, variant, expect_packed=k % ALPHA[variant] == 0 or (k >= ALPHA[variant] and variant in GEN))
+
+
+@pytest.mark.parametrize("variant", [0, 10, 13, 14])
+def test_packed_staged_special_rows_every_slot(ctx, variant):
+    """k >= 32 alpha: one lane per warp holds a special row, which the GEN
+    kernel stages in shared memory with its slot as a compile-time constant
+    (SPM 3, sw_fill16.cuh tile_gen); k = 32 alpha + d walks the row through
+    every slot and both halves of the strip over the matrix, several bands per
+    CTA (sw_set_grid 2).  Every special row against the oracle."""
+    al = ALPHA[variant]
+    for d in (1, al // 2 + 1):
+        k = 32 * al + d
+        A, B = synth.random_pair(700 + variant + d, 2 * al * k + 77, 530, plant_len=2000, s=0.05, g=0.01)
+        ctx.set_grid(2)
+        try:
+            check(ctx, A, B, PAPER, k, variant, expect_packed=True)
+        finally:
+            ctx.set_grid(0)
 
 
 def test_packed_ties_and_long_alignment(ctx):
