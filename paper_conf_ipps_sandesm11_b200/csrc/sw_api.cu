@@ -355,7 +355,7 @@ struct sw_ctx {
     std::vector<cudaEvent_t> ev_row;  // one per staging slot: the slot's final copy is done
     int nstage = 2;
     DevBuf seq, a2, b2, misc, slots, dbg;
-    DevBuf mm_parts, mm_scratch, mm_res, mm_codes, mm_moves, mm_err;  // Stages 3-5
+    DevBuf mm_parts, mm_scratch, mm_res, mm_codes, mm_moves, mm_err, mm_cnt;  // Stages 3-5
     DevBuf capbuf;  // Stage 2: (t, E) of every DP row at the special row's column
     DevBuf rowb[MAX_STRIPES], progress[MAX_STRIPES], sp[MAX_STRIPES];
     HostBuf flags[MAX_STRIPES];  // mapped pinned row_done flags per stripe
@@ -610,7 +610,7 @@ extern "C" void sw_shutdown(sw_ctx *ctx)
     if (ctx->side) cudaStreamSynchronize(ctx->side);
     if (ctx->aux) cudaStreamSynchronize(ctx->aux);
     for (DevBuf *b : {&ctx->seq, &ctx->a2, &ctx->b2, &ctx->misc, &ctx->slots, &ctx->dbg, &ctx->capbuf, &ctx->mm_parts,
-                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves, &ctx->mm_err, &ctx->s2row})
+                      &ctx->mm_scratch, &ctx->mm_res, &ctx->mm_codes, &ctx->mm_moves, &ctx->mm_err, &ctx->mm_cnt, &ctx->s2row})
         if (b->p) cudaFree(b->p);
     for (int s = 0; s < MAX_STRIPES; s++) {
         cudaSetDevice(ctx->unit_dev[s] >= 0 ? ctx->unit_dev[s] : ctx->device);  // a unit's buffers live on its entry's device
@@ -2443,7 +2443,7 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
                 if (cta != (pass == 0)) continue;
                 MMPart c = P;
                 c.off = scr;
-                scr += (cta ? (MM_NWP + 3) : 3) * (Wd + 1);
+                scr += (cta ? (2 * (MM_NWP + 1) + 2) : 3) * (Wd + 1);  // CTA: two lines + a ring per pass
                 bp.push_back(c);
                 order.push_back(q);
                 ncta += cta;
@@ -2454,10 +2454,13 @@ static int align_common(sw_ctx *ctx, const unsigned char *dA, int64_t m, const u
         CK(cudaMemcpyAsync(ctx->mm_parts.p, bp.data(), bp.size() * sizeof(MMPart), cudaMemcpyHostToDevice, st));
         g.scratch = (int2 *)ctx->mm_scratch.p;
         if (ncta > 0) {
+            if ((rc = grow(ctx, ctx->mm_cnt, (size_t)ncta * sizeof(int)))) return rc;
+            CK(cudaMemsetAsync(ctx->mm_cnt.p, 0, (size_t)ncta * sizeof(int), st));
+            g.cnt = (int *)ctx->mm_cnt.p;
             g.nparts = ncta;
             g.parts = (const MMPart *)ctx->mm_parts.p;
             g.res = (MMRes *)ctx->mm_res.p;
-            sw_mm_split_cta_kernel<<<ncta, 32 * MM_NWP, 0, st>>>(g);
+            sw_mm_split_cta_kernel<<<2 * ncta, 32 * MM_NWP, 0, st>>>(g);  // forward and reverse pass CTAs
             CK(cudaGetLastError());
             ctx->stats.kernel_launches++;
         }

@@ -27,6 +27,7 @@
 // lane 31 writes the chunk's bottom row back in place).  All int32; the
 // global recurrence has no 0 term.
 #pragma once
+#include <type_traits>
 #include "sw_fill.cuh"
 
 namespace swb {
@@ -63,6 +64,7 @@ struct MMArgs {
     char *moves;
     int *nmoves;
     int *err;            // set to 2 when a spin-wait times out (watchdog)
+    int *cnt;            // CTA split kernel: passes finished per partition (zeroed per launch)
     long long timeout_ns;
 };
 
@@ -133,18 +135,30 @@ __device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, 
     int2 cur = (1 + lane <= w) ? __ldcg(rin + 1 + lane) : make_int2(NEG, NEG);
     int2 nxt = (33 + lane <= w) ? __ldcg(rin + 33 + lane) : make_int2(NEG, NEG);
     const int nsteps = w + 31;
-    auto step = [&](int k, bool guard) {
+    // column b's code (pad: never a match / the PADPROF byte), loaded one step
+    // ahead so the byte load is off the step's dependency chain
+    auto col_code = [&](int b) -> uint32_t {
+        return (b >= 1 && b <= w) ? mm_code(__ldg(P.cs + (long long)b * P.cstep)) : (WIDE ? 6u : 4u);
+    };
+    uint32_t ccode = col_code(1 - lane);
+    // GUARD (compile time): some lane is outside columns 1..w; those lanes compute
+    // and discard (no early return: the warp stays converged for the shuffles)
+    auto step = [&](int k, auto guard_c) {
+        constexpr bool GUARD = decltype(guard_c)::value;
         int tu = __shfl_up_sync(0xffffffffu, tu_out, 1);
         int fu = __shfl_up_sync(0xffffffffu, fu_out, 1);
         const int rH = __shfl_sync(0xffffffffu, cur.x, k & 31);
         const int rF = __shfl_sync(0xffffffffu, cur.y, k & 31);
         if (lane == 0) { tu = rH - gf; fu = rF; }
         const int b = k - lane + 1;
-        if (guard && (b < 1 || b > w)) return;
-        const uint32_t sel = WIDE ? mm_code(P.cs[(long long)b * P.cstep]) : col_sel(mm_code(P.cs[(long long)b * P.cstep]));
+        const bool ok = !GUARD || (b >= 1 && b <= w);
+        const uint32_t code = ccode;
+        ccode = col_code(b + 1);
+        const uint32_t sel = WIDE ? code : code * 0x1111u + 0x8880u;  // col_sel(code)
         int td = tdiag;
-        tdiag = tu;
-        unsigned int code = 0;
+        const int tu_in = tu;  // t(r0, b): the next step's diagonal
+        int Tn[MM_ALPHA], En[MM_ALPHA];
+        unsigned int tb = 0;
         int capH = 0, capF = 0;
 #pragma unroll
         for (int r = 0; r < MM_ALPHA; r++) {
@@ -155,20 +169,28 @@ __device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, 
             if (MODE == 1) {
                 const unsigned int src = (x >= e && x >= f) ? 0u : (f >= e ? 1u : 2u);
                 const unsigned int ext = (E[r] + nge >= T[r] ? 4u : 0u) | (fu + nge >= tu ? 8u : 0u);
-                code |= (src | ext) << (4 * r);
+                tb |= (src | ext) << (4 * r);
             }
             if (CAPC && cap_lane && r0 + r + 1 == capR) { capH = hv; capF = f; }
             td = T[r];
-            T[r] = hv - gf;
-            E[r] = e;
-            tu = T[r];
+            Tn[r] = hv - gf;
+            En[r] = e;
+            tu = Tn[r];
             fu = f;
         }
-        tu_out = tu;
-        fu_out = fu;
-        if (MODE == 1 && r0 < h) codes[(long long)b * HW + r0 / 8] = code;
-        if (CAPC && cap_lane) cap[b] = make_int2(capH, capF);
-        if (lane == 31) rout[b] = make_int2(tu + gf, fu);
+        tdiag = ok ? tu_in : tdiag;
+#pragma unroll
+        for (int r = 0; r < MM_ALPHA; r++) {
+            T[r] = ok ? Tn[r] : T[r];
+            E[r] = ok ? En[r] : E[r];
+        }
+        if (ok) {
+            tu_out = tu;
+            fu_out = fu;
+            if (MODE == 1 && r0 < h) codes[(long long)b * HW + r0 / 8] = tb;
+            if (CAPC && cap_lane) cap[b] = make_int2(capH, capF);
+            if (lane == 31) rout[b] = make_int2(tu + gf, fu);
+        }
     };
     for (int kb = 0; kb < nsteps; kb += 32) {
         if (kb > 0) {
@@ -179,11 +201,11 @@ __device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, 
         }
         if (kb >= 32 && kb + 32 <= w) {
 #pragma unroll 4
-            for (int u = 0; u < 32; u++) step(kb + u, false);
+            for (int u = 0; u < 32; u++) step(kb + u, std::false_type{});
         } else {
             const int ke = min(kb + 32, nsteps);
 #pragma unroll 1
-            for (int k = kb; k < ke; k++) step(k, true);
+            for (int k = kb; k < ke; k++) step(k, std::true_type{});
         }
         publish(min(w, kb + 1));
     }
@@ -254,22 +276,25 @@ __device__ void mm_cta_pass(const MMArgs &g, const DpProb &P, int2 *ring, long l
     const int nchunks = (capR + MM_CHUNK - 1) / MM_CHUNK;
     for (int c = warp; c < nchunks; c += NWP) {
         const int in = c % R, out = (c + 1) % R;
-        if (lane == 0) {
-            s_cols[out] = 0;
-            __threadfence_block();
-            s_gen[out] = c;
-        }
+        if (lane == 0) s_cols[out] = 0;
+        __threadfence_block();
+        if (lane == 0) s_gen[out] = c;
         __syncwarp();
+        // every lane polls and the warp votes: the loop is warp-uniform, so the
+        // warp stays converged for the cell loop's shuffles (a lane-0 spin made
+        // ptxas route every step through its divergent-warp path)
         auto wait = [&](int need) {
             need = min(need, w);
-            if (lane == 0 && (s_gen[in] != c - 1 || s_cols[in] < need)) {
+            if (__any_sync(0xffffffffu, s_gen[in] != c - 1 || s_cols[in] < need)) {
                 const unsigned long long t0 = gtimer();
-                while (s_gen[in] != c - 1 || s_cols[in] < need) {
+                while (__any_sync(0xffffffffu, s_gen[in] != c - 1 || s_cols[in] < need)) {
                     __nanosleep(32);
-                    if (gtimer() - t0 > (unsigned long long)g.timeout_ns) { atomicExch(g.err, 2); break; }
+                    if (__any_sync(0xffffffffu, gtimer() - t0 > (unsigned long long)g.timeout_ns)) {
+                        if (lane == 0) atomicExch(g.err, 2);
+                        break;
+                    }
                 }
             }
-            __syncwarp();
             __threadfence_block();
         };
         auto publish = [&](int cols) {
@@ -286,16 +311,23 @@ __device__ void mm_cta_pass(const MMArgs &g, const DpProb &P, int2 *ring, long l
 }
 
 constexpr int MM_NWP = 8;  // warps per partition in the CTA split kernel
+// resident CTAs per SM the CTA split kernel is compiled for (2: 128 registers)
+#ifndef SWB_MM_MINB
+#define SWB_MM_MINB 2
+#endif
 
-// One CTA of MM_NWP warps per (large) partition: split it at the middle of
-// its larger dimension.  Same orientation, passes and junction rule as
+// Two CTAs of MM_NWP warps per (large) partition: CTA 2p runs the forward
+// pass from C_s, CTA 2p + 1 the reverse pass from C_e (independent, each with
+// its own ring), and the one that finishes second finds the junction on the
+// middle line.  Same orientation, passes and junction rule as
 // sw_mm_split_kernel.
-__global__ void __launch_bounds__(32 * MM_NWP) sw_mm_split_cta_kernel(const __grid_constant__ MMArgs g)
+__global__ void __launch_bounds__(32 * MM_NWP, SWB_MM_MINB) sw_mm_split_cta_kernel(const __grid_constant__ MMArgs g)
 {
     __shared__ int s_gen[MM_NWP + 1], s_cols[MM_NWP + 1];
     __shared__ unsigned long long s_key;
+    __shared__ int s_last;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int p = blockIdx.x;
+    const int p = blockIdx.x >> 1, pass = blockIdx.x & 1;
     if (p >= g.nparts) return;
     const MMPart Pt = g.parts[p];
     const bool tr = (Pt.j_e - Pt.j_s) > (Pt.i_e - Pt.i_s);
@@ -306,15 +338,26 @@ __global__ void __launch_bounds__(32 * MM_NWP) sw_mm_split_cta_kernel(const __gr
     const int ts = sw12(Pt.t_s), te = sw12(Pt.t_e);
     const int H = xe - xs, Wd = ye - ys, mid = H / 2;
     const long long rsz = Wd + 1;
-    int2 *ring = g.scratch + Pt.off;
-    int2 *capf = ring + (MM_NWP + 1) * rsz;
+    int2 *capf = g.scratch + Pt.off;
     int2 *capr = capf + rsz;
-    DpProb F{X + xs - 1, Y + ys - 1, 1, 1, mid, Wd, ts};
-    mm_cta_pass<MM_NWP>(g, F, ring, rsz, mid, capf, s_gen, s_cols, warp, lane);
-    DpProb R{X + xe, Y + ye, -1, -1, H - mid, Wd, te == 2 ? 3 : te == 1 ? 4 : 0};
-    mm_cta_pass<MM_NWP>(g, R, ring, rsz, H - mid, capr, s_gen, s_cols, warp, lane);
-    if (threadIdx.x == 0) s_key = 0ull;
+    int2 *ring = capr + rsz + pass * (MM_NWP + 1) * rsz;
+    if (pass == 0) {
+        DpProb F{X + xs - 1, Y + ys - 1, 1, 1, mid, Wd, ts};
+        mm_cta_pass<MM_NWP>(g, F, ring, rsz, mid, capf, s_gen, s_cols, warp, lane);
+    } else {
+        DpProb R{X + xe, Y + ye, -1, -1, H - mid, Wd, te == 2 ? 3 : te == 1 ? 4 : 0};
+        mm_cta_pass<MM_NWP>(g, R, ring, rsz, H - mid, capr, s_gen, s_cols, warp, lane);
+    }
+    // the last of the two passes finds the junction (threadfence-reduction order:
+    // this CTA's line is written and fenced before the counter)
+    if (threadIdx.x == 0) {
+        __threadfence();
+        s_last = atomicAdd(g.cnt + p, 1) == 1;
+        s_key = 0ull;
+    }
     __syncthreads();
+    if (!s_last) return;
+    __threadfence();
     long long key = -1;
     for (int b = threadIdx.x; b <= Wd; b += blockDim.x) {
         const int2 f = __ldcg(capf + b), r = __ldcg(capr + Wd - b);
