@@ -32,7 +32,11 @@
 
 namespace swb {
 
-constexpr int MM_ALPHA = 8;
+#ifndef SWB_MM_ALPHA
+#define SWB_MM_ALPHA 16
+#endif
+constexpr int MM_ALPHA = SWB_MM_ALPHA;  // rows per lane (a multiple of 8: one traceback word per 8 rows)
+static_assert(MM_ALPHA % 8 == 0, "MM_ALPHA rows per lane: whole 8-row traceback words");
 constexpr int MM_CHUNK = 32 * MM_ALPHA;
 constexpr long long MM_TB_CELLS = 1 << 16;  // Stage-5 partitions: at most this many cells
 
@@ -158,7 +162,7 @@ __device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, 
         int td = tdiag;
         const int tu_in = tu;  // t(r0, b): the next step's diagonal
         int Tn[MM_ALPHA], En[MM_ALPHA];
-        unsigned int tb = 0;
+        unsigned int tb[MM_ALPHA / 8] = {};
         int capH = 0, capF = 0;
 #pragma unroll
         for (int r = 0; r < MM_ALPHA; r++) {
@@ -169,7 +173,7 @@ __device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, 
             if (MODE == 1) {
                 const unsigned int src = (x >= e && x >= f) ? 0u : (f >= e ? 1u : 2u);
                 const unsigned int ext = (E[r] + nge >= T[r] ? 4u : 0u) | (fu + nge >= tu ? 8u : 0u);
-                tb |= (src | ext) << (4 * r);
+                tb[r / 8] |= (src | ext) << (4 * (r % 8));
             }
             if (CAPC && cap_lane && r0 + r + 1 == capR) { capH = hv; capF = f; }
             td = T[r];
@@ -187,7 +191,11 @@ __device__ __forceinline__ void mm_chunk_impl(const MMArgs &g, const DpProb &P, 
         if (ok) {
             tu_out = tu;
             fu_out = fu;
-            if (MODE == 1 && r0 < h) codes[(long long)b * HW + r0 / 8] = tb;
+            if (MODE == 1) {
+#pragma unroll
+                for (int q = 0; q < MM_ALPHA / 8; q++)
+                    if (r0 + 8 * q < h) codes[(long long)b * HW + r0 / 8 + q] = tb[q];
+            }
             if (CAPC && cap_lane) cap[b] = make_int2(capH, capF);
             if (lane == 31) rout[b] = make_int2(tu + gf, fu);
         }
