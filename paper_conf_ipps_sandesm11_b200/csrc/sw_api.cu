@@ -971,6 +971,9 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16, int
         const Candidate &C = cands[c];
         const Variant &V = variant_for(C.variant);
         if (C.packed && !packed_ok(V)) continue;
+        // alpha 34 (variant 14) is for band-cyclic fills on several GPUs (one wave
+        // of 8 x 148 CTAs on C4); on one GPU alpha 32 + the tail launch is faster
+        if (C.variant == 14 && gpus == 1) continue;
         if (!C.packed && !J.local) { best = c; break; }  // reverse pass: int32 only
         const void *fn = C.packed ? V.packed_fn : V.local_fn;
         if (!fn) continue;
@@ -986,7 +989,10 @@ static const Variant &choose_variant(sw_ctx *ctx, const Job &J, bool *use16, int
         // special rows that are not band bottoms are written by the compute
         // warps (SP1 tiles) instead of the I/O warp: measured +7.7 % on C2
         // (variant 8 at k = 3840 vs 4096, profiles/r01_fill_a30.txt)
-        if (J.k > 0 && J.k < J.m && J.k % bh != 0) t *= 1.077;
+        // (profiles/r02_spm3.txt: 1.099 at strip bottoms, 1.049 for one staged
+        // row per band, k >= bh; several generic rows per band run the
+        // per-slot select path: C3 at k = 4096 on alpha 34 was 5x slower)
+        if (J.k > 0 && J.k < J.m && J.k % bh != 0) t *= J.k % V.alpha == 0 ? 1.099 : J.k >= bh ? 1.049 : 4.0;
         if (t < best_t * 0.97) {
             best_t = t;
             best = c;

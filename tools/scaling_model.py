@@ -50,7 +50,7 @@ def special_factor(g, m, k):
     al, bh = GEOMS[g][0], GEOMS[g][1]
     if k <= 0 or k >= m or k % bh == 0:
         return 1.0
-    return 1.099 if k % al == 0 else 1.049
+    return 1.099 if k % al == 0 else 1.049 if k >= bh else 4.0
 
 
 def t_stripes(m, n, k, P, g):
