@@ -64,7 +64,7 @@ def test_device_count(mctx):
 
 
 @pytest.mark.parametrize("variant,packed,alpha,nw", [(1, True, 16, 8), (10, True, 32, 8), (13, True, 30, 4),
-                                                     (1, False, 16, 8), (0, False, 16, 4)])
+                                                     (14, True, 34, 8), (1, False, 16, 8), (0, False, 16, 4)])
 def test_cyclic_bands(mctx, variant, packed, alpha, nw):
     """Band-cyclic Stage 1: every entry runs bands, several per CTA at a small
     grid; special rows at strip bottoms (packed) or every row (int32)."""
@@ -75,6 +75,18 @@ def test_cyclic_bands(mctx, variant, packed, alpha, nw):
     k = alpha if packed else 1
     got, rows, st = run(mctx, A, B, PAPER, k, variant, packed, grid=1)
     assert st["devices"] == P and st["alpha"] == (-alpha if packed else alpha), st
+    compare(got, rows, A, B, PAPER, k)
+
+
+def test_cyclic_alpha34_staged_rows(mctx):
+    """The geometry band-cyclic C4 runs on several GPUs (alpha 34 x 8 warps)
+    with special rows that are neither strip nor band bottoms (k = band height
+    + 5: the band-uniform staged tiles of the GEN kernel), bands of every entry."""
+    P = mctx.device_count()
+    k = 8704 + 5
+    A, B = synth.random_pair(8200 + P, 3 * k + 111, 700, plant_len=1500, s=0.04, g=0.01)
+    got, rows, st = run(mctx, A, B, PAPER, k, 14, True, grid=1)
+    assert st["devices"] == P and st["alpha"] == -34, st
     compare(got, rows, A, B, PAPER, k)
 
 

@@ -105,6 +105,28 @@ def test_packed_staged_special_rows_every_slot(ctx, variant):
             ctx.set_grid(0)
 
 
+BAND_ROWS = {0: 2048, 8: 4096, 10: 8192, 13: 3840, 14: 8704}
+
+
+@pytest.mark.parametrize("variant", [0, 8, 10, 13, 14])
+def test_packed_band_staged_special_rows(ctx, variant):
+    """k >= the band height and not a multiple of alpha: a band holds at most
+    one special row, and every warp of that band runs the staged tiles of the
+    row's slot (band_sps, sw_fill16.cuh) while only the owning lane stores;
+    k = band height + d walks the row over slots, halves and warps, several
+    bands per CTA (sw_set_grid 2), the ragged last band included.  Every
+    special row against the oracle."""
+    al, bh = ALPHA[variant], BAND_ROWS[variant]
+    for d in (1, al // 2 + 3, 31 * al + al - 1):
+        k = bh + d
+        A, B = synth.random_pair(900 + variant + d, 5 * k + 333, 420, plant_len=3000, s=0.05, g=0.01)
+        ctx.set_grid(2)
+        try:
+            check(ctx, A, B, PAPER, k, variant, expect_packed=True)
+        finally:
+            ctx.set_grid(0)
+
+
 def test_packed_ties_and_long_alignment(ctx):
     X = synth.random_pair(3, 400, 1)[0]
     XXX = np.concatenate([X, X, X])
