@@ -153,7 +153,7 @@ def test_two_ranks_ipc_one_gpu():
 
 # ---------------------------------------------------------------- band-cyclic ranks, one GPU, CUDA IPC
 
-def _cyc_rank_main(rank, world, port, A, B, k, q):
+def _cyc_rank_main(rank, world, port, A, B, k, q, variant=1):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     import torch
@@ -166,7 +166,7 @@ def _cyc_rank_main(rank, world, port, A, B, k, q):
     try:
         torch.cuda.set_device(0)
         ctx = Context(0)
-        ctx.set_kernel(1, True)  # 4096-row bands: several per rank
+        ctx.set_kernel(variant, True)  # 4096-row (1) or 8704-row (14) bands: several per rank
         ctx.set_grid(2)          # the two processes time-share one GPU: keep their CTAs few
         dA = torch.from_numpy(A).cuda()
         dB = torch.from_numpy(B).cuda()
@@ -188,20 +188,21 @@ def _cyc_rank_main(rank, world, port, A, B, k, q):
         dist.destroy_process_group()
 
 
-def test_two_cyclic_ranks_ipc_one_gpu():
+@pytest.mark.parametrize("variant,bh,k", [(1, 4096, 512), (14, 8704, 8704 + 5)])
+def test_two_cyclic_ranks_ipc_one_gpu(variant, bh, k):
     """Band-cyclic ranks in two processes (CUDA IPC areas): every special row
     comes from exactly one rank, whole, bit-exact; the combined best is the
-    oracle's."""
+    oracle's.  Variant 14 (alpha 34, the geometry band-cyclic C4 runs on
+    several GPUs) with special rows inside the bands (the staged GEN tiles)."""
     import torch.multiprocessing as mp
 
-    A, B = synth.random_pair(12, 4 * 4096 + 1234, 1900, plant_len=1500, s=0.04, g=0.01)
-    k = 512
+    A, B = synth.random_pair(12 + variant, 4 * bh + 1234, 1900, plant_len=1500, s=0.04, g=0.01)
     world = 2
     port = 33000 + random.randint(0, 2000)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     os.environ["SWB_TIMEOUT_S"] = "60"
-    procs = [ctx.Process(target=_cyc_rank_main, args=(r, world, port, A, B, k, q)) for r in range(world)]
+    procs = [ctx.Process(target=_cyc_rank_main, args=(r, world, port, A, B, k, q, variant)) for r in range(world)]
     for p in procs:
         p.start()
     got = {}
